@@ -1,0 +1,336 @@
+#!/usr/bin/env python
+"""Benchmark: outer-product spGEMM C = A x A with the Block Reorganizer on B200.
+
+One *step* = one pass of the whole hot path over the workload: spgemm_plan (workload
+analysis + Block Reorganizer lists) + spgemm_execute (expansion, merge, C allocation and CSR
+compaction) + spgemm_destroy, through the C-ABI.  Inputs are resident in HBM when the timed
+region starts.  Metric (BASELINE.json): GFLOPS = 2 x intermediate products / s; the HBM
+roofline fraction of the dominant kernel and of the whole step are reported beside it.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+Multi-GPU: launched with torch.distributed.run, one rank per GPU, rows of C partitioned into
+balanced row blocks (strong scaling of one product); value = all products / max-over-ranks time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "spGEMM GFLOPS (2*intermediate products/s), C=AxA"
+UNIT = "GFLOPS"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks -------------------
+class ClockSampler:
+    """nvidia-smi samples during the timed region (sm clock, max clock, throttle reasons)."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ CPU oracle timing ------
+def time_oracle(inp, target_s: float, seed: int = 0):
+    """The oracle as it stands (fp64 Gustavson, OpenMP) on a bounded random row sample."""
+    import oracle
+    from oracle import stages
+    rowwork = stages.row_workload(inp)   # only to report products of the sample
+    rng = np.random.default_rng(seed)
+    perm = rng.permutation(inp.m).astype(np.int32)
+    cores = oracle.max_threads()
+    n = max(1, inp.m // 1000)
+    while True:
+        rows = np.sort(perm[:n])
+        t0 = time.perf_counter()
+        oracle.gustavson(inp, rows=rows)
+        dt = time.perf_counter() - t0
+        if dt >= target_s or n >= inp.m:
+            break
+        n = min(inp.m, int(n * min(8.0, max(1.5, 1.2 * target_s / max(dt, 1e-3)))))
+    prods = int(rowwork[rows].sum())
+    return {"value": 2.0 * prods / dt / 1e9, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{rows.size} random rows of {inp.m} ({prods} products, {dt:.1f} s)"}, dt
+
+
+# ------------------------------------------------------------------ helpers ----------------
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def flush_l2(buf):
+    buf.add_(1)  # write 512 MiB (> 126 MB L2) between timed steps
+
+
+def main():
+    args = parse()
+    ws, rank, local = dist_env()
+    import torch
+    if args.impl == "reference":
+        return run_reference(args, ws, rank)
+    import synth
+    import paper_conf_icde_leekyjkp20_b200 as spg
+    from paper_conf_icde_leekyjkp20_b200.build import build_library
+    if rank == 0:
+        build_library()
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.barrier()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    inp_full = synth.make_inputs(args.config, seed=args.seed)
+    A_full, B_full = spg.from_inputs(inp_full, dev)
+    if ws > 1:
+        bounds = spg.row_partition(A_full, B_full, ws)
+        inp = synth.row_slice_coo(inp_full, int(bounds[rank]), int(bounds[rank + 1]))
+        A, B = spg.from_inputs(inp, dev)
+    else:
+        inp, A, B = inp_full, A_full, B_full
+    stream = torch.cuda.current_stream(dev)
+    opts = dict(validate=0)
+    flush = torch.zeros(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def step():
+        with spg.Plan(A, B, stream=stream, **opts) as p:
+            C = p.execute()
+            return p, C
+
+    spg.set_timing(True)
+    for _ in range(max(args.warmup, 0)):
+        p, C = step()
+        del C
+    torch.cuda.synchronize()
+    st = None
+    # timed region
+    sampler = ClockSampler(local)
+    sampler.start()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    step_ms, kern = [], {}
+    launches = 0
+    nnz_c = 0
+    wall0 = time.perf_counter()
+    for _ in range(args.steps):
+        flush_l2(flush)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        p = spg.Plan(A, B, stream=stream, **opts)
+        C = p.execute()
+        st = p.stats()
+        p.destroy()
+        e1.record(stream)
+        e1.synchronize()
+        step_ms.append(e0.elapsed_time(e1))
+        tl = spg.last_timings()
+        launches += len(tl)
+        for nm, ms in tl:
+            kern.setdefault(nm, []).append(ms)
+        nnz_c = C.nnz
+        del C
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    wall = time.perf_counter() - wall0
+    clocks = sampler.stop()
+    total_ms = float(sum(step_ms))
+    products = st["nnz_chat"]
+    # max over ranks of the device time; total products over ranks
+    if ws > 1:
+        t = torch.tensor([total_ms, float(products), float(nnz_c), float(launches)], dtype=torch.float64, device=dev)
+        tmax = t.clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        tsum = t.clone()
+        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+        total_ms_all = float(tmax[0])
+        products_all = int(tsum[1])
+        nnz_c_all = int(tsum[2])
+        launches_all = int(tsum[3])
+    else:
+        total_ms_all, products_all, nnz_c_all, launches_all = total_ms, products, nnz_c, launches
+    ms_per_step = total_ms_all / args.steps
+    value = 2.0 * products_all / (ms_per_step / 1e3) / 1e9
+
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    peak_src = "measured" if "hbm_gbs" in peaks else "fallback"
+
+    # per-kernel shares; algorithmic bytes
+    k_ms = {nm: sum(v) / args.steps for nm, v in kern.items()}
+    nnz_a, nnz_b = inp.nnz_a, inp.nnz_b
+    bytes_step = 12 * nnz_a + 12 * nnz_b + 16 * (inp.m + 1 + inp.k + 1) // 2 + 16 * products + 12 * nnz_c + 8 * (inp.m + 1)
+    groups = {
+        "expand": (["expand_pieces", "expand_gathered"], 8 * products + 12 * nnz_a + 8 * nnz_b),
+        "merge": (["merge_pass", "merge_warp", "merge_warp_radix", "merge_cta_radix", "merge_limited"],
+                  8 * products + 8 * nnz_c + 16 * inp.m),
+        "compact": (["compact"], 16 * nnz_c + 8 * inp.m),
+    }
+    gms = {g: sum(k_ms.get(n, 0.0) for n in names) for g, (names, _) in groups.items()}
+    top = max(gms, key=lambda g: gms[g])
+    top_bytes = groups[top][1]
+    achieved = top_bytes / (gms[top] / 1e3) / 1e9 if gms[top] > 0 else 0.0
+    roofline = {"bound": "hbm", "kernel": top, "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
+                "frac": round(achieved / hbm, 4), "traffic": None, "peak_source": peak_src,
+                "ms": round(gms[top], 4), "algorithmic_bytes": int(top_bytes)}
+    step_bw = bytes_step / (ms_per_step / 1e3) / 1e9
+    breakdown = {nm: round(v, 4) for nm, v in sorted(k_ms.items(), key=lambda x: -x[1])}
+
+    out = {
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32 (fp64 merge accumulation)",
+        "data": "synthetic (seeded generator, synth/)",
+        "config": {"workload": f"{args.config}: " + synth.CONFIGS[args.config]["desc"], "m": inp_full.m,
+                   "nnz_a": inp_full.nnz_a, "products": products_all, "nnz_c": nnz_c_all,
+                   "parallelism": f"row-partition x{ws}" if ws > 1 else "single GPU",
+                   "l2": "flushed between steps (512 MiB write); Ĉ >> L2", "seed": args.seed,
+                   "step": "plan+execute+destroy via C-ABI, device-resident inputs"},
+        "roofline": roofline,
+        "step_roofline": {"achieved": round(step_bw, 1), "peak": hbm, "unit": "GB/s",
+                          "frac": round(step_bw / hbm, 4), "bytes": int(bytes_step),
+                          "def": "A + B + 2*Ĉ(8 B/product) + C, per step"},
+        "kernel_ms": breakdown,
+        "gpu_launches": launches_all,
+        "clocks": clocks,
+        "wall_s": round(wall, 3),
+    }
+    # e2e through the C-ABI with host buffers (H2D of A, B and D2H of C inside the timed region)
+    if not args.no_e2e:
+        Ah, Bh = spg.from_inputs(inp, "cpu")
+        h2d = sum(t.numel() * t.element_size() for t in (Ah.colptr, Ah.rowidx, Ah.val, Bh.rowptr, Bh.colidx, Bh.val))
+        es = []
+        d2h = 0
+        for it in range(1 + max(1, args.steps // 2)):
+            flush_l2(flush)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            with spg.Plan(Ah, Bh, stream=stream, **opts) as p:
+                Ch = p.execute(device="cpu")
+            torch.cuda.synchronize()
+            dt = time.perf_counter() - t0
+            d2h = sum(t.numel() * t.element_size() for t in (Ch.rowptr, Ch.colidx, Ch.val))
+            if it > 0:
+                es.append(dt)
+        e2e_t = sum(es) / len(es)
+        if ws > 1:
+            tt = torch.tensor([e2e_t], dtype=torch.float64, device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            e2e_t = float(tt[0])
+        out["e2e"] = {"value": round(2.0 * products_all / e2e_t / 1e9, 3), "unit": UNIT,
+                      "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+                      "ms_per_step": round(e2e_t * 1e3, 3)}
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        cb, _ = time_oracle(inp_full, target_s=10.0)
+        out["cpu_baseline"] = cb
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if ws > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def run_reference(args, ws, rank):
+    """--impl reference: the oracle (this tier's reference arm) on the host cores."""
+    if ws > 1 and rank != 0:
+        return
+    import synth
+    import oracle
+    inp = synth.make_inputs(args.config, seed=args.seed)
+    oracle.build()
+    for _ in range(max(args.warmup, 0)):
+        time_oracle(inp, target_s=1.0, seed=99)
+    vals = []
+    cbs = []
+    for s in range(args.steps):
+        cb, dt = time_oracle(inp, target_s=8.0, seed=s)
+        vals.append(cb["value"])
+        cbs.append(cb)
+    v = float(np.mean(vals))
+    cb = dict(cbs[-1])
+    cb["value"] = round(v, 4)
+    out = {"metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": ws, "steps": args.steps,
+           "warmup": args.warmup, "higher_is_better": True, "impl": "reference", "dtype": "f64",
+           "data": "synthetic (seeded generator, synth/)", "vs_baseline": None,
+           "config": {"workload": f"{args.config}: " + synth.CONFIGS[args.config]["desc"]},
+           "cpu_baseline": cb,
+           "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,110 @@
+// Common device helpers for the B200 (sm_100a) spGEMM library.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace spg {
+
+constexpr int kWarp = 32;
+constexpr int kNumSMs = 148;  // B200; the host queries the real count at plan time
+
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ int warp_id() { return threadIdx.x >> 5; }
+
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_incl_sum(T v) {
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        T o = __shfl_up_sync(0xffffffffu, v, d);
+        if (lane_id() >= d) v += o;
+    }
+    return v;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+    return v;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_min(T v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, d));
+    return v;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_max(T v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v = max(v, __shfl_xor_sync(0xffffffffu, v, d));
+    return v;
+}
+
+// Block-wide exclusive sum over THREADS threads; returns exclusive prefix, *total = sum.
+// `smem` needs THREADS/32 + 1 slots.  Contains __syncthreads (all threads must call).
+template <int THREADS, typename T>
+__device__ __forceinline__ T block_excl_sum(T v, T *smem, T *total) {
+    constexpr int NW = THREADS / 32;
+    T inc = warp_incl_sum(v);
+    if (lane_id() == 31) smem[warp_id()] = inc;
+    __syncthreads();
+    if (warp_id() == 0) {
+        T w = lane_id() < NW ? smem[lane_id()] : T(0);
+        T wi = warp_incl_sum(w);
+        if (lane_id() < NW) smem[lane_id()] = wi - w;
+        if (lane_id() == NW - 1) smem[NW] = wi;
+    }
+    __syncthreads();
+    T r = smem[warp_id()] + inc - v;
+    *total = smem[NW];
+    __syncthreads();
+    return r;
+}
+
+template <int THREADS, typename T>
+__device__ __forceinline__ T block_reduce_min(T v, T *smem) {
+    v = warp_min(v);
+    if (lane_id() == 0) smem[warp_id()] = v;
+    __syncthreads();
+    T r = smem[0];
+#pragma unroll
+    for (int w = 1; w < THREADS / 32; ++w) r = min(r, smem[w]);
+    __syncthreads();
+    return r;
+}
+
+template <int THREADS, typename T>
+__device__ __forceinline__ T block_reduce_max(T v, T *smem) {
+    v = warp_max(v);
+    if (lane_id() == 0) smem[warp_id()] = v;
+    __syncthreads();
+    T r = smem[0];
+#pragma unroll
+    for (int w = 1; w < THREADS / 32; ++w) r = max(r, smem[w]);
+    __syncthreads();
+    return r;
+}
+
+// Largest index i in [lo, hi) with ptr[i] <= x (ptr non-decreasing, ptr[lo] <= x).
+__device__ __forceinline__ int64_t upper_bound_idx(const int64_t *__restrict__ ptr, int64_t lo, int64_t hi,
+                                                   int64_t x) {
+    // returns last i with ptr[i] <= x, searching i in [lo, hi)
+    while (hi - lo > 1) {
+        int64_t mid = (lo + hi) >> 1;
+        if (__ldg(ptr + mid) <= x) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+__device__ __forceinline__ int ilog2_floor(uint64_t x) { return 63 - __clzll((long long)x); }
+__device__ __forceinline__ int ilog2_ceil(uint64_t x) { return x <= 1 ? 0 : 64 - __clzll((long long)(x - 1)); }
+
+}  // namespace spg

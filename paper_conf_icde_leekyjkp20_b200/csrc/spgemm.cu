@@ -1,0 +1,795 @@
+// C-ABI implementation (include/spgemm.h).  Host orchestration of the four stages; all
+// arithmetic of the path runs in the kernels of analysis.cuh / expand.cuh / merge.cuh.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/spgemm.h"
+#include "analysis.cuh"
+#include "expand.cuh"
+#include "merge.cuh"
+#include "scan.cuh"
+
+using namespace spg;
+
+// ------------------------------------------------------------------ errors ---------------
+static thread_local std::string g_err;
+
+static int fail(int code, const std::string &msg) {
+    g_err = msg;
+    return code;
+}
+
+#define CK(call)                                                                                 \
+    do {                                                                                         \
+        cudaError_t _e = (call);                                                                 \
+        if (_e != cudaSuccess) {                                                                 \
+            return fail(_e == cudaErrorMemoryAllocation ? SPGEMM_ERR_OUT_OF_MEMORY : SPGEMM_ERR_CUDA, \
+                        std::string(#call) + ": " + cudaGetErrorString(_e));                     \
+        }                                                                                        \
+    } while (0)
+
+#define TRY(call)                      \
+    do {                               \
+        int _r = (call);               \
+        if (_r != SPGEMM_OK) return _r; \
+    } while (0)
+
+// ------------------------------------------------------------------ timing ---------------
+struct TimerRec {
+    const char *name;
+    cudaEvent_t a, b;
+};
+static thread_local bool g_timing = false;
+static thread_local std::vector<TimerRec> g_timers;
+static thread_local std::vector<cudaEvent_t> g_event_pool;
+static thread_local size_t g_events_used = 0;
+
+static cudaEvent_t next_event() {
+    if (g_events_used == g_event_pool.size()) {
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        g_event_pool.push_back(e);
+    }
+    return g_event_pool[g_events_used++];
+}
+
+static void timers_reset() {
+    g_timers.clear();
+    g_events_used = 0;
+}
+
+struct TimedLaunch {
+    cudaStream_t s;
+    const char *name;
+    cudaEvent_t b = nullptr;
+    TimedLaunch(const char *n, cudaStream_t st) : s(st), name(n) {
+        if (g_timing) {
+            cudaEvent_t a = next_event();
+            b = next_event();
+            cudaEventRecord(a, s);
+            g_timers.push_back({name, a, b});
+        }
+    }
+    ~TimedLaunch() {
+        if (g_timing) cudaEventRecord(b, s);
+    }
+};
+
+#define LAUNCH(name, stream, ...)                      \
+    do {                                               \
+        {                                              \
+            TimedLaunch _tl(name, stream);             \
+            __VA_ARGS__;                               \
+        }                                              \
+        CK(cudaGetLastError());                        \
+    } while (0)
+
+// ------------------------------------------------------------------ memory ---------------
+static cudaMemPool_t pool_for_device(int dev) {
+    static cudaMemPool_t pools[64] = {};
+    if (!pools[dev]) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.handleTypes = cudaMemHandleTypeNone;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t p;
+        if (cudaMemPoolCreate(&p, &props) != cudaSuccess) return nullptr;
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[dev] = p;
+    }
+    return pools[dev];
+}
+
+struct spgemm_plan_s {
+    int dev = 0;
+    int num_sms = kNumSMs;
+    cudaMemPool_t pool = nullptr;
+    cudaStream_t last_stream = nullptr;
+    spgemm_options_t opt{};
+    int64_t m = 0, k = 0, n = 0, nnz_a = 0, nnz_b = 0;
+    const int64_t *a_colptr = nullptr;
+    const int32_t *a_rowidx = nullptr;
+    const float *a_val = nullptr;
+    const int64_t *b_rowptr = nullptr;
+    const int32_t *b_colidx = nullptr;
+    const float *b_val = nullptr;
+    std::vector<void *> owned;
+    int64_t bytes = 0;
+    // stage 1
+    int64_t *work = nullptr, *rowwork = nullptr, *rowoff = nullptr, *base = nullptr;
+    int32_t *deg = nullptr;
+    PlanScalars *scal = nullptr;
+    PlanScalars h_scal{};
+    int64_t nnz_chat = 0, nnz_chat_rowwise = 0, t_dom = 0, t_lim = 0;
+    // stage 2
+    int8_t *pair_cls = nullptr, *row_cls = nullptr;
+    int32_t *pair_order = nullptr, *row_order = nullptr;
+    int64_t pair_starts[kNumPairBuckets + 1] = {};
+    int64_t row_starts[kNumRowBuckets + 1] = {};
+    Piece *pieces = nullptr;
+    int64_t n_split_pieces = 0, n_whole = 0;
+    int64_t *piece_off = nullptr;
+    int64_t lim_runs = 0, lim_max_deg = 0, lim_max_L = 0, nlim = 0;
+    int64_t *run_start = nullptr, *run_base = nullptr;
+    int32_t *run_len = nullptr, *lim_index = nullptr, *run_fill = nullptr;
+    int32_t *scr_cursor = nullptr, *scr_col = nullptr;
+    float *scr_val = nullptr;
+    int64_t stage_cap = 0;
+    int lim_grid = 0;
+    unsigned long long *row_counter = nullptr;
+    // stage 3/4
+    int32_t *chat_col = nullptr;
+    float *chat_val = nullptr;
+    int64_t *ccount = nullptr, *crowptr = nullptr;
+    int64_t nnz_c = -1;
+    int state = 0;  // 1 planned, 2 expanded, 3 merged
+};
+
+template <typename T>
+static int palloc(spgemm_plan_s *p, T **ptr, int64_t count, cudaStream_t s) {
+    size_t bytes = (size_t)std::max<int64_t>(count, 1) * sizeof(T);
+    void *v = nullptr;
+    cudaError_t e = p->pool ? cudaMallocFromPoolAsync(&v, bytes, p->pool, s) : cudaMallocAsync(&v, bytes, s);
+    if (e != cudaSuccess)
+        return fail(SPGEMM_ERR_OUT_OF_MEMORY, std::string("device allocation of ") + std::to_string(bytes) +
+                                                  " bytes failed: " + cudaGetErrorString(e));
+    p->owned.push_back(v);
+    p->bytes += (int64_t)bytes;
+    *ptr = (T *)v;
+    return SPGEMM_OK;
+}
+
+// temporary allocation freed at the end of the caller's scope (stream-ordered)
+struct Temp {
+    void *v = nullptr;
+    cudaStream_t s;
+    explicit Temp(cudaStream_t st) : s(st) {}
+    ~Temp() {
+        if (v) cudaFreeAsync(v, s);
+    }
+};
+
+template <typename T>
+static int talloc(spgemm_plan_s *p, Temp &t, T **ptr, int64_t count) {
+    size_t bytes = (size_t)std::max<int64_t>(count, 1) * sizeof(T);
+    cudaError_t e = p->pool ? cudaMallocFromPoolAsync(&t.v, bytes, p->pool, t.s) : cudaMallocAsync(&t.v, bytes, t.s);
+    if (e != cudaSuccess) return fail(SPGEMM_ERR_OUT_OF_MEMORY, "temporary device allocation failed");
+    *ptr = (T *)t.v;
+    return SPGEMM_OK;
+}
+
+static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+static inline unsigned grid_for(int64_t n, int threads, int64_t cap = 148 * 64) {
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(n, threads), cap));
+}
+
+// ------------------------------------------------------------------ primitives -----------
+template <typename Tin>
+static int scan_excl(spgemm_plan_s *p, const Tin *in, int64_t n, int64_t *out, cudaStream_t s, const char *name) {
+    if (n == 0) {
+        CK(cudaMemsetAsync(out, 0, sizeof(int64_t), s));
+        return SPGEMM_OK;
+    }
+    const int64_t ntiles = cdiv(n, kScanTile);
+    Temp t(s);
+    int64_t *ts;
+    TRY(talloc(p, t, &ts, ntiles + 1));
+    LAUNCH(name, s, k_scan_tile_sums<Tin><<<(unsigned)ntiles, kScanThreads, 0, s>>>(in, n, ts));
+    LAUNCH(name, s, k_scan_spine<<<1, 1024, 0, s>>>(ts, ntiles));
+    LAUNCH(name, s, k_scan_apply<Tin><<<(unsigned)ntiles, kScanThreads, 0, s>>>(in, n, ts, out, ntiles));
+    return SPGEMM_OK;
+}
+
+// stable partition of [0, n) by bucket id; writes out_idx[n] and bucket starts (host) [nb+1]
+static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb, int32_t *out_idx,
+                     int64_t *d_starts, cudaStream_t s, const char *name) {
+    if (n == 0) {
+        CK(cudaMemsetAsync(d_starts, 0, sizeof(int64_t) * (nb + 1), s));
+        return SPGEMM_OK;
+    }
+    const int64_t ntiles = cdiv(n, kPartThreads);
+    Temp t1(s), t2(s);
+    int32_t *counts;
+    int64_t *offs;
+    TRY(talloc(p, t1, &counts, (int64_t)nb * ntiles));
+    TRY(talloc(p, t2, &offs, (int64_t)nb * ntiles + 1));
+    LAUNCH(name, s, k_part_count<<<(unsigned)ntiles, kPartThreads, 0, s>>>(bucket, n, nb, counts, ntiles));
+    TRY(scan_excl(p, counts, (int64_t)nb * ntiles, offs, s, name));
+    LAUNCH(name, s, k_part_scatter<<<(unsigned)ntiles, kPartThreads, 0, s>>>(bucket, n, nb, offs, ntiles, out_idx));
+    LAUNCH(name, s, k_bucket_starts<<<(unsigned)cdiv(nb + 1, 128), 128, 0, s>>>(offs, nb, ntiles, d_starts));
+    return SPGEMM_OK;
+}
+
+// ------------------------------------------------------------------ ABI ------------------
+extern "C" {
+
+int spgemm_abi_version(void) { return SPGEMM_ABI_VERSION; }
+
+const char *spgemm_last_error(void) { return g_err.c_str(); }
+
+void spgemm_default_options(spgemm_options_t *o) {
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->alpha = 0.0;
+    o->dom_waves = 16;
+    o->dom_min_work = 32768;
+    o->split_ca_max = 256;
+    o->piece_work = 16384;
+    o->split_b_tile = 4096;
+    o->beta = 0.0;
+    o->limit_ctas_per_sm = 1;
+    o->enable_split = 1;
+    o->enable_gather = 1;
+    o->enable_limit = 1;
+    o->validate = 1;
+}
+
+int spgemm_set_timing(int32_t enable) {
+    g_timing = enable != 0;
+    return SPGEMM_OK;
+}
+
+int spgemm_last_timings(const char **names, float *ms, int32_t capacity, int32_t *count) {
+    if (!count) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "count is NULL");
+    *count = (int32_t)g_timers.size();
+    for (size_t q = 0; q < g_timers.size() && (int32_t)q < capacity; ++q) {
+        cudaEventSynchronize(g_timers[q].b);
+        float t = 0.f;
+        cudaEventElapsedTime(&t, g_timers[q].a, g_timers[q].b);
+        if (names) names[q] = g_timers[q].name;
+        if (ms) ms[q] = t;
+    }
+    return SPGEMM_OK;
+}
+
+static int check_csx(int64_t nseg, int64_t other, int64_t nnz, const void *ptr, const void *idx, const void *val,
+                     int32_t where, const char *what) {
+    if (!ptr || (nnz > 0 && (!idx || !val)))
+        return fail(SPGEMM_ERR_INVALID_ARGUMENT, std::string(what) + ": NULL array");
+    if (nseg < 0 || other < 0 || nnz < 0 || nseg >= (1ll << 31) || other >= (1ll << 31))
+        return fail(SPGEMM_ERR_INVALID_ARGUMENT, std::string(what) + ": bad dimensions");
+    if (where != SPGEMM_DEVICE && where != SPGEMM_HOST)
+        return fail(SPGEMM_ERR_INVALID_ARGUMENT, std::string(what) + ": bad `where`");
+    return SPGEMM_OK;
+}
+
+static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t *B, cudaStream_t s);
+
+int spgemm_plan(const spgemm_csc_t *A, const spgemm_csr_t *B, const spgemm_options_t *opt, void *stream,
+                spgemm_plan_t *out) {
+    if (!out) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan out-pointer is NULL");
+    *out = nullptr;
+    if (!A || !B) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "A or B is NULL");
+    TRY(check_csx(A->ncols, A->nrows, A->nnz, A->colptr, A->rowidx, A->val, A->where, "A"));
+    TRY(check_csx(B->nrows, B->ncols, B->nnz, B->rowptr, B->colidx, B->val, B->where, "B"));
+    if (A->ncols != B->nrows) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "A.ncols != B.nrows");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(SPGEMM_ERR_NO_DEVICE, "no CUDA device");
+    spgemm_plan_s *p = new spgemm_plan_s();
+    if (opt) p->opt = *opt; else spgemm_default_options(&p->opt);
+    spgemm_options_t d;
+    spgemm_default_options(&d);
+    if (p->opt.dom_waves <= 0) p->opt.dom_waves = d.dom_waves;
+    if (p->opt.dom_min_work <= 0) p->opt.dom_min_work = d.dom_min_work;
+    if (p->opt.split_ca_max <= 0) p->opt.split_ca_max = d.split_ca_max;
+    if (p->opt.piece_work <= 0) p->opt.piece_work = d.piece_work;
+    if (p->opt.split_b_tile <= 0) p->opt.split_b_tile = d.split_b_tile;
+    if (p->opt.limit_ctas_per_sm <= 0) p->opt.limit_ctas_per_sm = d.limit_ctas_per_sm;
+    int r = plan_impl(p, A, B, (cudaStream_t)stream);
+    if (r != SPGEMM_OK) {
+        std::string keep = g_err;
+        spgemm_destroy(p);
+        g_err = keep;
+        return r;
+    }
+    *out = p;
+    return SPGEMM_OK;
+}
+
+static int upload(spgemm_plan_s *p, const void *src, int64_t bytes, int32_t where, const void **dst, cudaStream_t s) {
+    if (where == SPGEMM_DEVICE) {
+        *dst = src;
+        return SPGEMM_OK;
+    }
+    unsigned char *d;
+    TRY(palloc(p, &d, std::max<int64_t>(bytes, 1), s));
+    if (bytes > 0) CK(cudaMemcpyAsync(d, src, (size_t)bytes, cudaMemcpyHostToDevice, s));
+    *dst = d;
+    return SPGEMM_OK;
+}
+
+static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t *B, cudaStream_t s) {
+    CK(cudaGetDevice(&p->dev));
+    CK(cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, p->dev));
+    p->pool = pool_for_device(p->dev);
+    p->last_stream = s;
+    timers_reset();
+    p->m = A->nrows;
+    p->k = A->ncols;
+    p->n = B->ncols;
+    p->nnz_a = A->nnz;
+    p->nnz_b = B->nnz;
+    const int64_t M = p->m, K = p->k;
+    TRY(upload(p, A->colptr, (K + 1) * 8, A->where, (const void **)&p->a_colptr, s));
+    TRY(upload(p, A->rowidx, p->nnz_a * 4, A->where, (const void **)&p->a_rowidx, s));
+    TRY(upload(p, A->val, p->nnz_a * 4, A->where, (const void **)&p->a_val, s));
+    TRY(upload(p, B->rowptr, (K + 1) * 8, B->where, (const void **)&p->b_rowptr, s));
+    TRY(upload(p, B->colidx, p->nnz_b * 4, B->where, (const void **)&p->b_colidx, s));
+    TRY(upload(p, B->val, p->nnz_b * 4, B->where, (const void **)&p->b_val, s));
+
+    TRY(palloc(p, &p->scal, 1, s));
+    CK(cudaMemsetAsync(p->scal, 0, sizeof(PlanScalars), s));
+    if (p->opt.validate) {
+        int *flag = &p->scal->invalid;
+        LAUNCH("validate", s, k_validate_ptr<<<grid_for(K + 1, 256, 1 << 30), 256, 0, s>>>(p->a_colptr, K, p->nnz_a, flag, 1));
+        LAUNCH("validate", s, k_validate_ptr<<<grid_for(K + 1, 256, 1 << 30), 256, 0, s>>>(p->b_rowptr, K, p->nnz_b, flag, 2));
+        PlanScalars hs;
+        CK(cudaMemcpyAsync(&hs, p->scal, sizeof(hs), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hs.invalid) return fail(SPGEMM_ERR_INVALID_INPUT, "malformed colptr of A or rowptr of B");
+        if (p->nnz_a > 0)
+            LAUNCH("validate", s, k_validate_idx<<<grid_for(cdiv(p->nnz_a, 8), 256, 1 << 30), 256, 0, s>>>(
+                p->a_colptr, p->a_rowidx, K, p->nnz_a, M, flag, 4));
+        if (p->nnz_b > 0)
+            LAUNCH("validate", s, k_validate_idx<<<grid_for(cdiv(p->nnz_b, 8), 256, 1 << 30), 256, 0, s>>>(
+                p->b_rowptr, p->b_colidx, K, p->nnz_b, p->n, flag, 8));
+    }
+
+    // ---- stage (1): workload analysis -------------------------------------------------
+    TRY(palloc(p, &p->work, K, s));
+    TRY(palloc(p, &p->rowwork, M, s));
+    TRY(palloc(p, &p->rowoff, M + 1, s));
+    TRY(palloc(p, &p->deg, M, s));
+    TRY(palloc(p, &p->base, p->nnz_a, s));
+    if (M > 0) {
+        CK(cudaMemsetAsync(p->rowwork, 0, M * 8, s));
+        CK(cudaMemsetAsync(p->deg, 0, M * 4, s));
+    }
+    if (K > 0)
+        LAUNCH("pair_work", s, k_pair_work<<<grid_for(K, 256, p->num_sms * 8), 256, 0, s>>>(p->a_colptr, p->b_rowptr, K,
+                                                                                     p->work, p->scal));
+    if (p->nnz_a > 0)
+        LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg));
+    TRY(scan_excl(p, p->rowwork, M, p->rowoff, s, "row_offsets"));
+    if (M > 0)
+        LAUNCH("row_reduce", s, k_row_reduce<<<grid_for(M, 256, p->num_sms * 8), 256, 0, s>>>(p->rowwork, p->deg, M, p->scal));
+    if (p->nnz_a > 0) {
+        Temp tc(s);
+        unsigned long long *cursor;
+        TRY(talloc(p, tc, &cursor, M));
+        CK(cudaMemcpyAsync(cursor, p->rowoff, M * 8, cudaMemcpyDeviceToDevice, s));
+        LAUNCH("run_base", s, k_run_base<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, cursor, p->base));
+    }
+    CK(cudaMemcpyAsync(&p->h_scal, p->scal, sizeof(PlanScalars), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&p->nnz_chat_rowwise, p->rowoff + M, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));  // sync 1: nnz(Ĉ) both ways, #non-empty blocks
+    if (p->h_scal.invalid) return fail(SPGEMM_ERR_INVALID_INPUT, "malformed indices (range / order) in A or B");
+    p->nnz_chat = (int64_t)p->h_scal.nnz_chat;
+    if (p->nnz_chat != p->nnz_chat_rowwise)
+        return fail(SPGEMM_ERR_CUDA, "internal: block-wise and row-wise nnz(Ĉ) disagree");
+
+    // thresholds (host; R1, R2, R6)
+    const spgemm_options_t &o = p->opt;
+    if (o.alpha > 0)
+        p->t_dom = (int64_t)std::floor((double)p->nnz_chat / ((double)std::max<uint64_t>(p->h_scal.k_nonempty, 1) * o.alpha));
+    else
+        p->t_dom = std::max<int64_t>(o.dom_min_work, cdiv(p->nnz_chat, (int64_t)p->num_sms * o.dom_waves));
+    const int64_t cap = 4096;
+    if (o.beta > 0)
+        p->t_lim = std::min<int64_t>(cap, (int64_t)std::floor((double)p->nnz_chat /
+                                                             ((double)std::max<uint64_t>(p->h_scal.m_nonempty, 1) * o.beta)));
+    else
+        p->t_lim = cap;
+
+    // ---- stage (2): categorisation and reorganizer lists -------------------------------
+    TRY(palloc(p, &p->pair_cls, K, s));
+    TRY(palloc(p, &p->row_cls, M, s));
+    TRY(palloc(p, &p->pair_order, K, s));
+    TRY(palloc(p, &p->row_order, M, s));
+    TRY(palloc(p, &p->piece_off, K + 1, s));
+    int64_t *d_starts;
+    TRY(palloc(p, &d_starts, kNumPairBuckets + kNumRowBuckets + 4, s));
+    {
+        Temp tb(s), tr(s), tn(s);
+        uint8_t *pb, *rbk;
+        int64_t *npieces;
+        TRY(talloc(p, tb, &pb, K));
+        TRY(talloc(p, tr, &rbk, M));
+        TRY(talloc(p, tn, &npieces, K));
+        ClassifyParams cp{p->t_dom, o.split_ca_max, o.enable_split, o.enable_gather};
+        if (K > 0)
+            LAUNCH("pair_classify", s, k_pair_classify<<<grid_for(K, 256), 256, 0, s>>>(p->a_colptr, p->b_rowptr, p->work, K,
+                                                                                    cp, p->pair_cls, pb));
+        TRY(partition(p, pb, K, kNumPairBuckets, p->pair_order, d_starts, s, "pair_partition"));
+        if (M > 0)
+            LAUNCH("row_classify", s, k_row_classify<<<grid_for(M, 256), 256, 0, s>>>(p->rowwork, p->deg, M, p->t_lim,
+                                                                                  p->row_cls, rbk));
+        TRY(partition(p, rbk, M, kNumRowBuckets, p->row_order, d_starts + kNumPairBuckets + 1, s, "row_partition"));
+        CK(cudaMemcpyAsync(p->pair_starts, d_starts, sizeof(int64_t) * (kNumPairBuckets + 1), cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(p->row_starts, d_starts + kNumPairBuckets + 1, sizeof(int64_t) * (kNumRowBuckets + 1),
+                           cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));  // sync 2a: bin populations
+        // B-Splitting: piece counts of the dominators (ascending k), scan, fill
+        const int64_t ndom = p->pair_starts[kPairBucketSplit + 1] - p->pair_starts[kPairBucketSplit];
+        SplitParams sp{o.piece_work, o.split_b_tile, o.split_ca_max};
+        p->n_whole = p->pair_starts[kPairBucketPiece + 1] - p->pair_starts[kPairBucketPiece];
+        if (ndom > 0) {
+            const int32_t *dom = p->pair_order + p->pair_starts[kPairBucketSplit];
+            LAUNCH("piece_count", s, k_piece_count<<<grid_for(ndom, 128), 128, 0, s>>>(dom, ndom, p->a_colptr, p->b_rowptr,
+                                                                                   sp, npieces));
+            TRY(scan_excl(p, npieces, ndom, p->piece_off, s, "piece_scan"));
+            CK(cudaMemcpyAsync(&p->n_split_pieces, p->piece_off + ndom, 8, cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));  // sync 2b: #pieces
+        }
+        TRY(palloc(p, &p->pieces, p->n_split_pieces + p->n_whole, s));
+        if (ndom > 0) {
+            const int32_t *dom = p->pair_order + p->pair_starts[kPairBucketSplit];
+            LAUNCH("piece_fill", s, k_piece_fill<<<(unsigned)cdiv(ndom * 32, 256), 256, 0, s>>>(
+                dom, ndom, p->a_colptr, p->b_rowptr, sp, p->piece_off, p->pieces));
+        }
+        if (p->n_whole > 0)
+            LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_whole, 256), 256, 0, s>>>(
+                p->pair_order + p->pair_starts[kPairBucketPiece], p->n_whole, p->a_colptr, p->b_rowptr,
+                p->pieces + p->n_split_pieces));
+    }
+    // limited rows: index map, run lists, B-Limited scratch
+    p->nlim = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketLim0];
+    if (p->nlim > 0) {
+        const int32_t *lrows = p->row_order + p->row_starts[kRowBucketLim0];
+        TRY(palloc(p, &p->lim_index, M, s));
+        TRY(palloc(p, &p->run_start, p->nlim + 1, s));
+        TRY(palloc(p, &p->run_fill, p->nlim, s));
+        CK(cudaMemsetAsync(p->lim_index, 0xff, M * 4, s));
+        CK(cudaMemsetAsync(p->run_fill, 0, p->nlim * 4, s));
+        {
+            Temp tn(s);
+            int64_t *nruns;
+            TRY(talloc(p, tn, &nruns, p->nlim));
+            LAUNCH("lim_index", s, k_lim_index<<<grid_for(p->nlim, 256), 256, 0, s>>>(lrows, p->nlim, p->deg, p->lim_index,
+                                                                                  nruns));
+            TRY(scan_excl(p, nruns, p->nlim, p->run_start, s, "lim_scan"));
+        }
+        // sizes for the run lists and the per-block scratch (sync 3, small)
+        int64_t h[1];
+        CK(cudaMemcpyAsync(h, p->run_start + p->nlim, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        p->lim_runs = h[0];
+        p->lim_max_deg = (int64_t)p->h_scal.max_deg;
+        p->lim_max_L = (int64_t)p->h_scal.max_rowwork;
+        TRY(palloc(p, &p->run_base, p->lim_runs, s));
+        TRY(palloc(p, &p->run_len, p->lim_runs, s));
+        LAUNCH("lim_runs", s, k_lim_runs<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->base, p->lim_index, p->run_start, p->run_fill,
+            p->run_base, p->run_len));
+        p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
+        p->stage_cap = std::min<int64_t>(p->lim_max_L, p->n);
+        TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * p->lim_max_deg, s));
+        TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
+        TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
+        TRY(palloc(p, &p->row_counter, 1, s));
+    }
+    // Ĉ and merge state
+    TRY(palloc(p, &p->chat_col, p->nnz_chat, s));
+    TRY(palloc(p, &p->chat_val, p->nnz_chat, s));
+    TRY(palloc(p, &p->ccount, M, s));
+    TRY(palloc(p, &p->crowptr, M + 1, s));
+    p->state = 1;
+    return SPGEMM_OK;
+}
+
+int spgemm_expand(spgemm_plan_t p, void *stream) {
+    if (!p) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan is NULL");
+    if (p->state < 1) return fail(SPGEMM_ERR_STATE, "plan not ready");
+    cudaStream_t s = (cudaStream_t)stream;
+    p->last_stream = s;
+    CK(cudaSetDevice(p->dev));
+    const int64_t np = p->n_split_pieces + p->n_whole;
+    if (np > 0)
+        LAUNCH("expand_pieces", s, k_expand_pieces<<<(unsigned)np, kPieceThreads, 0, s>>>(
+            p->pieces, p->a_val, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
+    for (int nb = 0; nb < 6; ++nb) {
+        const int64_t lo = p->pair_starts[kPairBucketGather0 + nb * 16];
+        const int64_t cnt = p->pair_starts[kPairBucketGather0 + nb * 16 + 16] - lo;
+        if (cnt == 0) continue;
+        const int32_t *list = p->pair_order + lo;
+        const unsigned grid = (unsigned)cdiv(cnt << nb, 256);
+#define GATHER_CASE(N)                                                                                      \
+    case N:                                                                                                 \
+        LAUNCH("expand_gathered", s, k_expand_gathered<N><<<grid, 256, 0, s>>>(                             \
+            list, cnt, p->a_colptr, p->a_val, p->b_rowptr, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val)); \
+        break;
+        switch (nb) {
+            GATHER_CASE(0)
+            GATHER_CASE(1)
+            GATHER_CASE(2)
+            GATHER_CASE(3)
+            GATHER_CASE(4)
+            GATHER_CASE(5)
+        }
+#undef GATHER_CASE
+    }
+    p->state = 2;
+    return SPGEMM_OK;
+}
+
+int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
+    if (!p) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan is NULL");
+    if (p->state < 2) return fail(SPGEMM_ERR_STATE, "spgemm_merge before spgemm_expand");
+    if (p->state >= 3) return fail(SPGEMM_ERR_STATE, "plan already merged (plans are single-use)");
+    cudaStream_t s = (cudaStream_t)stream;
+    p->last_stream = s;
+    CK(cudaSetDevice(p->dev));
+    const int64_t M = p->m;
+    if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
+    auto rows_of = [&](int b0, int b1, int64_t *cnt) {
+        *cnt = p->row_starts[b1] - p->row_starts[b0];
+        return p->row_order + p->row_starts[b0];
+    };
+    int64_t cnt;
+    const int32_t *rows = rows_of(kRowBucketPass, kRowBucketPass + 1, &cnt);
+    if (cnt > 0)
+        LAUNCH("merge_pass", s, k_merge_pass<<<grid_for(cnt, 256), 256, 0, s>>>(rows, cnt, p->rowoff, p->ccount));
+    rows = rows_of(kRowBucketWarp, kRowBucketWarp + 1, &cnt);
+    if (cnt > 0)
+        LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
+                                                                                      p->chat_col, p->chat_val, p->ccount));
+    rows = rows_of(kRowBucketWarpRadix, kRowBucketWarpRadix + 1, &cnt);
+    if (cnt > 0) {
+        CK(cudaFuncSetAttribute(k_merge_warp_radix, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRadixSmem));
+        LAUNCH("merge_warp_radix", s, k_merge_warp_radix<<<(unsigned)cdiv(cnt, kWarpRadixWarps), kWarpRadixWarps * 32,
+                                                           kWarpRadixSmem, s>>>(rows, cnt, p->rowoff, p->chat_col,
+                                                                                p->chat_val, p->ccount));
+    }
+    rows = rows_of(kRowBucketCtaRadix, kRowBucketCtaRadix + 1, &cnt);
+    if (cnt > 0) {
+        constexpr int CAP = 4096;
+        const int smem = CAP * 16 + kCtaRadixWarps * 256 * 4;
+        CK(cudaFuncSetAttribute(k_merge_cta_radix<CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        LAUNCH("merge_cta_radix", s, k_merge_cta_radix<CAP><<<(unsigned)std::min<int64_t>(cnt, (int64_t)p->num_sms * 3 * 16),
+                                                               kCtaRadixThreads, smem, s>>>(rows, cnt, p->rowoff,
+                                                                                            p->chat_col, p->chat_val,
+                                                                                            p->ccount));
+    }
+    if (p->nlim > 0) {
+        CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
+        LimitedArgs g;
+        g.rows = p->row_order + p->row_starts[kRowBucketLim0];
+        g.nrows = p->nlim;
+        g.rowoff = p->rowoff;
+        g.run_start = p->run_start;
+        g.run_base = p->run_base;
+        g.run_len = p->run_len;
+        g.chat_col = p->chat_col;
+        g.chat_val = p->chat_val;
+        g.ccount = p->ccount;
+        g.scratch_cursor = p->scr_cursor;
+        g.scratch_col = p->scr_col;
+        g.scratch_val = p->scr_val;
+        g.max_deg = p->lim_max_deg;
+        g.stage_cap = p->stage_cap;
+        g.row_counter = p->row_counter;
+        CK(cudaFuncSetAttribute(k_merge_limited, cudaFuncAttributeMaxDynamicSharedMemorySize, kLimSmem));
+        LAUNCH("merge_limited", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
+    }
+    TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
+    CK(cudaMemcpyAsync(&p->nnz_c, p->crowptr + M, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    p->state = 3;
+    if (nnz_c) *nnz_c = p->nnz_c;
+    return SPGEMM_OK;
+}
+
+int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
+    if (!p || !C) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan or C is NULL");
+    if (p->state < 3) return fail(SPGEMM_ERR_STATE, "spgemm_output before spgemm_merge");
+    if (!C->rowptr || (p->nnz_c > 0 && (!C->colidx || !C->val)))
+        return fail(SPGEMM_ERR_INVALID_ARGUMENT, "C arrays are NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(cudaSetDevice(p->dev));
+    C->nrows = p->m;
+    C->ncols = p->n;
+    C->nnz = p->nnz_c;
+    const int64_t nnz = p->nnz_c;
+    int32_t *dcol = C->colidx;
+    float *dval = C->val;
+    Temp t1(s), t2(s);
+    if (C->where == SPGEMM_HOST) {
+        TRY(talloc(p, t1, &dcol, nnz));
+        TRY(talloc(p, t2, &dval, nnz));
+    }
+    if (nnz > 0)
+        LAUNCH("compact", s, k_compact<<<(unsigned)cdiv(nnz, kCompactTile), kCompactThreads, 0, s>>>(
+            p->crowptr, p->m, p->rowoff, p->chat_col, p->chat_val, nnz, dcol, dval));
+    if (C->where == SPGEMM_HOST) {
+        CK(cudaMemcpyAsync(C->rowptr, p->crowptr, (p->m + 1) * 8, cudaMemcpyDeviceToHost, s));
+        if (nnz > 0) {
+            CK(cudaMemcpyAsync(C->colidx, dcol, nnz * 4, cudaMemcpyDeviceToHost, s));
+            CK(cudaMemcpyAsync(C->val, dval, nnz * 4, cudaMemcpyDeviceToHost, s));
+        }
+        CK(cudaStreamSynchronize(s));
+    } else {
+        CK(cudaMemcpyAsync(C->rowptr, p->crowptr, (p->m + 1) * 8, cudaMemcpyDeviceToDevice, s));
+    }
+    return SPGEMM_OK;
+}
+
+int spgemm_execute(spgemm_plan_t p, spgemm_alloc_fn alloc, void *ctx, int32_t out_where, spgemm_csr_out_t *C,
+                   void *stream) {
+    if (!p || !alloc || !C) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan, alloc or C is NULL");
+    if (out_where != SPGEMM_DEVICE && out_where != SPGEMM_HOST)
+        return fail(SPGEMM_ERR_INVALID_ARGUMENT, "bad out_where");
+    TRY(spgemm_expand(p, stream));
+    int64_t nnz;
+    TRY(spgemm_merge(p, stream, &nnz));
+    C->where = out_where;
+    C->rowptr = (int64_t *)alloc((size_t)(p->m + 1) * 8, out_where, ctx);
+    C->colidx = (int32_t *)alloc((size_t)std::max<int64_t>(nnz, 1) * 4, out_where, ctx);
+    C->val = (float *)alloc((size_t)std::max<int64_t>(nnz, 1) * 4, out_where, ctx);
+    if (!C->rowptr || !C->colidx || !C->val) return fail(SPGEMM_ERR_OUT_OF_MEMORY, "C allocation callback failed");
+    return spgemm_output(p, C, stream);
+}
+
+int spgemm_get_stats(spgemm_plan_t p, spgemm_stats_t *st) {
+    if (!p || !st) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan or stats is NULL");
+    memset(st, 0, sizeof(*st));
+    st->m = p->m;
+    st->k = p->k;
+    st->n = p->n;
+    st->nnz_a = p->nnz_a;
+    st->nnz_b = p->nnz_b;
+    st->nnz_chat = p->nnz_chat;
+    st->nnz_chat_rowwise = p->nnz_chat_rowwise;
+    st->nnz_c = p->nnz_c;
+    st->k_nonempty = (int64_t)p->h_scal.k_nonempty;
+    st->m_nonempty = (int64_t)p->h_scal.m_nonempty;
+    st->t_dom = p->t_dom;
+    st->t_lim = p->t_lim;
+    st->n_dominator = p->pair_starts[kPairBucketSplit + 1] - p->pair_starts[kPairBucketSplit];
+    st->n_normal = p->n_whole;
+    st->n_low = p->pair_starts[kPairBucketEmpty] - p->pair_starts[kPairBucketGather0];
+    st->n_pieces_split = p->n_split_pieces;
+    for (int b = 0; b < 6; ++b)
+        st->n_gather_bin[b] = p->pair_starts[kPairBucketGather0 + b * 16 + 16] - p->pair_starts[kPairBucketGather0 + b * 16];
+    st->n_rows_bin[0] = p->row_starts[kRowBucketEmpty + 1] - p->row_starts[kRowBucketEmpty];
+    st->n_rows_bin[1] = p->row_starts[kRowBucketPass + 1] - p->row_starts[kRowBucketPass];
+    st->n_rows_bin[2] = p->row_starts[kRowBucketWarp + 1] - p->row_starts[kRowBucketWarp];
+    st->n_rows_bin[3] = p->row_starts[kRowBucketWarpRadix + 1] - p->row_starts[kRowBucketWarpRadix];
+    st->n_rows_bin[4] = p->row_starts[kRowBucketCtaRadix + 1] - p->row_starts[kRowBucketCtaRadix];
+    st->n_rows_bin[5] = p->nlim;
+    st->bytes_workspace = p->bytes;
+    return SPGEMM_OK;
+}
+
+int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_t *size) {
+    if (!p || !size) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan or size is NULL");
+    CK(cudaSetDevice(p->dev));
+    CK(cudaDeviceSynchronize());
+    const void *src = nullptr;
+    int64_t bytes = 0;
+    std::vector<int64_t> tmp;
+    switch (what) {
+        case SPGEMM_VIEW_WORK: src = p->work; bytes = p->k * 8; break;
+        case SPGEMM_VIEW_ROWWORK: src = p->rowwork; bytes = p->m * 8; break;
+        case SPGEMM_VIEW_ROWOFF: src = p->rowoff; bytes = (p->m + 1) * 8; break;
+        case SPGEMM_VIEW_PAIR_CLASS: src = p->pair_cls; bytes = p->k; break;
+        case SPGEMM_VIEW_ROW_CLASS: src = p->row_cls; bytes = p->m; break;
+        case SPGEMM_VIEW_CHAT_COL:
+            if (p->state != 2) return fail(SPGEMM_ERR_STATE, "Ĉ is only inspectable between expand and merge");
+            src = p->chat_col; bytes = p->nnz_chat * 4; break;
+        case SPGEMM_VIEW_CHAT_VAL:
+            if (p->state != 2) return fail(SPGEMM_ERR_STATE, "Ĉ is only inspectable between expand and merge");
+            src = p->chat_val; bytes = p->nnz_chat * 4; break;
+        case SPGEMM_VIEW_CROWPTR:
+            if (p->state < 3) return fail(SPGEMM_ERR_STATE, "C row pointers exist after merge");
+            src = p->crowptr; bytes = (p->m + 1) * 8; break;
+        case SPGEMM_VIEW_GATHER: {
+            const int64_t lo = p->pair_starts[kPairBucketGather0], hi = p->pair_starts[kPairBucketEmpty];
+            src = p->pair_order + lo;
+            bytes = (hi - lo) * 4;
+            break;
+        }
+        case SPGEMM_VIEW_PIECES: {
+            bytes = p->n_split_pieces * 5 * 8;
+            *size = bytes;
+            if (cap < bytes) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "capacity too small");
+            std::vector<Piece> hp((size_t)p->n_split_pieces);
+            if (p->n_split_pieces) CK(cudaMemcpy(hp.data(), p->pieces, hp.size() * sizeof(Piece), cudaMemcpyDeviceToHost));
+            int64_t *o = (int64_t *)dst;
+            for (size_t q = 0; q < hp.size(); ++q) {
+                o[q * 5 + 0] = hp[q].k;
+                o[q * 5 + 1] = hp[q].a_lo;
+                o[q * 5 + 2] = hp[q].a_lo + hp[q].a_len;
+                o[q * 5 + 3] = hp[q].b_lo;
+                o[q * 5 + 4] = hp[q].b_lo + hp[q].b_len;
+            }
+            return SPGEMM_OK;
+        }
+        default: return fail(SPGEMM_ERR_INVALID_ARGUMENT, "unknown view");
+    }
+    *size = bytes;
+    if (cap < bytes) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "capacity too small");
+    if (bytes > 0) CK(cudaMemcpy(dst, src, (size_t)bytes, cudaMemcpyDeviceToHost));
+    return SPGEMM_OK;
+}
+
+int spgemm_row_partition(const spgemm_csc_t *A, const spgemm_csr_t *B, int32_t parts, int64_t *bounds_host,
+                         void *stream) {
+    if (!A || !B || !bounds_host || parts < 1) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "bad row_partition arguments");
+    TRY(check_csx(A->ncols, A->nrows, A->nnz, A->colptr, A->rowidx, A->val, A->where, "A"));
+    TRY(check_csx(B->nrows, B->ncols, B->nnz, B->rowptr, B->colidx, B->val, B->where, "B"));
+    if (A->ncols != B->nrows) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "A.ncols != B.nrows");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(SPGEMM_ERR_NO_DEVICE, "no CUDA device");
+    spgemm_plan_s tmp;
+    spgemm_plan_s *p = &tmp;
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(cudaGetDevice(&p->dev));
+    p->pool = pool_for_device(p->dev);
+    p->last_stream = s;
+    const int64_t M = A->nrows, K = A->ncols;
+    int r = [&]() -> int {
+        TRY(upload(p, A->colptr, (K + 1) * 8, A->where, (const void **)&p->a_colptr, s));
+        TRY(upload(p, A->rowidx, A->nnz * 4, A->where, (const void **)&p->a_rowidx, s));
+        TRY(upload(p, B->rowptr, (K + 1) * 8, B->where, (const void **)&p->b_rowptr, s));
+        TRY(palloc(p, &p->rowwork, M, s));
+        TRY(palloc(p, &p->deg, M, s));
+        TRY(palloc(p, &p->rowoff, M + 1, s));
+        int64_t *bounds;
+        TRY(palloc(p, &bounds, parts + 1, s));
+        if (M > 0) {
+            CK(cudaMemsetAsync(p->rowwork, 0, M * 8, s));
+            CK(cudaMemsetAsync(p->deg, 0, M * 4, s));
+        }
+        if (A->nnz > 0)
+            LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(A->nnz, 8), 256), 256, 0, s>>>(
+                p->a_colptr, p->a_rowidx, K, A->nnz, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg));
+        TRY(scan_excl(p, p->rowwork, M, p->rowoff, s, "row_offsets"));
+        LAUNCH("partition_bounds", s, k_partition_bounds<<<(unsigned)cdiv(parts + 1, 128), 128, 0, s>>>(p->rowoff, M, parts, bounds));
+        CK(cudaMemcpyAsync(bounds_host, bounds, (parts + 1) * 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        return SPGEMM_OK;
+    }();
+    for (void *v : p->owned) cudaFreeAsync(v, s);
+    p->owned.clear();
+    return r;
+}
+
+int spgemm_destroy(spgemm_plan_t p) {
+    if (!p) return SPGEMM_OK;
+    cudaSetDevice(p->dev);
+    for (void *v : p->owned) cudaFreeAsync(v, p->last_stream);
+    delete p;
+    return SPGEMM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,289 @@
+"""GPU parity: every stage of the CUDA path, called through the C-ABI, against the oracle on
+the same seeded inputs.  Integer / index work is compared bit-exactly; C values within the
+north-star tolerance (relative 1e-5 per entry vs the fp64 oracle; for signed inputs the
+rounding bound 2^-23 * sum|a_ik b_kj| is added)."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from oracle import stages
+import paper_conf_icde_leekyjkp20_b200 as spg
+
+pytestmark = pytest.mark.gpu
+
+RTOL = 1e-5
+
+
+def _sms():
+    return torch.cuda.get_device_properties(0).multi_processor_count
+
+
+def _plan(inp, **opts):
+    A, B = spg.from_inputs(inp, "cuda")
+    return spg.Plan(A, B, **opts), (A, B)
+
+
+def _abs_inputs(inp):
+    return synth.SparseInputs(inp.name + "|abs|", inp.m, inp.k, inp.n, inp.a_colptr, inp.a_rowidx,
+                              np.abs(inp.a_val), inp.b_rowptr, inp.b_colidx, np.abs(inp.b_val))
+
+
+def assert_c_matches(C, inp, signed=False):
+    rowptr, col, val = oracle.gustavson(inp)
+    got_rowptr = C.rowptr.cpu().numpy()
+    got_col = C.colidx.cpu().numpy()
+    got_val = C.val.cpu().numpy().astype(np.float64)
+    np.testing.assert_array_equal(got_rowptr, rowptr)       # structure bit-exact
+    np.testing.assert_array_equal(got_col, col)
+    tol = RTOL * np.abs(val)
+    if signed:
+        _, _, mag = oracle.gustavson(_abs_inputs(inp))
+        tol = tol + 2.0 ** -23 * mag
+    bad = np.abs(got_val - val) > tol
+    assert not bad.any(), f"{bad.sum()} values out of tolerance, e.g. got {got_val[bad][:4]} want {val[bad][:4]}"
+
+
+def _deg(inp):
+    ca, rb, _ = stages.pair_workload(inp)
+    col_of = np.repeat(np.arange(inp.k), ca)
+    d = np.zeros(inp.m, dtype=np.int64)
+    np.add.at(d, inp.a_rowidx.astype(np.int64), (rb[col_of] > 0).astype(np.int64))
+    return d
+
+
+CASES = [
+    ("C1", dict()),
+    ("C1", dict(enable_gather=0)),
+    ("C1", dict(enable_split=0)),
+    ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
+    ("C1", dict(alpha=2.0)),
+    ("C1", dict(beta=10.0)),
+]
+
+
+def _inp(name, seed=1, **kw):
+    if name == "C1":
+        return synth.make_inputs("C1", seed=seed, **kw)
+    raise KeyError(name)
+
+
+# ------------------------------------------------------------------ stage (1) -------------
+@pytest.mark.parametrize("seed", [1, 2])
+def test_stage1_workload(seed):
+    inp = _inp("C1", seed)
+    p, keep = _plan(inp)
+    ca, rb, work = stages.pair_workload(inp)
+    rowwork = stages.row_workload(inp)
+    np.testing.assert_array_equal(p.inspect(spg.VIEW_WORK, np.int64), work)
+    np.testing.assert_array_equal(p.inspect(spg.VIEW_ROWWORK, np.int64), rowwork)
+    np.testing.assert_array_equal(p.inspect(spg.VIEW_ROWOFF, np.int64), stages.chat_row_offsets(rowwork))
+    st = p.stats()
+    assert st["nnz_chat"] == st["nnz_chat_rowwise"] == int(work.sum())
+    assert st["k_nonempty"] == int((work > 0).sum()) and st["m_nonempty"] == int((rowwork > 0).sum())
+    p.destroy()
+
+
+# ------------------------------------------------------------------ stage (2) -------------
+@pytest.mark.parametrize("name,opts", CASES)
+def test_stage2_reorganizer(name, opts):
+    inp = _inp(name)
+    p, keep = _plan(inp, **opts)
+    o = spg.options(**opts)
+    st = p.stats()
+    ca, rb, work = stages.pair_workload(inp)
+    t_dom = stages.dominator_threshold(int(work.sum()), int((work > 0).sum()), o.alpha, _sms(), o.dom_waves,
+                                       o.dom_min_work)
+    assert st["t_dom"] == t_dom
+    cls = stages.classify_pairs(ca, rb, work, t_dom, o.split_ca_max)
+    np.testing.assert_array_equal(p.inspect(spg.VIEW_PAIR_CLASS, np.int8), cls)
+    if o.enable_split:
+        want = stages.split_pieces(inp, cls, o.piece_work, o.split_b_tile, o.split_ca_max)
+        got = p.inspect(spg.VIEW_PIECES, np.int64).reshape(-1, 5)
+        np.testing.assert_array_equal(got, want)
+        assert st["n_pieces_split"] == len(want)
+    if o.enable_gather:
+        lists = stages.gather_lists(ca, rb, cls)
+        np.testing.assert_array_equal(p.inspect(spg.VIEW_GATHER, np.int32),
+                                      np.concatenate([lists[b] for b in range(6)]))
+        assert st["n_gather_bin"] == [len(lists[b]) for b in range(6)]
+    rowwork = stages.row_workload(inp)
+    t_lim = stages.limiting_threshold(int(work.sum()), int((rowwork > 0).sum()), o.beta, 4096)
+    assert st["t_lim"] == t_lim
+    want_rows = stages.row_bins(rowwork, t_lim)
+    got_rows = p.inspect(spg.VIEW_ROW_CLASS, np.int8)
+    single = (_deg(inp) == 1) & (rowwork > 0)
+    np.testing.assert_array_equal(got_rows == 0, want_rows == stages.ROW_EMPTY)
+    np.testing.assert_array_equal(got_rows == 1, single)
+    np.testing.assert_array_equal(got_rows == 5, (want_rows == stages.ROW_LIMITED) & ~single)
+    np.testing.assert_array_equal(got_rows == 2, (want_rows == stages.ROW_WARP) & ~single)
+    np.testing.assert_array_equal((got_rows == 3) | (got_rows == 4), (want_rows == stages.ROW_CTA) & ~single)
+    p.destroy()
+
+
+# ------------------------------------------------------------------ stage (3) -------------
+def _rows_sorted(m, rowoff, cols, vals):
+    out = []
+    for i in range(m):
+        c = cols[rowoff[i]:rowoff[i + 1]]
+        v = vals[rowoff[i]:rowoff[i + 1]]
+        o = np.lexsort((v, c))
+        out.append((c[o], v[o]))
+    return out
+
+
+@pytest.mark.parametrize("name,opts", CASES[:4])
+def test_stage3_expansion_is_eq2(name, opts):
+    inp = _inp(name)
+    p, keep = _plan(inp, **opts)
+    p.expand()
+    cols = p.inspect(spg.VIEW_CHAT_COL, np.int32)
+    vals = p.inspect(spg.VIEW_CHAT_VAL, np.float32)
+    rowoff = p.inspect(spg.VIEW_ROWOFF, np.int64)
+    r, c, v = stages.expand_outer(inp)
+    # each oracle product a*b (exact in fp64) rounded once to fp32 = the kernel's fp32 multiply
+    v32 = v.astype(np.float32)
+    order = np.lexsort((v32, c, r))
+    r, c, v32 = r[order], c[order], v32[order]
+    o_rowoff = np.zeros(inp.m + 1, dtype=np.int64)
+    np.cumsum(np.bincount(r, minlength=inp.m), out=o_rowoff[1:])
+    np.testing.assert_array_equal(rowoff, o_rowoff)
+    got = _rows_sorted(inp.m, rowoff, cols, vals)
+    gc = np.concatenate([g[0] for g in got])
+    gv = np.concatenate([g[1] for g in got])
+    np.testing.assert_array_equal(gc, c)
+    np.testing.assert_array_equal(gv.view(np.uint32), v32.view(np.uint32))   # bit-exact
+    p.destroy()
+
+
+# ------------------------------------------------------------------ stage (4) + output ----
+@pytest.mark.parametrize("name,opts", CASES)
+def test_c_matches_oracle(name, opts):
+    inp = _inp(name)
+    A, B = spg.from_inputs(inp, "cuda")
+    C = spg.matmul(A, B, **opts)
+    assert_c_matches(C, inp)
+
+
+@pytest.mark.parametrize("shape,dens,seed,skew,values", [
+    ((1, 1, 1), (1.0, 1.0), 1, False, "real"),
+    ((7, 5, 9), (0.3, 0.4), 2, False, "real"),
+    ((33, 20, 41), (0.1, 0.15), 4, True, "signed"),
+    ((40, 64, 40), (0.05, 0.5), 5, False, "int"),
+    ((20, 3, 30), (0.0, 0.5), 6, False, "real"),
+    ((25, 30, 12), (0.3, 0.0), 7, False, "real"),
+    ((64, 1, 64), (0.5, 0.5), 8, False, "real"),
+    ((300, 700, 500), (0.03, 0.05), 9, True, "signed"),
+])
+def test_random_tiny(shape, dens, seed, skew, values):
+    inp = synth.random_tiny(*shape, dens[0], dens[1], seed, values=values, skew=skew)
+    A, B = spg.from_inputs(inp, "cuda")
+    for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3)):
+        C = spg.matmul(A, B, **opts)
+        assert_c_matches(C, inp, signed=(values == "signed"))
+
+
+def test_integer_values_exact():
+    inp = synth.make_inputs("C1", seed=5, values="int")
+    A, B = spg.from_inputs(inp, "cuda")
+    C = spg.matmul(A, B)
+    rowptr, col, val = oracle.gustavson(inp)
+    np.testing.assert_array_equal(C.colidx.cpu().numpy(), col)
+    np.testing.assert_array_equal(C.val.cpu().numpy().astype(np.float64), val)   # exact
+
+
+def test_wide_limited_rows_span_many_windows():
+    """Rows whose Ĉ bucket is longer than the non-limited capacity and whose column span
+    covers several 16384-column windows of the B-Limited merge."""
+    rng = np.random.default_rng(3)
+    m, k, n = 40, 120, 70000
+    ar, ac = np.nonzero(rng.random((m, k)) < 0.25)
+    br = np.repeat(np.arange(k), 300)
+    bc = np.concatenate([np.sort(rng.choice(n, 300, replace=False)) for _ in range(k)])
+    # a few narrow-span hub columns so that equal columns collide heavily
+    bc[:300] = np.arange(300) * 3
+    inp = synth.from_coo("wide", m, k, n, (ar, ac, synth.edge_values(ar, ac, 1)),
+                         (br, bc, synth.edge_values(br, bc, 2)))
+    A, B = spg.from_inputs(inp, "cuda")
+    with spg.Plan(A, B) as p:
+        st = p.stats()
+        assert st["n_rows_bin"][5] > 0
+        p.expand()
+        p.merge()
+        C = p.output()
+    assert_c_matches(C, inp)
+
+
+def test_empty_and_degenerate():
+    for shape in [(5, 0, 7), (0, 4, 3), (3, 4, 0)]:
+        m, k, n = shape
+        inp = synth.random_tiny(max(m, 1), max(k, 1), max(n, 1), 0.0, 0.0, 1)
+        inp = synth.SparseInputs("e", m, k, n, np.zeros(k + 1, np.int64), np.zeros(0, np.int32),
+                                 np.zeros(0, np.float32), np.zeros(k + 1, np.int64), np.zeros(0, np.int32),
+                                 np.zeros(0, np.float32))
+        A, B = spg.from_inputs(inp, "cuda")
+        C = spg.matmul(A, B)
+        assert C.nnz == 0 and C.rowptr.cpu().tolist() == [0] * (m + 1)
+
+
+def test_host_inputs_and_outputs():
+    inp = synth.make_inputs("C1", seed=7)
+    A, B = spg.from_inputs(inp, "cpu")
+    C = spg.matmul(A, B, device="cpu")
+    assert not C.val.is_cuda
+    assert_c_matches(C, inp)
+
+
+def test_validation_rejects_malformed():
+    inp = synth.make_inputs("C1", seed=1)
+    bad = inp.a_rowidx.copy()
+    s = int(inp.a_colptr[10])
+    if inp.a_colptr[11] - s >= 2:
+        bad[s], bad[s + 1] = bad[s + 1], bad[s]
+    else:
+        bad[s] = inp.m + 5
+    inp2 = synth.SparseInputs("bad", inp.m, inp.k, inp.n, inp.a_colptr, bad, inp.a_val, inp.b_rowptr,
+                              inp.b_colidx, inp.b_val)
+    A, B = spg.from_inputs(inp2, "cuda")
+    with pytest.raises(spg.SpgemmError, match="malformed"):
+        spg.Plan(A, B)
+
+
+# ------------------------------------------------------------------ full sizes -------------
+@pytest.mark.parametrize("name", ["C2"])
+def test_full_size_sampled(name):
+    """BASELINE.json configs[1] at full size, in the bench's launch configuration: sampled rows
+    compared with the oracle one by one, plus whole-matrix properties."""
+    inp = synth.make_inputs(name, seed=1)
+    A, B = spg.from_inputs(inp, "cuda")
+    with spg.Plan(A, B) as p:
+        st = p.stats()
+        C = p.execute()
+    ca, rb, work = stages.pair_workload(inp)
+    assert st["nnz_chat"] == int(work.sum())
+    rowptr = C.rowptr.cpu().numpy()
+    col = C.colidx.cpu().numpy()
+    val = C.val.cpu().numpy().astype(np.float64)
+    rng = np.random.default_rng(0)
+    rowwork = stages.row_workload(inp)
+    heavy = np.argsort(rowwork)[-200:]
+    rows = np.unique(np.concatenate([rng.integers(0, inp.m, 3000), heavy])).astype(np.int32)
+    orp, ocol, oval = oracle.gustavson(inp, rows=rows)
+    for t, i in enumerate(rows):
+        gc = col[rowptr[i]:rowptr[i + 1]]
+        np.testing.assert_array_equal(gc, ocol[orp[t]:orp[t + 1]])
+        ov = oval[orp[t]:orp[t + 1]]
+        assert np.all(np.abs(val[rowptr[i]:rowptr[i + 1]] - ov) <= RTOL * np.abs(ov))
+    # canonical CSR: rows sorted strictly ascending
+    d = np.diff(col)
+    row_start = np.zeros(col.size, bool)
+    row_start[rowptr[:-1][np.diff(rowptr) > 0]] = True
+    assert np.all((d > 0) | row_start[1:])
+    # C 1 = A (B 1)
+    ones_b = np.bincount(np.repeat(np.arange(inp.k), np.diff(inp.b_rowptr)), weights=inp.b_val.astype(np.float64),
+                         minlength=inp.k)
+    a_cols = np.repeat(np.arange(inp.k), ca)
+    rhs = np.bincount(inp.a_rowidx, weights=inp.a_val.astype(np.float64) * ones_b[a_cols], minlength=inp.m)
+    lhs = np.bincount(np.repeat(np.arange(inp.m), np.diff(rowptr)), weights=val, minlength=inp.m)
+    np.testing.assert_allclose(lhs, rhs, rtol=1e-5)
