@@ -20,16 +20,18 @@ constexpr int kPairBucketGather0 = 2;
 constexpr int kPairBucketEmpty = 98;
 constexpr int kNumPairBuckets = 99;
 // row processing classes (SPGEMM_VIEW_ROW_CLASS) and buckets
-enum : int8_t { RC_EMPTY = 0, RC_PASS = 1, RC_WARP = 2, RC_WARP_RADIX = 3, RC_CTA_RADIX = 4, RC_LIMITED = 5 };
+enum : int8_t { RC_EMPTY = 0, RC_PASS = 1, RC_WARP = 2, RC_WARP_SORT = 3, RC_GROUP_SORT = 4, RC_LIMITED = 5 };
 constexpr int kRowBucketPass = 0;
-constexpr int kRowBucketWarp = 1;
-constexpr int kRowBucketWarpRadix = 2;
-constexpr int kRowBucketCtaRadix = 3;
-constexpr int kRowBucketLim0 = 4;   // 4 + (39 - floor(log2 L)): longest rows first
-constexpr int kRowBucketEmpty = 44;
-constexpr int kNumRowBuckets = 45;
-constexpr int kWarpRowMax = 32;       // register bitonic bin
-constexpr int kWarpRadixMax = 512;    // per-warp smem radix bin
+constexpr int kRowBucketWarp = 1;      // L <= 32: register bitonic
+constexpr int kRowBucketSort256 = 2;   // L <= 256: one warp, smem natural merge sort
+constexpr int kRowBucketSort1K = 3;    // L <= 1024: two warps
+constexpr int kRowBucketSort4K = 4;    // L <= t_lim: eight warps
+constexpr int kRowBucketLim0 = 5;      // 5 + (39 - floor(log2 L)): longest rows first
+constexpr int kRowBucketEmpty = 45;
+constexpr int kNumRowBuckets = 46;
+constexpr int kWarpRowMax = 32;
+constexpr int kSort256Max = 256;
+constexpr int kSort1KMax = 1024;
 
 struct PlanScalars {
     unsigned long long nnz_chat;     // sum_k work[k]
@@ -321,8 +323,9 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
         else if (deg[i] == 1) { c = RC_PASS; b = kRowBucketPass; }
         else if (L > t_lim) { c = RC_LIMITED; b = kRowBucketLim0 + (39 - min(39, ilog2_floor((uint64_t)L))); }
         else if (L <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
-        else if (L <= kWarpRadixMax) { c = RC_WARP_RADIX; b = kRowBucketWarpRadix; }
-        else { c = RC_CTA_RADIX; b = kRowBucketCtaRadix; }
+        else if (L <= kSort256Max) { c = RC_WARP_SORT; b = kRowBucketSort256; }
+        else if (L <= kSort1KMax) { c = RC_WARP_SORT; b = kRowBucketSort1K; }
+        else { c = RC_GROUP_SORT; b = kRowBucketSort4K; }
         rcls[i] = c;
         bucket[i] = (uint8_t)b;
     }

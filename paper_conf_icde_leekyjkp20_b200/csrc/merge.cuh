@@ -6,20 +6,25 @@
 // BASELINE.json north_star: "a row-bucketed sort plus segmented reduce into CSR".
 //
 // Every bin sorts the row's (col, val) pairs by col and reduces equal-col segments in fp64,
-// rounding once to fp32; the merged row is written back in place at the start of the row's
-// Ĉ bucket and its length to ccount[i].  Bins (rows of one class run one kernel):
-//   warp      L <= 32        one warp, register bitonic network (shuffles)
-//   warpradix L <= 512       one warp, stable LSD radix sort in the warp's smem slice
-//   ctaradix  L <= t_lim     one CTA, stable LSD radix sort in smem (warp-ordered ranking)
-//   limited   L >  t_lim     B-Limited: persistent CTAs with a 128 KB smem column window each
-//                            (1 resident block per SM): dense fp64 window = counting sort with
-//                            the segment reduction fused into the bucket accumulation.
+// rounding once to fp32; the merged row is written back in place at the head of the row's
+// Ĉ bucket and its length to ccount[i].
+//
+// A row's bucket is a concatenation of runs -- one per stored a_ik, each in B's ascending
+// column order -- so the sort is a *natural merge sort*: ascending runs are detected, then
+// merged pairwise level by level; each thread produces a contiguous slice of every level's
+// output, locating its start by a merge-path binary search.  Rows with R runs need
+// ceil(log2 R) levels (C2: 4-10 runs on the rows that hold most products).
+//
+// Bins (one kernel each): single-run rows are already merged (passthrough); L <= 32 one warp,
+// register bitonic network; L <= 256 / L <= 1024 one warp per row, row in the warp's smem
+// slice; L <= t_lim (4096) four warps per row; L > t_lim B-Limited (see k_merge_limited).
 #pragma once
 #include "analysis.cuh"
 
 namespace spg {
 
 constexpr int32_t kKeyPad = 0x7fffffff;
+constexpr unsigned kFull = 0xffffffffu;
 
 // ------------------------------------------------------------------------ warp bin ---
 __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ rows, int64_t nrows,
@@ -38,27 +43,27 @@ __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ 
     for (int k = 2; k <= 32; k <<= 1) {
 #pragma unroll
         for (int j = k >> 1; j > 0; j >>= 1) {
-            int32_t pk = __shfl_xor_sync(0xffffffffu, key, j);
-            double pv = __shfl_xor_sync(0xffffffffu, v, j);
+            int32_t pk = __shfl_xor_sync(kFull, key, j);
+            double pv = __shfl_xor_sync(kFull, v, j);
             bool up = (lane & k) == 0;
             bool lower = (lane & j) == 0;
             bool take = lower == up ? (pk < key) : (pk > key);
             if (take) { key = pk; v = pv; }
         }
     }
-    const int32_t prev = __shfl_up_sync(0xffffffffu, key, 1);
-    const int32_t next = __shfl_down_sync(0xffffffffu, key, 1);
+    const int32_t prev = __shfl_up_sync(kFull, key, 1);
+    const int32_t next = __shfl_down_sync(kFull, key, 1);
     const bool valid = key != kKeyPad;
     const bool head = lane == 0 || prev != key;
-    const unsigned heads = __ballot_sync(0xffffffffu, head);
+    const unsigned heads = __ballot_sync(kFull, head);
     const int seg_start = 31 - __clz(heads & (lanemask_lt() | (1u << lane)));
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-        double o = __shfl_up_sync(0xffffffffu, v, d);
+        double o = __shfl_up_sync(kFull, v, d);
         if (lane - d >= seg_start) v += o;
     }
     const bool tail = valid && (lane == 31 || next != key);
-    const unsigned tails = __ballot_sync(0xffffffffu, tail);
+    const unsigned tails = __ballot_sync(kFull, tail);
     if (tail) {
         const int pos = __popc(tails & lanemask_lt());
         chat_col[s + pos] = key;
@@ -67,102 +72,169 @@ __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ 
     if (lane == 0) ccount[i] = __popc(tails);
 }
 
-// ------------------------------------------------------------- radix sort helpers ---
-// Stable LSD radix pass over a[0..L) -> b, 8-bit digit of (key - kmin) >> shift, executed by
-// a group of NW warps; warp w owns the contiguous chunk [w*C, (w+1)*C) and ranks equal
-// digits inside a 32-element step with __match_any_sync (lane order = element order).
-// cnt[w*256 + d]: per-warp digit counters.  Requires the caller to sync the group around it.
-template <int NW>
-struct RadixGroup {
-    __device__ static void sync() {
-        if constexpr (NW == 1) __syncwarp(); else __syncthreads();
+// ------------------------------------------------------------------ thread groups ---
+// A group of NW warps works on one row; GROUPS groups share a CTA.  Groups synchronise with
+// __syncwarp (NW = 1), __syncthreads (one group per CTA) or a named barrier (bar.sync id, n).
+template <int NW, int GROUPS>
+struct Group {
+    static constexpr int T = NW * 32;
+    int gid, gtid;
+    __device__ __forceinline__ Group() : gid(threadIdx.x / T), gtid(threadIdx.x % T) {}
+    __device__ __forceinline__ void sync() const {
+        if constexpr (NW == 1) __syncwarp();
+        else if constexpr (GROUPS == 1) __syncthreads();
+        else asm volatile("bar.sync %0, %1;" ::"r"(1 + gid), "r"(T) : "memory");
+    }
+    // exclusive prefix sum over the group; `sc` = NW + 1 ints private to the group
+    __device__ __forceinline__ int excl_sum(int v, int *sc, int *total) const {
+        const int inc = warp_incl_sum(v);
+        if constexpr (NW == 1) {
+            *total = __shfl_sync(kFull, inc, 31);
+            return inc - v;
+        } else {
+            const int w = gtid >> 5;
+            if (lane_id() == 31) sc[w] = inc;
+            sync();
+            if (gtid == 0) {
+                int run = 0;
+                for (int q = 0; q < NW; ++q) { const int t = sc[q]; sc[q] = run; run += t; }
+                sc[NW] = run;
+            }
+            sync();
+            const int r = sc[w] + inc - v;
+            *total = sc[NW];
+            sync();
+            return r;
+        }
+    }
+    __device__ __forceinline__ int reduce_min(int v, int *sc) const {
+        v = warp_min(v);
+        if constexpr (NW == 1) return v;
+        else {
+            if (lane_id() == 0) sc[gtid >> 5] = v;
+            sync();
+            int r = sc[0];
+            for (int q = 1; q < NW; ++q) r = min(r, sc[q]);
+            sync();
+            return r;
+        }
+    }
+    __device__ __forceinline__ int reduce_max(int v, int *sc) const {
+        v = warp_max(v);
+        if constexpr (NW == 1) return v;
+        else {
+            if (lane_id() == 0) sc[gtid >> 5] = v;
+            sync();
+            int r = sc[0];
+            for (int q = 1; q < NW; ++q) r = max(r, sc[q]);
+            sync();
+            return r;
+        }
     }
 };
 
-template <int NW>
-__device__ __forceinline__ void radix_pass(const int32_t *ka, const float *va, int32_t *kb, float *vb, int L,
-                                           int32_t kmin, int shift, int *cnt, int64_t *scan_sm, int gtid,
-                                           int gwarp) {
-    const int lane = lane_id();
-    const int C = (L + NW - 1) / NW;
-    const int c0 = min(L, gwarp * C), c1 = min(L, c0 + C);
-    for (int t = gtid; t < NW * 256; t += NW * 32) cnt[t] = 0;
-    RadixGroup<NW>::sync();
-    for (int p = c0 + lane; p < c1; p += 32) {
-        int d = ((ka[p] - kmin) >> shift) & 255;
-        atomicAdd(&cnt[gwarp * 256 + d], 1);
-    }
-    RadixGroup<NW>::sync();
-    if constexpr (NW == 1) {
-        // warp scan over 256 digits: lane owns digits [8*lane, 8*lane+8)
-        int loc[8];
-        int sum = 0;
-#pragma unroll
-        for (int q = 0; q < 8; ++q) { loc[q] = cnt[lane * 8 + q]; sum += loc[q]; }
-        int ex = warp_incl_sum(sum) - sum;
-#pragma unroll
-        for (int q = 0; q < 8; ++q) { cnt[lane * 8 + q] = ex; ex += loc[q]; }
-    } else {
-        // thread d (< 256) owns digit d across the NW warps
-        int d = gtid;
-        int tot = 0;
-        if (d < 256)
-            for (int w = 0; w < NW; ++w) tot += cnt[w * 256 + d];
-        int64_t total;
-        int64_t ex = block_excl_sum<NW * 32, int64_t>((int64_t)tot, scan_sm, &total);
-        if (d < 256) {
-            int run = (int)ex;
-            for (int w = 0; w < NW; ++w) {
-                int c = cnt[w * 256 + d];
-                cnt[w * 256 + d] = run;
-                run += c;
+__device__ __forceinline__ void cp_async4(void *smem_dst, const void *gmem_src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(d), "l"(gmem_src) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+// Smem footprint of a sorter with capacity CAP: keys/vals double-buffered + run bounds.
+template <int CAP>
+struct SortSmem {
+    static constexpr int kBoundsA = CAP + 1, kBoundsB = CAP / 2 + 2;
+    static constexpr int kBytes = CAP * 16 + (kBoundsA + kBoundsB) * 4;
+};
+
+// Natural merge sort of k[0..L) (with v) held in smem by group g.  Returns 0 if the sorted
+// data ends in (k0, v0), 1 if in (k1, v1).
+template <int NW, int GROUPS, int CAP>
+__device__ __forceinline__ int natural_merge_sort(const Group<NW, GROUPS> &g, int32_t *k0, float *v0, int32_t *k1,
+                                                  float *v1, int *bA, int *bB, int L, int *sc) {
+    constexpr int T = NW * 32;
+    const int E = (L + T - 1) / T;
+    const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
+    // run heads: p == 0 or k[p] <= k[p-1]
+    int nh = 0;
+    for (int p = p0; p < p1; ++p) nh += (p == 0 || k0[p] <= k0[p - 1]);
+    int R;
+    int pos = g.excl_sum(nh, sc, &R);
+    for (int p = p0; p < p1; ++p)
+        if (p == 0 || k0[p] <= k0[p - 1]) bA[pos++] = p;
+    if (g.gtid == 0) bA[R] = L;
+    g.sync();
+    int32_t *ks = k0, *kd = k1;
+    float *vs = v0, *vd = v1;
+    int *bs = bA, *bd = bB;
+    int which = 0;
+    while (R > 1) {
+        const int pairs = (R + 1) >> 1;
+        if (p0 < p1) {
+            int lo = 0, hi = pairs;          // pair q: last q with bs[2q] <= p0
+            while (hi - lo > 1) {
+                const int mid = (lo + hi) >> 1;
+                if (bs[2 * mid] <= p0) lo = mid; else hi = mid;
+            }
+            int q = lo;
+            int o = p0;
+            while (o < p1) {
+                const int a0 = bs[2 * q];
+                const int a1 = bs[min(2 * q + 1, R)];
+                const int b1 = bs[min(2 * q + 2, R)];
+                const int na = a1 - a0, nb = b1 - a1;
+                const int d = o - a0;
+                int ilo = max(0, d - nb), ihi = min(d, na);
+                while (ilo < ihi) {           // merge path: first i with A[i] > B[d-i-1]
+                    const int mi = (ilo + ihi) >> 1;
+                    if (ks[a0 + mi] <= ks[a1 + d - mi - 1]) ilo = mi + 1; else ihi = mi;
+                }
+                int ia = ilo, jb = d - ilo;
+                int32_t ka = ia < na ? ks[a0 + ia] : kKeyPad;
+                float va = ia < na ? vs[a0 + ia] : 0.f;
+                int32_t kb = jb < nb ? ks[a1 + jb] : kKeyPad;
+                float vb = jb < nb ? vs[a1 + jb] : 0.f;
+                const int oend = min(p1, b1);
+                for (; o < oend; ++o) {
+                    const bool tA = jb >= nb || (ia < na && ka <= kb);
+                    kd[o] = tA ? ka : kb;
+                    vd[o] = tA ? va : vb;
+                    ia += tA;
+                    jb += !tA;
+                    const bool ok = tA ? ia < na : jb < nb;
+                    const int idx = tA ? a0 + ia : a1 + jb;
+                    const int32_t nk = ok ? ks[idx] : kKeyPad;
+                    const float nv = ok ? vs[idx] : 0.f;
+                    if (tA) { ka = nk; va = nv; } else { kb = nk; vb = nv; }
+                }
+                ++q;
             }
         }
+        g.sync();
+        for (int q = g.gtid; q <= pairs; q += T) bd[q] = q < pairs ? bs[2 * q] : L;
+        g.sync();
+        { int32_t *t = ks; ks = kd; kd = t; }
+        { float *t = vs; vs = vd; vd = t; }
+        { int *t = bs; bs = bd; bd = t; }
+        which ^= 1;
+        R = pairs;
     }
-    RadixGroup<NW>::sync();
-    for (int p0 = c0; p0 < c1; p0 += 32) {
-        const int p = p0 + lane;
-        const bool ok = p < c1;
-        int32_t k = ok ? ka[p] : 0;
-        float v = ok ? va[p] : 0.f;
-        int d = ok ? (((k - kmin) >> shift) & 255) : 256 + lane;
-        unsigned peers = __match_any_sync(0xffffffffu, d);
-        int rank = __popc(peers & lanemask_lt());
-        int pos = ok ? cnt[gwarp * 256 + d] + rank : 0;
-        __syncwarp();
-        if (ok) {
-            kb[pos] = k;
-            vb[pos] = v;
-            if (rank == 0) cnt[gwarp * 256 + d] += __popc(peers);
-        }
-        __syncwarp();
-    }
-    RadixGroup<NW>::sync();
+    return which;
 }
 
-// Segmented reduce of a sorted row kept in smem (k[0..L), v[0..L)) by a group of NW warps;
-// writes the merged row to out_col/out_val[0..U) and returns U.  Each thread owns a contiguous
-// run of ITEMS elements; a segment is summed in fp64 by the thread owning its head.
-template <int NW>
-__device__ __forceinline__ int segmented_reduce_out(const int32_t *k, const float *v, int L, int32_t kmin,
-                                                    int32_t *__restrict__ out_col, float *__restrict__ out_val,
-                                                    int64_t *scan_sm, int gtid) {
+// Segmented reduce of a sorted row in smem; writes the merged row to out_col/out_val[0..U)
+// and returns U.  Each thread owns a contiguous slice; a segment is summed in fp64 by the
+// thread owning its head.
+template <int NW, int GROUPS>
+__device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, const int32_t *k, const float *v,
+                                                    int L, int32_t *__restrict__ out_col, float *__restrict__ out_val,
+                                                    int *sc) {
     constexpr int T = NW * 32;
-    const int items = (L + T - 1) / T;
-    const int p0 = min(L, gtid * items), p1 = min(L, p0 + items);
+    const int E = (L + T - 1) / T;
+    const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
     int nh = 0;
     for (int p = p0; p < p1; ++p) nh += (p == 0 || k[p] != k[p - 1]);
     int total;
-    int pos;
-    if constexpr (NW == 1) {
-        int inc = warp_incl_sum(nh);
-        pos = inc - nh;
-        total = __shfl_sync(0xffffffffu, inc, 31);
-    } else {
-        int64_t t64;
-        pos = (int)block_excl_sum<T, int64_t>((int64_t)nh, scan_sm, &t64);
-        total = (int)t64;
-    }
+    int pos = g.excl_sum(nh, sc, &total);
     for (int p = p0; p < p1; ++p) {
         if (p == 0 || k[p] != k[p - 1]) {
             const int32_t key = k[p];
@@ -173,113 +245,74 @@ __device__ __forceinline__ int segmented_reduce_out(const int32_t *k, const floa
             ++pos;
         }
     }
-    (void)kmin;
     return total;
 }
 
-// ------------------------------------------------------------------ warp radix bin ---
-constexpr int kWarpRadixWarps = 8;
-constexpr int kWarpRadixSmem = kWarpRadixWarps * (kWarpRadixMax * 16 + 256 * 4);
-
-__global__ void __launch_bounds__(kWarpRadixWarps * 32) k_merge_warp_radix(
-    const int32_t *__restrict__ rows, int64_t nrows, const int64_t *__restrict__ rowoff,
-    int32_t *__restrict__ chat_col, float *__restrict__ chat_val, int64_t *__restrict__ ccount) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int w = warp_id(), lane = lane_id();
-    unsigned char *my = smem_raw + w * (kWarpRadixMax * 16 + 256 * 4);
-    int32_t *k0 = (int32_t *)my;
-    float *v0 = (float *)(my + kWarpRadixMax * 4);
-    int32_t *k1 = (int32_t *)(my + kWarpRadixMax * 8);
-    float *v1 = (float *)(my + kWarpRadixMax * 12);
-    int *cnt = (int *)(my + kWarpRadixMax * 16);
-    const int64_t gw = (int64_t)blockIdx.x * kWarpRadixWarps + w;
-    if (gw >= nrows) return;
-    const int i = rows[gw];
-    const int64_t s = rowoff[i];
-    const int L = (int)(rowoff[i + 1] - s);
-    int32_t mn = kKeyPad, mx = 0;
-    for (int p = lane; p < L; p += 32) {
-        int32_t c = chat_col[s + p];
-        k0[p] = c;
-        v0[p] = chat_val[s + p];
-        mn = min(mn, c);
-        mx = max(mx, c);
+// Load Ĉ[s, s+L) into smem (cp.async), sort, reduce, write the merged row back to Ĉ[s, ...).
+template <int NW, int GROUPS, int CAP>
+__device__ __forceinline__ int merge_row_in_smem(const Group<NW, GROUPS> &g, unsigned char *slice, int *sc,
+                                                 int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
+                                                 int64_t s, int L, int32_t *__restrict__ out_col,
+                                                 float *__restrict__ out_val) {
+    constexpr int T = NW * 32;
+    int32_t *k0 = (int32_t *)slice;
+    float *v0 = (float *)(slice + CAP * 4);
+    int32_t *k1 = (int32_t *)(slice + CAP * 8);
+    float *v1 = (float *)(slice + CAP * 12);
+    int *bA = (int *)(slice + CAP * 16);
+    int *bB = bA + SortSmem<CAP>::kBoundsA;
+    for (int p = g.gtid; p < L; p += T) {
+        cp_async4(k0 + p, chat_col + s + p);
+        cp_async4(v0 + p, chat_val + s + p);
     }
-    mn = warp_min(mn);
-    mx = warp_max(mx);
-    __syncwarp();
-    const uint32_t span = (uint32_t)(mx - mn);
-    const int bits = span ? 32 - __clz(span) : 0;
-    for (int sh = 0; sh < bits; sh += 8) {
-        radix_pass<1>(k0, v0, k1, v1, L, mn, sh, cnt, nullptr, lane, 0);
-        int32_t *tk = k0; k0 = k1; k1 = tk;
-        float *tv = v0; v0 = v1; v1 = tv;
-    }
-    const int U = segmented_reduce_out<1>(k0, v0, L, mn, chat_col + s, chat_val + s, nullptr, lane);
-    if (lane == 0) ccount[i] = U;
+    cp_async_wait_all();
+    g.sync();
+    const int which = natural_merge_sort<NW, GROUPS, CAP>(g, k0, v0, k1, v1, bA, bB, L, sc);
+    const int U = segmented_reduce_out<NW, GROUPS>(g, which ? k1 : k0, which ? v1 : v0, L, out_col, out_val, sc);
+    g.sync();
+    return U;
 }
 
-// ------------------------------------------------------------------- CTA radix bin ---
-constexpr int kCtaRadixThreads = 256;
-constexpr int kCtaRadixWarps = kCtaRadixThreads / 32;
-
-template <int CAP>
-__global__ void __launch_bounds__(kCtaRadixThreads) k_merge_cta_radix(
-    const int32_t *__restrict__ rows, int64_t nrows, const int64_t *__restrict__ rowoff,
-    int32_t *__restrict__ chat_col, float *__restrict__ chat_val, int64_t *__restrict__ ccount) {
+template <int NW, int GROUPS, int CAP>
+__global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *__restrict__ rows, int64_t nrows,
+                                                                const int64_t *__restrict__ rowoff,
+                                                                int32_t *__restrict__ chat_col,
+                                                                float *__restrict__ chat_val,
+                                                                int64_t *__restrict__ ccount) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    int32_t *k0 = (int32_t *)smem_raw;
-    float *v0 = (float *)(smem_raw + CAP * 4);
-    int32_t *k1 = (int32_t *)(smem_raw + CAP * 8);
-    float *v1 = (float *)(smem_raw + CAP * 12);
-    int *cnt = (int *)(smem_raw + CAP * 16);
-    __shared__ int64_t scan_sm[kCtaRadixWarps + 1];
-    __shared__ int32_t red_sm[kCtaRadixWarps];
-    for (int64_t r = blockIdx.x; r < nrows; r += gridDim.x) {
+    __shared__ int sc_all[GROUPS][NW + 1];
+    const Group<NW, GROUPS> g;
+    unsigned char *slice = smem_raw + (size_t)g.gid * SortSmem<CAP>::kBytes;
+    for (int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
         const int i = rows[r];
         const int64_t s = rowoff[i];
         const int L = (int)(rowoff[i + 1] - s);
-        int32_t mn = kKeyPad, mx = 0;
-        for (int p = threadIdx.x; p < L; p += kCtaRadixThreads) {
-            int32_t c = chat_col[s + p];
-            k0[p] = c;
-            v0[p] = chat_val[s + p];
-            mn = min(mn, c);
-            mx = max(mx, c);
-        }
-        mn = block_reduce_min<kCtaRadixThreads>(mn, red_sm);
-        mx = block_reduce_max<kCtaRadixThreads>(mx, red_sm);
-        const uint32_t span = (uint32_t)(mx - mn);
-        const int bits = span ? 32 - __clz(span) : 0;
-        int32_t *ka = k0, *kb = k1;
-        float *va = v0, *vb = v1;
-        for (int sh = 0; sh < bits; sh += 8) {
-            radix_pass<kCtaRadixWarps>(ka, va, kb, vb, L, mn, sh, cnt, scan_sm, threadIdx.x, warp_id());
-            int32_t *tk = ka; ka = kb; kb = tk;
-            float *tv = va; va = vb; vb = tv;
-        }
-        const int U = segmented_reduce_out<kCtaRadixWarps>(ka, va, L, mn, chat_col + s, chat_val + s, scan_sm,
-                                                           threadIdx.x);
-        if (threadIdx.x == 0) ccount[i] = U;
-        __syncthreads();
+        const int U = merge_row_in_smem<NW, GROUPS, CAP>(g, slice, sc_all[g.gid], chat_col, chat_val, s, L,
+                                                         chat_col + s, chat_val + s);
+        if (g.gtid == 0) ccount[i] = U;
     }
 }
 
 // ------------------------------------------------------------------- limited bin ---
-// B-Limiting (L463-L477 L, Fig. 7): each block takes a 128 KB shared-memory column window so
-// at most `limit_ctas_per_sm` (default 1) limited merge blocks are resident per SM; the grid is
-// persistent (#SMs x limit) and claims rows longest-first from the limited list.
-//
-// Row i's Ĉ bucket is a set of runs (one per A entry (i,k)), each sorted by column (B's order).
-// The block sweeps the row's column span in windows of S columns; per-run cursors advance
-// monotonically, so every product is read once.  Inside a window the products are counted
-// into their column bucket (fp64 accumulator + touched bit): a counting sort with the
-// segment reduction fused into the bucket.  Emitting the set bits in order yields the
-// window's merged, sorted output.  The merged row is staged in the block's private global
-// scratch and copied back in place once the whole row has been read.
+// B-Limiting (L463-L477 L, Fig. 7): limited merge blocks take ~200 KB of shared memory each,
+// so one is resident per SM (x limit_ctas_per_sm); the grid is persistent and claims rows
+// longest-first.  Per row, by size and density:
+//   * L <= kLimCap: the whole row is sorted in smem (natural merge sort) and written in place;
+//   * dense rows (many products per column of their span): column windows of kLimWindow
+//     columns with an fp64 accumulator + touched bits (a counting sort whose bucket
+//     accumulation fuses the segment reduction); runs are swept with monotone cursors;
+//   * sparse long rows: column windows sized so their products fit kLimCap; each window's
+//     sub-runs (found by binary search from the run cursors) are gathered into smem and
+//     merge-sorted.
+// The merged output of the two windowed paths is staged in the block's global scratch and
+// copied to the head of the row's bucket after the whole row has been read.
 constexpr int kLimThreads = 512;
-constexpr int kLimWindow = 16384;                       // columns per window (S)
-constexpr int kLimSmem = kLimWindow * 8 + (kLimWindow / 32) * 4;
+constexpr int kLimNW = kLimThreads / 32;
+constexpr int kLimCap = 9216;
+constexpr int kLimWindow = 16384;
+constexpr int kLimSmem = SortSmem<kLimCap>::kBytes > kLimWindow * 8 + (kLimWindow / 32) * 4
+                             ? SortSmem<kLimCap>::kBytes
+                             : kLimWindow * 8 + (kLimWindow / 32) * 4;
 
 struct LimitedArgs {
     const int32_t *rows;          // limited rows, longest first
@@ -292,6 +325,7 @@ struct LimitedArgs {
     float *chat_val;
     int64_t *ccount;
     int32_t *scratch_cursor;      // [grid][max_deg]
+    int32_t *scratch_cnt;         // [grid][max_deg]
     int32_t *scratch_col;         // [grid][stage_cap]
     float *scratch_val;
     int64_t max_deg;
@@ -308,20 +342,29 @@ __device__ __forceinline__ void smem_add_f64(double *addr, double v) {
     } while (old != assumed);
 }
 
+// number of entries of run [b, b+len) from position cur whose column is < wend (run sorted)
+__device__ __forceinline__ int count_below(const int32_t *__restrict__ col, int64_t b, int cur, int len, int32_t wend) {
+    int lo = cur, hi = len;     // first p in [cur, len) with col[b+p] >= wend
+    int step = 1;               // galloping from the cursor, then binary search
+    while (lo + step < hi && col[b + lo + step - 1] < wend) { lo += step; step <<= 1; }
+    hi = min(hi, lo + step);
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (col[b + mid] < wend) lo = mid + 1; else hi = mid;
+    }
+    return lo - cur;
+}
+
 __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    double *acc = (double *)smem_raw;
-    uint32_t *bits = (uint32_t *)(smem_raw + kLimWindow * 8);
-    __shared__ int64_t scan_sm[kLimThreads / 32 + 1];
-    __shared__ int32_t red_sm[kLimThreads / 32];
+    __shared__ int sc[kLimNW + 1];
     __shared__ int64_t row_sm;
-    constexpr int NW = kLimThreads / 32;
+    const Group<kLimNW, 1> grp;
+    const int lane = lane_id(), w = warp_id();
     int32_t *cursor = g.scratch_cursor + (int64_t)blockIdx.x * g.max_deg;
+    int32_t *cnt = g.scratch_cnt + (int64_t)blockIdx.x * g.max_deg;
     int32_t *st_col = g.scratch_col + (int64_t)blockIdx.x * g.stage_cap;
     float *st_val = g.scratch_val + (int64_t)blockIdx.x * g.stage_cap;
-    for (int t = threadIdx.x; t < kLimWindow; t += kLimThreads) acc[t] = 0.0;
-    for (int t = threadIdx.x; t < kLimWindow / 32; t += kLimThreads) bits[t] = 0u;
-    const int lane = lane_id(), w = warp_id();
     while (true) {
         if (threadIdx.x == 0) row_sm = (int64_t)atomicAdd(g.row_counter, 1ull);
         __syncthreads();
@@ -329,83 +372,192 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         __syncthreads();
         if (r >= g.nrows) break;
         const int i = g.rows[r];
-        const int64_t rs = g.run_start[r], R = g.run_start[r + 1] - rs;
+        const int64_t s = g.rowoff[i];
+        const int64_t L = g.rowoff[i + 1] - s;
+        if (L <= kLimCap) {
+            const int U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)L,
+                                                                g.chat_col + s, g.chat_val + s);
+            if (threadIdx.x == 0) g.ccount[i] = U;
+            continue;
+        }
+        const int64_t rs = g.run_start[r];
+        const int R = (int)(g.run_start[r + 1] - rs);
         const int64_t *rbase = g.run_base + rs;
         const int32_t *rlen = g.run_len + rs;
-        // column span of the row: first / last column of every run
         int32_t mn = kKeyPad, mx = 0;
-        for (int64_t q = threadIdx.x; q < R; q += kLimThreads) {
+        for (int q = threadIdx.x; q < R; q += kLimThreads) {
             const int64_t b = rbase[q];
             mn = min(mn, g.chat_col[b]);
             mx = max(mx, g.chat_col[b + rlen[q] - 1]);
             cursor[q] = 0;
         }
-        mn = block_reduce_min<kLimThreads>(mn, red_sm);
-        mx = block_reduce_max<kLimThreads>(mx, red_sm);
+        mn = grp.reduce_min(mn, sc);
+        mx = grp.reduce_max(mx, sc);
+        const int64_t span = (int64_t)mx - mn + 1;
+        const int64_t nwin_dense = (span + kLimWindow - 1) / kLimWindow;
+        const bool dense = L * 4 >= span && (int64_t)R * nwin_dense <= 2 * L;
         int64_t nout = 0;
-        for (int64_t w0 = mn; w0 <= mx; w0 += kLimWindow) {
-            const int32_t wend = (int32_t)min((int64_t)mx + 1, w0 + kLimWindow);
-            // sweep: warp per run, 128 products per step (4 loads in flight per lane)
-            for (int64_t q = w; q < R; q += NW) {
-                const int64_t b = rbase[q];
-                const int len = rlen[q];
-                int cur = cursor[q];
-                while (cur < len) {
-                    int32_t c[4];
-                    float v[4];
+        if (dense) {
+            double *acc = (double *)smem_raw;
+            uint32_t *bits = (uint32_t *)(smem_raw + kLimWindow * 8);
+            for (int t = threadIdx.x; t < kLimWindow; t += kLimThreads) acc[t] = 0.0;
+            for (int t = threadIdx.x; t < kLimWindow / 32; t += kLimThreads) bits[t] = 0u;
+            __syncthreads();
+            for (int64_t w0 = mn; w0 <= mx; w0 += kLimWindow) {
+                const int32_t wend = (int32_t)min((int64_t)mx + 1, w0 + kLimWindow);
+                for (int q = w; q < R; q += kLimNW) {       // warp per run, 128 products per step
+                    const int64_t b = rbase[q];
+                    const int len = rlen[q];
+                    int cur = cursor[q];
+                    while (cur < len) {
+                        int32_t c[4];
+                        float v[4];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const int p = cur + u * 32 + lane;
-                        c[u] = p < len ? g.chat_col[b + p] : kKeyPad;
-                        v[u] = p < len ? g.chat_val[b + p] : 0.f;
-                    }
-                    int taken = 0;
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) {
-                        const bool in = c[u] < wend;
-                        if (in) {
-                            const int x = c[u] - (int32_t)w0;
-                            smem_add_f64(acc + x, (double)v[u]);
-                            atomicOr(bits + (x >> 5), 1u << (x & 31));
+                        for (int u = 0; u < 4; ++u) {
+                            const int p = cur + u * 32 + lane;
+                            c[u] = p < len ? g.chat_col[b + p] : kKeyPad;
+                            v[u] = p < len ? g.chat_val[b + p] : 0.f;
                         }
-                        taken += __popc(__ballot_sync(0xffffffffu, in));
+                        int taken = 0;
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) {
+                            const bool in = c[u] < wend;
+                            if (in) {
+                                const int x = c[u] - (int32_t)w0;
+                                smem_add_f64(acc + x, (double)v[u]);
+                                atomicOr(bits + (x >> 5), 1u << (x & 31));
+                            }
+                            taken += __popc(__ballot_sync(kFull, in));
+                        }
+                        cur += taken;
+                        if (taken < 128) break;
                     }
-                    cur += taken;
-                    if (taken < 128) break;
+                    if (lane == 0) cursor[q] = cur;
                 }
-                if (lane == 0) cursor[q] = cur;
-            }
-            __syncthreads();
-            // emit the window's touched columns in ascending order
-            constexpr int WPT = (kLimWindow / 32) / kLimThreads;  // bit words per thread
-            int cntw = 0;
-            uint32_t word[WPT > 0 ? WPT : 1];
+                __syncthreads();
+                constexpr int WPT = (kLimWindow / 32) / kLimThreads;
+                int cntw = 0;
+                uint32_t word[WPT];
 #pragma unroll
-            for (int u = 0; u < WPT; ++u) {
-                word[u] = bits[threadIdx.x * WPT + u];
-                cntw += __popc(word[u]);
-            }
-            int64_t tot;
-            int64_t pos = nout + block_excl_sum<kLimThreads, int64_t>((int64_t)cntw, scan_sm, &tot);
-#pragma unroll
-            for (int u = 0; u < WPT; ++u) {
-                uint32_t m = word[u];
-                while (m) {
-                    const int bpos = __ffs(m) - 1;
-                    m &= m - 1;
-                    const int x = (threadIdx.x * WPT + u) * 32 + bpos;
-                    st_col[pos] = (int32_t)w0 + x;
-                    st_val[pos] = (float)acc[x];
-                    acc[x] = 0.0;
-                    ++pos;
+                for (int u = 0; u < WPT; ++u) {
+                    word[u] = bits[threadIdx.x * WPT + u];
+                    cntw += __popc(word[u]);
                 }
-                bits[threadIdx.x * WPT + u] = 0u;
+                int tot;
+                int64_t pos = nout + grp.excl_sum(cntw, sc, &tot);
+#pragma unroll
+                for (int u = 0; u < WPT; ++u) {
+                    uint32_t m = word[u];
+                    while (m) {
+                        const int bpos = __ffs(m) - 1;
+                        m &= m - 1;
+                        const int x = (threadIdx.x * WPT + u) * 32 + bpos;
+                        st_col[pos] = (int32_t)w0 + x;
+                        st_val[pos] = (float)acc[x];
+                        acc[x] = 0.0;
+                        ++pos;
+                    }
+                    bits[threadIdx.x * WPT + u] = 0u;
+                }
+                nout += tot;
+                __syncthreads();
             }
-            nout += tot;
-            __syncthreads();
+        } else {
+            // sparse: windows whose products fit the smem sorter
+            int32_t *k0 = (int32_t *)smem_raw;
+            float *v0 = (float *)(smem_raw + kLimCap * 4);
+            int64_t remaining = L;
+            int64_t w0 = mn;
+            while (w0 <= mx) {
+                int64_t width = max((int64_t)1, (int64_t)((double)(mx + 1 - w0) * (kLimCap / 2) / (double)max(remaining, (int64_t)1)));
+                int total = 0;
+                int32_t wend = 0;
+                int32_t head = kKeyPad;
+                while (true) {
+                    wend = (int32_t)min((int64_t)mx + 1, w0 + width);
+                    int part = 0;
+                    int32_t hmin = kKeyPad;
+                    for (int q = threadIdx.x; q < R; q += kLimThreads) {
+                        const int64_t b = rbase[q];
+                        const int cur = cursor[q], len = rlen[q];
+                        if (cur < len) hmin = min(hmin, g.chat_col[b + cur]);
+                        const int c = count_below(g.chat_col, b, cur, len, wend);
+                        cnt[q] = c;
+                        part += c;
+                    }
+                    int tot;
+                    grp.excl_sum(part, sc, &tot);
+                    total = tot;
+                    head = grp.reduce_min(hmin, sc);
+                    if (total <= kLimCap || width == 1) break;
+                    width = max((int64_t)1, width / 2);
+                }
+                if (total == 0) {              // empty window: jump to the next product's column
+                    w0 = max((int64_t)wend, (int64_t)head);
+                    continue;
+                }
+                if (total > kLimCap) {         // one column (w0) present in > kLimCap runs
+                    double part = 0.0;
+                    for (int q = threadIdx.x; q < R; q += kLimThreads) {
+                        if (cnt[q] > 0) {
+                            part += (double)g.chat_val[rbase[q] + cursor[q]];
+                            cursor[q] += 1;
+                        }
+                    }
+                    part = warp_sum(part);
+                    __shared__ double dred[kLimNW];
+                    if (lane == 0) dred[w] = part;
+                    __syncthreads();
+                    if (threadIdx.x == 0) {
+                        double t = 0.0;
+                        for (int q = 0; q < kLimNW; ++q) t += dred[q];
+                        st_col[nout] = (int32_t)w0;
+                        st_val[nout] = (float)t;
+                    }
+                    __syncthreads();
+                    nout += 1;
+                    remaining -= total;
+                    w0 = wend;
+                    continue;
+                }
+                // exclusive scan of cnt[0..R) into offsets (cnt[R] = total), then warp-per-run gather
+                int base_off = 0;
+                for (int q0 = 0; q0 < R; q0 += kLimThreads) {
+                    const int q = q0 + threadIdx.x;
+                    const int c = q < R ? cnt[q] : 0;
+                    int tot;
+                    const int ex = grp.excl_sum(c, sc, &tot);
+                    if (q < R) cnt[q] = base_off + ex;
+                    base_off += tot;
+                }
+                if (threadIdx.x == 0) cnt[R] = base_off;
+                __syncthreads();
+                for (int q = w; q < R; q += kLimNW) {
+                    const int off = cnt[q], c = cnt[q + 1] - off;
+                    if (c == 0) continue;
+                    const int64_t b = rbase[q] + cursor[q];
+                    for (int t = lane; t < c; t += 32) {
+                        cp_async4(k0 + off + t, g.chat_col + b + t);
+                        cp_async4(v0 + off + t, g.chat_val + b + t);
+                    }
+                    if (lane == 0) cursor[q] += c;
+                }
+                cp_async_wait_all();
+                __syncthreads();
+                int32_t *k1 = (int32_t *)(smem_raw + kLimCap * 8);
+                float *v1 = (float *)(smem_raw + kLimCap * 12);
+                int *bA = (int *)(smem_raw + kLimCap * 16);
+                int *bB = bA + SortSmem<kLimCap>::kBoundsA;
+                const int which = natural_merge_sort<kLimNW, 1, kLimCap>(grp, k0, v0, k1, v1, bA, bB, total, sc);
+                const int U = segmented_reduce_out<kLimNW, 1>(grp, which ? k1 : k0, which ? v1 : v0, total,
+                                                              st_col + nout, st_val + nout, sc);
+                __syncthreads();
+                nout += U;
+                remaining -= total;
+                w0 = wend;
+            }
         }
         // copy the merged row back into the head of its Ĉ bucket
-        const int64_t s = g.rowoff[i];
         for (int64_t p = threadIdx.x; p < nout; p += kLimThreads) {
             g.chat_col[s + p] = st_col[p];
             g.chat_val[s + p] = st_val[p];

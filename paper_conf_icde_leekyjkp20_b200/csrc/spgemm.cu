@@ -34,9 +34,9 @@ static int fail(int code, const std::string &msg) {
         }                                                                                        \
     } while (0)
 
-#define TRY(call)                      \
-    do {                               \
-        int _r = (call);               \
+#define TRY(...)                        \
+    do {                                \
+        int _r = (__VA_ARGS__);         \
         if (_r != SPGEMM_OK) return _r; \
     } while (0)
 
@@ -140,7 +140,7 @@ struct spgemm_plan_s {
     int64_t lim_runs = 0, lim_max_deg = 0, lim_max_L = 0, nlim = 0;
     int64_t *run_start = nullptr, *run_base = nullptr;
     int32_t *run_len = nullptr, *lim_index = nullptr, *run_fill = nullptr;
-    int32_t *scr_cursor = nullptr, *scr_col = nullptr;
+    int32_t *scr_cursor = nullptr, *scr_cnt = nullptr, *scr_col = nullptr;
     float *scr_val = nullptr;
     int64_t stage_cap = 0;
     int lim_grid = 0;
@@ -225,6 +225,18 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     TRY(scan_excl(p, counts, (int64_t)nb * ntiles, offs, s, name));
     LAUNCH(name, s, k_part_scatter<<<(unsigned)ntiles, kPartThreads, 0, s>>>(bucket, n, nb, offs, ntiles, out_idx));
     LAUNCH(name, s, k_bucket_starts<<<(unsigned)cdiv(nb + 1, 128), 128, 0, s>>>(offs, nb, ntiles, d_starts));
+    return SPGEMM_OK;
+}
+
+template <int NW, int GROUPS, int CAP>
+static int launch_sort_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
+                           int ctas_per_sm) {
+    if (cnt == 0) return SPGEMM_OK;
+    const int smem = SortSmem<CAP>::kBytes * GROUPS;
+    CK(cudaFuncSetAttribute(k_merge_rows<NW, GROUPS, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 8);
+    LAUNCH(name, s, k_merge_rows<NW, GROUPS, CAP><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
+        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
     return SPGEMM_OK;
 }
 
@@ -494,6 +506,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
         p->stage_cap = std::min<int64_t>(p->lim_max_L, p->n);
         TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * p->lim_max_deg, s));
+        p->lim_max_deg += 1;   // cnt[] holds R+1 offsets
+        TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * p->lim_max_deg, s));
         TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
         TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
         TRY(palloc(p, &p->row_counter, 1, s));
@@ -563,23 +577,12 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     if (cnt > 0)
         LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
                                                                                       p->chat_col, p->chat_val, p->ccount));
-    rows = rows_of(kRowBucketWarpRadix, kRowBucketWarpRadix + 1, &cnt);
-    if (cnt > 0) {
-        CK(cudaFuncSetAttribute(k_merge_warp_radix, cudaFuncAttributeMaxDynamicSharedMemorySize, kWarpRadixSmem));
-        LAUNCH("merge_warp_radix", s, k_merge_warp_radix<<<(unsigned)cdiv(cnt, kWarpRadixWarps), kWarpRadixWarps * 32,
-                                                           kWarpRadixSmem, s>>>(rows, cnt, p->rowoff, p->chat_col,
-                                                                                p->chat_val, p->ccount));
-    }
-    rows = rows_of(kRowBucketCtaRadix, kRowBucketCtaRadix + 1, &cnt);
-    if (cnt > 0) {
-        constexpr int CAP = 4096;
-        const int smem = CAP * 16 + kCtaRadixWarps * 256 * 4;
-        CK(cudaFuncSetAttribute(k_merge_cta_radix<CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        LAUNCH("merge_cta_radix", s, k_merge_cta_radix<CAP><<<(unsigned)std::min<int64_t>(cnt, (int64_t)p->num_sms * 3 * 16),
-                                                               kCtaRadixThreads, smem, s>>>(rows, cnt, p->rowoff,
-                                                                                            p->chat_col, p->chat_val,
-                                                                                            p->ccount));
-    }
+    rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
+    TRY(launch_sort_bin<1, 8, 256>(p, s, rows, cnt, "merge_sort256", 5));
+    rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
+    TRY(launch_sort_bin<2, 4, 1024>(p, s, rows, cnt, "merge_sort1k", 2));
+    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+    TRY(launch_sort_bin<8, 1, 4096>(p, s, rows, cnt, "merge_sort4k", 2));
     if (p->nlim > 0) {
         CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
         LimitedArgs g;
@@ -593,6 +596,7 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         g.chat_val = p->chat_val;
         g.ccount = p->ccount;
         g.scratch_cursor = p->scr_cursor;
+        g.scratch_cnt = p->scr_cnt;
         g.scratch_col = p->scr_col;
         g.scratch_val = p->scr_val;
         g.max_deg = p->lim_max_deg;
@@ -683,8 +687,8 @@ int spgemm_get_stats(spgemm_plan_t p, spgemm_stats_t *st) {
     st->n_rows_bin[0] = p->row_starts[kRowBucketEmpty + 1] - p->row_starts[kRowBucketEmpty];
     st->n_rows_bin[1] = p->row_starts[kRowBucketPass + 1] - p->row_starts[kRowBucketPass];
     st->n_rows_bin[2] = p->row_starts[kRowBucketWarp + 1] - p->row_starts[kRowBucketWarp];
-    st->n_rows_bin[3] = p->row_starts[kRowBucketWarpRadix + 1] - p->row_starts[kRowBucketWarpRadix];
-    st->n_rows_bin[4] = p->row_starts[kRowBucketCtaRadix + 1] - p->row_starts[kRowBucketCtaRadix];
+    st->n_rows_bin[3] = p->row_starts[kRowBucketSort1K + 1] - p->row_starts[kRowBucketSort256];
+    st->n_rows_bin[4] = p->row_starts[kRowBucketSort4K + 1] - p->row_starts[kRowBucketSort4K];
     st->n_rows_bin[5] = p->nlim;
     st->bytes_workspace = p->bytes;
     return SPGEMM_OK;

@@ -193,18 +193,32 @@ def test_integer_values_exact():
     np.testing.assert_array_equal(C.val.cpu().numpy().astype(np.float64), val)   # exact
 
 
-def test_wide_limited_rows_span_many_windows():
-    """Rows whose Ĉ bucket is longer than the non-limited capacity and whose column span
-    covers several 16384-column windows of the B-Limited merge."""
-    rng = np.random.default_rng(3)
-    m, k, n = 40, 120, 70000
-    ar, ac = np.nonzero(rng.random((m, k)) < 0.25)
-    br = np.repeat(np.arange(k), 300)
-    bc = np.concatenate([np.sort(rng.choice(n, 300, replace=False)) for _ in range(k)])
-    # a few narrow-span hub columns so that equal columns collide heavily
-    bc[:300] = np.arange(300) * 3
-    inp = synth.from_coo("wide", m, k, n, (ar, ac, synth.edge_values(ar, ac, 1)),
-                         (br, bc, synth.edge_values(br, bc, 2)))
+def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False):
+    rng = np.random.default_rng(seed)
+    ar, ac = np.nonzero(rng.random((m, k)) < a_density)
+    br = np.repeat(np.arange(k), run_len)
+    cols = []
+    for q in range(k):
+        c = rng.choice(np.arange(1, n) if hub_col else n, run_len - (1 if hub_col else 0), replace=False)
+        if hub_col:
+            c = np.concatenate([[0], c])
+        cols.append(np.sort(c))
+    bc = np.concatenate(cols)
+    if narrow:
+        bc[:run_len] = np.arange(run_len) * 3
+    return synth.from_coo("wide", m, k, n, (ar, ac, synth.edge_values(ar, ac, seed)),
+                          (br, bc, synth.edge_values(br, bc, seed + 1)))
+
+
+@pytest.mark.parametrize("m,k,n,dens,run_len,hub,narrow", [
+    (40, 120, 70000, 0.25, 300, False, True),     # limited rows ~9K: in-smem path and sparse windows
+    (24, 200, 400000, 0.5, 200, False, False),     # sparse long rows: several smem windows
+    (16, 100, 30000, 0.3, 2000, False, False),     # dense rows: fp64 column windows
+    (2, 10000, 1000000, 1.0, 21, True, False),     # column 0 in 10000 runs: single-column overflow
+])
+def test_limited_paths(m, k, n, dens, run_len, hub, narrow):
+    """B-Limited merge: rows longer than the non-limited capacity, through every sub-path."""
+    inp = _wide_inputs(m, k, n, dens, run_len, 3, hub_col=hub, narrow=narrow)
     A, B = spg.from_inputs(inp, "cuda")
     with spg.Plan(A, B) as p:
         st = p.stats()
