@@ -275,12 +275,13 @@ def main():
         h2d = sum(t.numel() * t.element_size() for t in (Ah.colptr, Ah.rowidx, Ah.val, Bh.rowptr, Bh.colidx, Bh.val))
         es = []
         d2h = 0
+        pool = spg.HostBufferPool()
         for it in range(1 + max(1, args.steps // 2)):
             flush_l2(flush)
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             with spg.Plan(Ah, Bh, stream=stream, **opts) as p:
-                Ch = p.execute(device="cpu")
+                Ch = p.execute(device="cpu", pool=pool)
             torch.cuda.synchronize()
             dt = time.perf_counter() - t0
             d2h = sum(t.numel() * t.element_size() for t in (Ch.rowptr, Ch.colidx, Ch.val))

@@ -196,14 +196,18 @@ class Plan:
         _check(lib().spgemm_output(self.h, ctypes.byref(c), self.stream))
         return out
 
-    def execute(self, device=None) -> CSR:
-        """spgemm_execute: expand + merge + allocate C through a callback + compaction."""
+    def execute(self, device=None, pool: "Optional[HostBufferPool]" = None) -> CSR:
+        """spgemm_execute: expand + merge + allocate C through a callback + compaction.
+        With device='cpu', C lands in pinned host memory (from `pool` when given)."""
         dev = torch.device("cuda") if device is None else torch.device(device)
         where = SPGEMM_HOST if dev.type == "cpu" else SPGEMM_DEVICE
         bufs = []
 
         def _alloc(nbytes, w, ctx):
-            t = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=dev, pin_memory=(w == SPGEMM_HOST))
+            if pool is not None and w == SPGEMM_HOST:
+                t = pool.get(len(bufs), max(int(nbytes), 1))
+            else:
+                t = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=dev, pin_memory=(w == SPGEMM_HOST))
             bufs.append(t)
             return t.data_ptr()
 
@@ -244,6 +248,20 @@ class Plan:
             self.destroy()
         except Exception:
             pass
+
+
+class HostBufferPool:
+    """Reusable pinned host buffers for repeated host-output calls (C rowptr / colidx / val)."""
+
+    def __init__(self):
+        self.bufs = {}
+
+    def get(self, slot: int, nbytes: int) -> torch.Tensor:
+        b = self.bufs.get(slot)
+        if b is None or b.numel() < nbytes:
+            b = torch.empty(int(nbytes * 1.25) + 64, dtype=torch.uint8, pin_memory=True)
+            self.bufs[slot] = b
+        return b[:nbytes]
 
 
 def matmul(A: CSC, B: CSR, device=None, stream=None, **opts) -> CSR:

@@ -248,6 +248,180 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
     return total;
 }
 
+// ------------------------------------------------------------- bucket sort + reduce ---
+// MSD counting sort of one row by a group of T threads, then fp64 segmented reduction:
+//   1. each thread loads EPT elements (striped) into registers; min/max of the columns;
+//   2. nb = 2^ceil(log2 L) buckets over the column span, bucket = (col - min) >> sh;
+//      histogram with shared-memory integer atomics, exclusive scan (each thread owns a
+//      contiguous range of buckets);
+//   3. scatter by atomic rank into dk/dv; every bucket now holds the keys of a 2^sh-wide
+//      column range (on average < 2 elements), finished by an insertion sort;
+//   4. each thread walks its buckets in order and reduces equal columns in fp64, compacting
+//      in place inside its own bucket range; warps then copy their contiguous output slice
+//      to global memory with coalesced stores.
+// Equal columns always share a bucket, so no segment crosses a thread's range.  A bucket with
+// more than kBucketMax entries (many distinct columns packed into a narrow range) makes the
+// function return -1 before anything is written; the caller falls back to the natural merge sort.
+constexpr int kBucketMax = 64;
+
+__device__ __forceinline__ int nextpow2_log(int x) { return x <= 1 ? 0 : 32 - __clz(x - 1); }
+
+// Copy a warp's contiguous output slice: lane l staged u_l entries at (sk, sv)[st_l ..) and
+// they go to out[wbase + ex_l ..), ex_l = exclusive prefix of u over the warp's lanes.
+__device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const int32_t *sk, const float *sv,
+                                             int32_t *__restrict__ out_col, float *__restrict__ out_val) {
+    const int lane = lane_id();
+    const int inc = warp_incl_sum(u);
+    const int ex = inc - u;
+    const int wtot = __shfl_sync(kFull, inc, 31);
+    for (int o = lane; o < wtot; o += 32) {
+        int pos = 0;   // owner = number of lanes with inc <= o
+#pragma unroll
+        for (int step = 16; step > 0; step >>= 1) {
+            const int probe = __shfl_sync(kFull, inc, min(pos + step - 1, 31));
+            if (pos + step <= 32 && probe <= o) pos += step;
+        }
+        const int owner = min(pos, 31);
+        const int src = __shfl_sync(kFull, st, owner) + (o - __shfl_sync(kFull, ex, owner));
+        out_col[wbase + o] = sk[src];
+        out_val[wbase + o] = sv[src];
+    }
+    return wtot;
+}
+
+template <int NW, int GROUPS, int EPT>
+__device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
+                                                  int L, int32_t *dk, float *dv, int *hist, int32_t *out_col,
+                                                  float *out_val, int *sc) {
+    constexpr int T = NW * 32;
+    int32_t key[EPT];
+    float val[EPT];
+    int32_t mn = kKeyPad, mx = 0;
+#pragma unroll
+    for (int e = 0; e < EPT; ++e) {
+        const int p = g.gtid + e * T;
+        key[e] = p < L ? sk[p] : kKeyPad;
+        val[e] = p < L ? sv[p] : 0.f;
+        if (p < L) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
+    }
+    mn = g.reduce_min(mn, sc);
+    mx = g.reduce_max(mx, sc);
+    const uint32_t span = (uint32_t)(mx - mn);
+    const int lognb = nextpow2_log(L);
+    const int nb = 1 << lognb;
+    const int bits = span ? 32 - __clz(span) : 0;
+    const int sh = max(0, bits - lognb);
+    for (int b = g.gtid; b < nb; b += T) hist[b] = 0;
+    g.sync();
+#pragma unroll
+    for (int e = 0; e < EPT; ++e)
+        if (g.gtid + e * T < L) atomicAdd(&hist[(key[e] - mn) >> sh], 1);
+    g.sync();
+    const int bpt = (nb + T - 1) / T;
+    const int b0 = min(nb, g.gtid * bpt), b1 = min(nb, b0 + bpt);
+    int cnt = 0, mxc = 0;
+    for (int b = b0; b < b1; ++b) {
+        const int c = hist[b];
+        cnt += c;
+        mxc = max(mxc, c);
+    }
+    int tot;
+    int ex = g.excl_sum(cnt, sc, &tot);
+    if (g.reduce_max(mxc, sc) > kBucketMax) return -1;
+    const int my_start = ex;
+    for (int b = b0; b < b1; ++b) {
+        const int c = hist[b];
+        hist[b] = ex;
+        ex += c;
+    }
+    g.sync();
+#pragma unroll
+    for (int e = 0; e < EPT; ++e) {
+        if (g.gtid + e * T < L) {
+            const int pos = atomicAdd(&hist[(key[e] - mn) >> sh], 1);
+            dk[pos] = key[e];
+            dv[pos] = val[e];
+        }
+    }
+    g.sync();
+    // hist[b] now = end of bucket b.  Sort + reduce my buckets, compacting in place.
+    int w = my_start;
+    int start = my_start;
+    for (int b = b0; b < b1; ++b) {
+        const int end = hist[b];
+        for (int q = start + 1; q < end; ++q) {       // insertion sort (buckets are tiny)
+            const int32_t kk = dk[q];
+            const float vv = dv[q];
+            int j = q;
+            while (j > start && dk[j - 1] > kk) {
+                dk[j] = dk[j - 1];
+                dv[j] = dv[j - 1];
+                --j;
+            }
+            dk[j] = kk;
+            dv[j] = vv;
+        }
+        int q = start;
+        while (q < end) {
+            const int32_t kk = dk[q];
+            double acc = (double)dv[q];
+            ++q;
+            while (q < end && dk[q] == kk) acc += (double)dv[q++];
+            dk[w] = kk;
+            dv[w] = (float)acc;
+            ++w;
+        }
+        start = end;
+    }
+    const int u = w - my_start;
+    int U;
+    const int off = g.excl_sum(u, sc, &U);
+    __syncwarp();
+    const int64_t wbase = __shfl_sync(kFull, off, 0);
+    warp_copy_out(my_start, u, wbase, dk, dv, out_col, out_val);
+    return U;
+}
+
+constexpr int ceil_pow2(int x) { return x <= 1 ? 1 : 2 * ceil_pow2((x + 1) / 2); }
+
+template <int NW, int EPT>
+struct BucketSmem {
+    static constexpr int kCap = NW * 32 * EPT;
+    static constexpr int kNb = ceil_pow2(kCap);
+    static constexpr int kBytes = kCap * 8 + kNb * 4;
+};
+
+// Rows of one bin: bucket sort per row; rows whose buckets overflow go to a fallback list.
+template <int NW, int GROUPS, int EPT>
+__global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_bucket(const int32_t *__restrict__ rows, int64_t nrows,
+                                                                  const int64_t *__restrict__ rowoff,
+                                                                  int32_t *__restrict__ chat_col,
+                                                                  float *__restrict__ chat_val,
+                                                                  int64_t *__restrict__ ccount,
+                                                                  int32_t *__restrict__ fb_rows,
+                                                                  unsigned *__restrict__ fb_count) {
+    using S = BucketSmem<NW, EPT>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ int sc_all[GROUPS][NW + 1];
+    const Group<NW, GROUPS> g;
+    unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
+    int32_t *dk = (int32_t *)slice;
+    float *dv = (float *)(slice + S::kCap * 4);
+    int *hist = (int *)(slice + S::kCap * 8);
+    for (int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
+        const int i = rows[r];
+        const int64_t s = rowoff[i];
+        const int L = (int)(rowoff[i + 1] - s);
+        const int U = bucket_sort_reduce<NW, GROUPS, EPT>(g, chat_col + s, chat_val + s, L, dk, dv, hist,
+                                                          chat_col + s, chat_val + s, sc_all[g.gid]);
+        if (g.gtid == 0) {
+            if (U >= 0) ccount[i] = U;
+            else fb_rows[atomicAdd(fb_count, 1u)] = i;
+        }
+        g.sync();
+    }
+}
+
 // Load Ĉ[s, s+L) into smem (cp.async), sort, reduce, write the merged row back to Ĉ[s, ...).
 template <int NW, int GROUPS, int CAP>
 __device__ __forceinline__ int merge_row_in_smem(const Group<NW, GROUPS> &g, unsigned char *slice, int *sc,
@@ -278,7 +452,9 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
                                                                 const int64_t *__restrict__ rowoff,
                                                                 int32_t *__restrict__ chat_col,
                                                                 float *__restrict__ chat_val,
-                                                                int64_t *__restrict__ ccount) {
+                                                                int64_t *__restrict__ ccount,
+                                                                const unsigned *__restrict__ dev_count) {
+    if (dev_count) nrows = *dev_count;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ int sc_all[GROUPS][NW + 1];
     const Group<NW, GROUPS> g;
@@ -309,6 +485,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
 constexpr int kLimThreads = 512;
 constexpr int kLimNW = kLimThreads / 32;
 constexpr int kLimCap = 9216;
+constexpr int kLimEPT = kLimCap / kLimThreads;   // 18
 constexpr int kLimWindow = 16384;
 constexpr int kLimSmem = SortSmem<kLimCap>::kBytes > kLimWindow * 8 + (kLimWindow / 32) * 4
                              ? SortSmem<kLimCap>::kBytes
@@ -375,9 +552,16 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t s = g.rowoff[i];
         const int64_t L = g.rowoff[i + 1] - s;
         if (L <= kLimCap) {
-            const int U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)L,
-                                                                g.chat_col + s, g.chat_val + s);
+            int32_t *dk = (int32_t *)smem_raw;
+            float *dv = (float *)(smem_raw + kLimCap * 4);
+            int *hist = (int *)(smem_raw + kLimCap * 8);
+            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)L, dk, dv, hist,
+                                                            g.chat_col + s, g.chat_val + s, sc);
+            if (U < 0)
+                U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)L,
+                                                          g.chat_col + s, g.chat_val + s);
             if (threadIdx.x == 0) g.ccount[i] = U;
+            __syncthreads();
             continue;
         }
         const int64_t rs = g.run_start[r];
@@ -544,13 +728,17 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 cp_async_wait_all();
                 __syncthreads();
-                int32_t *k1 = (int32_t *)(smem_raw + kLimCap * 8);
-                float *v1 = (float *)(smem_raw + kLimCap * 12);
-                int *bA = (int *)(smem_raw + kLimCap * 16);
-                int *bB = bA + SortSmem<kLimCap>::kBoundsA;
-                const int which = natural_merge_sort<kLimNW, 1, kLimCap>(grp, k0, v0, k1, v1, bA, bB, total, sc);
-                const int U = segmented_reduce_out<kLimNW, 1>(grp, which ? k1 : k0, which ? v1 : v0, total,
-                                                              st_col + nout, st_val + nout, sc);
+                int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, k0, v0, total, k0, v0, (int *)(smem_raw + kLimCap * 8),
+                                                                st_col + nout, st_val + nout, sc);
+                if (U < 0) {
+                    int32_t *k1 = (int32_t *)(smem_raw + kLimCap * 8);
+                    float *v1 = (float *)(smem_raw + kLimCap * 12);
+                    int *bA = (int *)(smem_raw + kLimCap * 16);
+                    int *bB = bA + SortSmem<kLimCap>::kBoundsA;
+                    const int which = natural_merge_sort<kLimNW, 1, kLimCap>(grp, k0, v0, k1, v1, bA, bB, total, sc);
+                    U = segmented_reduce_out<kLimNW, 1>(grp, which ? k1 : k0, which ? v1 : v0, total,
+                                                        st_col + nout, st_val + nout, sc);
+                }
                 __syncthreads();
                 nout += U;
                 remaining -= total;

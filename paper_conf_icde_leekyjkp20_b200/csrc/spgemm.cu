@@ -149,6 +149,8 @@ struct spgemm_plan_s {
     int32_t *chat_col = nullptr;
     float *chat_val = nullptr;
     int64_t *ccount = nullptr, *crowptr = nullptr;
+    int32_t *fb_rows = nullptr;
+    unsigned *fb_count = nullptr;
     int64_t nnz_c = -1;
     int state = 0;  // 1 planned, 2 expanded, 3 merged
 };
@@ -228,15 +230,15 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     return SPGEMM_OK;
 }
 
-template <int NW, int GROUPS, int CAP>
-static int launch_sort_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
-                           int ctas_per_sm) {
+template <int NW, int GROUPS, int EPT>
+static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
+                             int ctas_per_sm) {
     if (cnt == 0) return SPGEMM_OK;
-    const int smem = SortSmem<CAP>::kBytes * GROUPS;
-    CK(cudaFuncSetAttribute(k_merge_rows<NW, GROUPS, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 8);
-    LAUNCH(name, s, k_merge_rows<NW, GROUPS, CAP><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
-        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
+    const int smem = BucketSmem<NW, EPT>::kBytes * GROUPS;
+    CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
+    LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
+        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
     return SPGEMM_OK;
 }
 
@@ -516,6 +518,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     TRY(palloc(p, &p->chat_col, p->nnz_chat, s));
     TRY(palloc(p, &p->chat_val, p->nnz_chat, s));
     TRY(palloc(p, &p->ccount, M, s));
+    TRY(palloc(p, &p->fb_rows, M, s));
+    TRY(palloc(p, &p->fb_count, 1, s));
     TRY(palloc(p, &p->crowptr, M + 1, s));
     p->state = 1;
     return SPGEMM_OK;
@@ -577,12 +581,20 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     if (cnt > 0)
         LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
                                                                                       p->chat_col, p->chat_val, p->ccount));
+    CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
     rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-    TRY(launch_sort_bin<1, 8, 256>(p, s, rows, cnt, "merge_sort256", 5));
+    TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
     rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-    TRY(launch_sort_bin<2, 4, 1024>(p, s, rows, cnt, "merge_sort1k", 2));
+    TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
     rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-    TRY(launch_sort_bin<8, 1, 4096>(p, s, rows, cnt, "merge_sort4k", 2));
+    TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    {   // rows whose buckets overflowed: natural merge sort (count read on the device)
+        constexpr int CAP = 4096;
+        const int smem = SortSmem<CAP>::kBytes;
+        CK(cudaFuncSetAttribute(k_merge_rows<8, 1, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
+            p->fb_rows, 0, p->rowoff, p->chat_col, p->chat_val, p->ccount, p->fb_count));
+    }
     if (p->nlim > 0) {
         CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
         LimitedArgs g;

@@ -229,6 +229,28 @@ def test_limited_paths(m, k, n, dens, run_len, hub, narrow):
     assert_c_matches(C, inp)
 
 
+@pytest.mark.parametrize("k,cluster,spread", [(10, 20, 10), (40, 40, 60), (60, 100, 2)])
+def test_clustered_columns_fallback(k, cluster, spread):
+    """Rows whose columns cluster in a narrow range of a wide span overflow the bucket sort's
+    buckets; the natural merge sort fallback (and the limited kernel's inline fallback) take them."""
+    rng = np.random.default_rng(5)
+    m, n = 6, 1_000_000
+    ar, ac = np.nonzero(np.ones((m, k), dtype=bool))
+    br, bc = [], []
+    for q in range(k):
+        c = np.concatenate([np.arange(q * cluster, (q + 1) * cluster),
+                            rng.choice(np.arange(10 ** 5, n), spread, replace=False)])
+        c = np.unique(c)
+        br.append(np.full(c.size, q))
+        bc.append(c)
+    br, bc = np.concatenate(br), np.concatenate(bc)
+    inp = synth.from_coo("clustered", m, k, n, (ar, ac, synth.edge_values(ar, ac, 1)),
+                         (br, bc, synth.edge_values(br, bc, 2)))
+    A, B = spg.from_inputs(inp, "cuda")
+    C = spg.matmul(A, B)
+    assert_c_matches(C, inp)
+
+
 def test_empty_and_degenerate():
     for shape in [(5, 0, 7), (0, 4, 3), (3, 4, 0)]:
         m, k, n = shape
