@@ -274,7 +274,8 @@ __device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const
     const int inc = warp_incl_sum(u);
     const int ex = inc - u;
     const int wtot = __shfl_sync(kFull, inc, 31);
-    for (int o = lane; o < wtot; o += 32) {
+    for (int o0 = 0; o0 < wtot; o0 += 32) {      // warp-uniform trip count (shuffles below)
+        const int o = o0 + lane;
         int pos = 0;   // owner = number of lanes with inc <= o
 #pragma unroll
         for (int step = 16; step > 0; step >>= 1) {
@@ -283,8 +284,10 @@ __device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const
         }
         const int owner = min(pos, 31);
         const int src = __shfl_sync(kFull, st, owner) + (o - __shfl_sync(kFull, ex, owner));
-        out_col[wbase + o] = sk[src];
-        out_val[wbase + o] = sv[src];
+        if (o < wtot) {
+            out_col[wbase + o] = sk[src];
+            out_val[wbase + o] = sv[src];
+        }
     }
     return wtot;
 }
@@ -765,28 +768,75 @@ __global__ void k_merge_pass(const int32_t *__restrict__ rows, int64_t nrows, co
 }
 
 // ------------------------------------------------------------------ CSR compaction ---
-// Output entry q of C belongs to row r with crowptr[r] <= q < crowptr[r+1]; it is read from
-// Ĉ[rowoff[r] + q - crowptr[r]].  Tiles of 2048 outputs per block, rows found by binary search.
-constexpr int kCompactThreads = 256;
-constexpr int kCompactTile = 2048;
+// Row i's merged entries sit at Ĉ[rowoff[i] ..) and move to C[crowptr[i] ..).  One warp per
+// row (4 loads in flight per lane); rows longer than kCompactWarpMax get a CTA each.
+constexpr int kCompactWarpMax = 8192;
+constexpr int kCompactLongThreads = 512;
 
-__global__ void __launch_bounds__(kCompactThreads) k_compact(const int64_t *__restrict__ crowptr, int64_t M,
-                                                             const int64_t *__restrict__ rowoff,
-                                                             const int32_t *__restrict__ chat_col,
-                                                             const float *__restrict__ chat_val, int64_t nnz_c,
-                                                             int32_t *__restrict__ out_col, float *__restrict__ out_val) {
-    __shared__ int64_t lohi[2];
-    const int64_t q0 = (int64_t)blockIdx.x * kCompactTile;
-    const int64_t q1 = min(nnz_c, q0 + kCompactTile);
-    if (threadIdx.x == 0) lohi[0] = upper_bound_idx(crowptr, 0, M, q0);
-    if (threadIdx.x == 1) lohi[1] = upper_bound_idx(crowptr, 0, M, q1 - 1);
-    __syncthreads();
-    const int64_t lo = lohi[0], hi = lohi[1] + 1;
-    for (int64_t q = q0 + threadIdx.x; q < q1; q += kCompactThreads) {
-        const int64_t r = upper_bound_idx(crowptr, lo, hi, q);
-        const int64_t src = rowoff[r] + (q - crowptr[r]);
-        out_col[q] = chat_col[src];
-        out_val[q] = chat_val[src];
+__global__ void __launch_bounds__(256) k_compact_rows(const int64_t *__restrict__ crowptr, int64_t M,
+                                                      const int64_t *__restrict__ rowoff,
+                                                      const int32_t *__restrict__ chat_col,
+                                                      const float *__restrict__ chat_val,
+                                                      int32_t *__restrict__ out_col, float *__restrict__ out_val) {
+    const int lane = lane_id();
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < M;
+         i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t dst = crowptr[i];
+        const int64_t cnt = crowptr[i + 1] - dst;
+        if (cnt == 0 || cnt > kCompactWarpMax) continue;
+        const int64_t src = rowoff[i];
+        for (int p0 = 0; p0 < cnt; p0 += 128) {
+            int32_t c[4];
+            float v[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int p = p0 + q * 32 + lane;
+                c[q] = p < cnt ? chat_col[src + p] : 0;
+                v[q] = p < cnt ? chat_val[src + p] : 0.f;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int p = p0 + q * 32 + lane;
+                if (p < cnt) {
+                    out_col[dst + p] = c[q];
+                    out_val[dst + p] = v[q];
+                }
+            }
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kCompactLongThreads) k_compact_long(const int32_t *__restrict__ rows, int64_t nrows,
+                                                                      const int64_t *__restrict__ crowptr,
+                                                                      const int64_t *__restrict__ rowoff,
+                                                                      const int32_t *__restrict__ chat_col,
+                                                                      const float *__restrict__ chat_val,
+                                                                      int32_t *__restrict__ out_col,
+                                                                      float *__restrict__ out_val) {
+    for (int64_t r = blockIdx.x; r < nrows; r += gridDim.x) {
+        const int i = rows[r];
+        const int64_t dst = crowptr[i];
+        const int64_t cnt = crowptr[i + 1] - dst;
+        if (cnt <= kCompactWarpMax) continue;
+        const int64_t src = rowoff[i];
+        for (int64_t p0 = 0; p0 < cnt; p0 += 4 * kCompactLongThreads) {
+            int32_t c[4];
+            float v[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int64_t p = p0 + q * kCompactLongThreads + threadIdx.x;
+                c[q] = p < cnt ? chat_col[src + p] : 0;
+                v[q] = p < cnt ? chat_val[src + p] : 0.f;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int64_t p = p0 + q * kCompactLongThreads + threadIdx.x;
+                if (p < cnt) {
+                    out_col[dst + p] = c[q];
+                    out_val[dst + p] = v[q];
+                }
+            }
+        }
     }
 }
 

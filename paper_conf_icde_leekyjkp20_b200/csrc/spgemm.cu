@@ -643,9 +643,15 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
         TRY(talloc(p, t1, &dcol, nnz));
         TRY(talloc(p, t2, &dval, nnz));
     }
-    if (nnz > 0)
-        LAUNCH("compact", s, k_compact<<<(unsigned)cdiv(nnz, kCompactTile), kCompactThreads, 0, s>>>(
-            p->crowptr, p->m, p->rowoff, p->chat_col, p->chat_val, nnz, dcol, dval));
+    if (nnz > 0) {
+        LAUNCH("compact", s, k_compact_rows<<<grid_for(p->m * 32, 256, (int64_t)p->num_sms * 16), 256, 0, s>>>(
+            p->crowptr, p->m, p->rowoff, p->chat_col, p->chat_val, dcol, dval));
+        if (p->nlim > 0)
+            LAUNCH("compact", s, k_compact_long<<<(unsigned)std::min<int64_t>(p->nlim, (int64_t)p->num_sms * 4),
+                                                   kCompactLongThreads, 0, s>>>(
+                p->row_order + p->row_starts[kRowBucketLim0], p->nlim, p->crowptr, p->rowoff, p->chat_col,
+                p->chat_val, dcol, dval));
+    }
     if (C->where == SPGEMM_HOST) {
         CK(cudaMemcpyAsync(C->rowptr, p->crowptr, (p->m + 1) * 8, cudaMemcpyDeviceToHost, s));
         if (nnz > 0) {

@@ -251,6 +251,21 @@ def test_clustered_columns_fallback(k, cluster, spread):
     assert_c_matches(C, inp)
 
 
+def test_row_partition_and_row_blocks():
+    """spgemm_row_partition equals the oracle's balanced partition (R8), and C assembled from
+    independently computed row blocks (the multi-GPU decomposition) equals the oracle's C."""
+    from paper_conf_icde_leekyjkp20_b200 import dist as pdist
+    inp = synth.make_inputs("C1", seed=3)
+    A, B = spg.from_inputs(inp, "cuda")
+    rw = stages.row_workload(inp)
+    for parts in (1, 2, 3, 8):
+        np.testing.assert_array_equal(spg.row_partition(A, B, parts), stages.balanced_row_partition(rw, parts))
+    bounds = spg.row_partition(A, B, 4)
+    blocks = [spg.matmul(pdist.csc_row_slice(A, int(bounds[r]), int(bounds[r + 1])), B) for r in range(4)]
+    C = pdist.concat_row_blocks(blocks)
+    assert_c_matches(C, inp)
+
+
 def test_empty_and_degenerate():
     for shape in [(5, 0, 7), (0, 4, 3), (3, 4, 0)]:
         m, k, n = shape
