@@ -39,6 +39,9 @@ struct PlanScalars {
     unsigned long long m_nonempty;   // #rows with rowwork > 0
     unsigned long long max_rowwork;
     unsigned long long max_deg;      // max runs (A entries with nnz(b_k*) > 0) in a row
+    unsigned long long lim_runs;     // sum of runs over limited rows
+    unsigned long long lim_max_deg;  // max runs of a limited row
+    unsigned long long lim_max_L;    // max products of a limited row
     int invalid;                     // validation failure bits
     int pad;
 };
@@ -188,6 +191,25 @@ __global__ void k_partition_bounds(const int64_t *__restrict__ rowoff, int64_t M
 }
 
 // ---------------------------------------------------------------- stage (2) --------------
+struct SplitParams {
+    int64_t piece_work;
+    int32_t b_tile;
+    int32_t split_ca_max;
+};
+
+// Splitting factor f = 2^n (L410-L413 L): smallest power of two whose greedy chunk of
+// ceil(ca/f) column entries keeps a piece within piece_work products and split_ca_max
+// computations per thread.
+__device__ __forceinline__ int64_t splitting_factor(int64_t ca, int64_t blen, const SplitParams &p) {
+    int64_t f = 1;
+    while (f < ca) {
+        int64_t chunk = (ca + f - 1) / f;
+        if (chunk * blen <= p.piece_work && chunk <= p.split_ca_max) break;
+        f <<= 1;
+    }
+    return f;
+}
+
 struct ClassifyParams {
     int64_t t_dom;
     int32_t split_ca_max;
@@ -200,7 +222,8 @@ struct ClassifyParams {
 __global__ void __launch_bounds__(256) k_pair_classify(const int64_t *__restrict__ a_colptr,
                                                        const int64_t *__restrict__ b_rowptr,
                                                        const int64_t *__restrict__ work, int64_t K, ClassifyParams p,
-                                                       int8_t *__restrict__ cls, uint8_t *__restrict__ bucket) {
+                                                       SplitParams sp, int8_t *__restrict__ cls,
+                                                       uint8_t *__restrict__ bucket, int64_t *__restrict__ npieces) {
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x) {
         int64_t ca = a_colptr[k + 1] - a_colptr[k];
         int64_t rb = b_rowptr[k + 1] - b_rowptr[k];
@@ -228,40 +251,14 @@ __global__ void __launch_bounds__(256) k_pair_classify(const int64_t *__restrict
         }
         cls[k] = c;
         bucket[k] = (uint8_t)b;
-    }
-}
-
-struct SplitParams {
-    int64_t piece_work;
-    int32_t b_tile;
-    int32_t split_ca_max;
-};
-
-// Splitting factor f = 2^n (L410-L413 L): smallest power of two whose greedy chunk of
-// ceil(ca/f) column entries keeps a piece within piece_work products and split_ca_max
-// computations per thread.
-__device__ __forceinline__ int64_t splitting_factor(int64_t ca, int64_t blen, const SplitParams &p) {
-    int64_t f = 1;
-    while (f < ca) {
-        int64_t chunk = (ca + f - 1) / f;
-        if (chunk * blen <= p.piece_work && chunk <= p.split_ca_max) break;
-        f <<= 1;
-    }
-    return f;
-}
-
-__global__ void k_piece_count(const int32_t *__restrict__ dom, int64_t ndom, const int64_t *__restrict__ a_colptr,
-                              const int64_t *__restrict__ b_rowptr, SplitParams p, int64_t *__restrict__ npieces) {
-    for (int64_t d = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; d < ndom; d += (int64_t)gridDim.x * blockDim.x) {
-        int k = dom[d];
-        int64_t ca = a_colptr[k + 1] - a_colptr[k];
-        int64_t rb = b_rowptr[k + 1] - b_rowptr[k];
-        int64_t blen = min(rb, (int64_t)p.b_tile);
-        int64_t f = splitting_factor(ca, blen, p);
-        int64_t chunk = (ca + f - 1) / f;
-        int64_t npa = (ca + chunk - 1) / chunk;       // non-empty greedy pieces
-        int64_t nb = (rb + p.b_tile - 1) / p.b_tile;
-        npieces[d] = npa * nb;
+        int64_t np = 0;
+        if (b == kPairBucketSplit) {   // B-Splitting piece count (pieces are laid out in ascending k)
+            const int64_t blen = min(rb, (int64_t)sp.b_tile);
+            const int64_t f = splitting_factor(ca, blen, sp);
+            const int64_t chunk = (ca + f - 1) / f;
+            np = ((ca + chunk - 1) / chunk) * ((rb + sp.b_tile - 1) / sp.b_tile);
+        }
+        npieces[k] = np;
     }
 }
 
@@ -279,7 +276,7 @@ __global__ void k_piece_fill(const int32_t *__restrict__ dom, int64_t ndom, cons
     int64_t chunk = (ca + f - 1) / f;
     int64_t npa = (ca + chunk - 1) / chunk;
     int64_t nb = (rb + p.b_tile - 1) / p.b_tile;
-    int64_t base = piece_off[d];
+    int64_t base = piece_off[k];
     for (int64_t q = lane_id(); q < npa * nb; q += 32) {
         int64_t t = q / npa, a = q % npa;
         Piece pc;
@@ -314,20 +311,41 @@ __global__ void k_piece_whole(const int32_t *__restrict__ list, int64_t n, const
 // a row made of a single run (one A entry) is already sorted and duplicate-free.
 __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict__ rowwork,
                                                       const int32_t *__restrict__ deg, int64_t M, int64_t t_lim,
-                                                      int8_t *__restrict__ rcls, uint8_t *__restrict__ bucket) {
+                                                      int8_t *__restrict__ rcls, uint8_t *__restrict__ bucket,
+                                                      PlanScalars *sc) {
+    __shared__ unsigned long long sm[3][8];
+    unsigned long long runs = 0, mdeg = 0, mlen = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
         int64_t L = rowwork[i];
         int8_t c;
         int b;
         if (L == 0) { c = RC_EMPTY; b = kRowBucketEmpty; }
         else if (deg[i] == 1) { c = RC_PASS; b = kRowBucketPass; }
-        else if (L > t_lim) { c = RC_LIMITED; b = kRowBucketLim0 + (39 - min(39, ilog2_floor((uint64_t)L))); }
+        else if (L > t_lim) {
+            c = RC_LIMITED;
+            b = kRowBucketLim0 + (39 - min(39, ilog2_floor((uint64_t)L)));
+            runs += (unsigned long long)deg[i];
+            mdeg = max(mdeg, (unsigned long long)deg[i]);
+            mlen = max(mlen, (unsigned long long)L);
+        }
         else if (L <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
         else if (L <= kSort256Max) { c = RC_WARP_SORT; b = kRowBucketSort256; }
         else if (L <= kSort1KMax) { c = RC_WARP_SORT; b = kRowBucketSort1K; }
         else { c = RC_GROUP_SORT; b = kRowBucketSort4K; }
         rcls[i] = c;
         bucket[i] = (uint8_t)b;
+    }
+    runs = warp_sum(runs);
+    mdeg = warp_max(mdeg);
+    mlen = warp_max(mlen);
+    if (lane_id() == 0) { sm[0][warp_id()] = runs; sm[1][warp_id()] = mdeg; sm[2][warp_id()] = mlen; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long a = 0, b = 0, c = 0;
+        for (int w = 0; w < 8; ++w) { a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); }
+        if (a) atomicAdd(&sc->lim_runs, a);
+        if (b) atomicMax(&sc->lim_max_deg, b);
+        if (c) atomicMax(&sc->lim_max_L, c);
     }
 }
 

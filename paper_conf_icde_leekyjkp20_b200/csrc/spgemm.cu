@@ -433,6 +433,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     TRY(palloc(p, &p->piece_off, K + 1, s));
     int64_t *d_starts;
     TRY(palloc(p, &d_starts, kNumPairBuckets + kNumRowBuckets + 4, s));
+    SplitParams sp{o.piece_work, o.split_b_tile, o.split_ca_max};
     {
         Temp tb(s), tr(s), tn(s);
         uint8_t *pb, *rbk;
@@ -443,39 +444,32 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         ClassifyParams cp{p->t_dom, o.split_ca_max, o.enable_split, o.enable_gather};
         if (K > 0)
             LAUNCH("pair_classify", s, k_pair_classify<<<grid_for(K, 256), 256, 0, s>>>(p->a_colptr, p->b_rowptr, p->work, K,
-                                                                                    cp, p->pair_cls, pb));
+                                                                                    cp, sp, p->pair_cls, pb, npieces));
+        TRY(scan_excl(p, npieces, K, p->piece_off, s, "piece_scan"));
         TRY(partition(p, pb, K, kNumPairBuckets, p->pair_order, d_starts, s, "pair_partition"));
         if (M > 0)
             LAUNCH("row_classify", s, k_row_classify<<<grid_for(M, 256), 256, 0, s>>>(p->rowwork, p->deg, M, p->t_lim,
-                                                                                  p->row_cls, rbk));
+                                                                                  p->row_cls, rbk, p->scal));
         TRY(partition(p, rbk, M, kNumRowBuckets, p->row_order, d_starts + kNumPairBuckets + 1, s, "row_partition"));
         CK(cudaMemcpyAsync(p->pair_starts, d_starts, sizeof(int64_t) * (kNumPairBuckets + 1), cudaMemcpyDeviceToHost, s));
         CK(cudaMemcpyAsync(p->row_starts, d_starts + kNumPairBuckets + 1, sizeof(int64_t) * (kNumRowBuckets + 1),
                            cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));  // sync 2a: bin populations
-        // B-Splitting: piece counts of the dominators (ascending k), scan, fill
-        const int64_t ndom = p->pair_starts[kPairBucketSplit + 1] - p->pair_starts[kPairBucketSplit];
-        SplitParams sp{o.piece_work, o.split_b_tile, o.split_ca_max};
-        p->n_whole = p->pair_starts[kPairBucketPiece + 1] - p->pair_starts[kPairBucketPiece];
-        if (ndom > 0) {
-            const int32_t *dom = p->pair_order + p->pair_starts[kPairBucketSplit];
-            LAUNCH("piece_count", s, k_piece_count<<<grid_for(ndom, 128), 128, 0, s>>>(dom, ndom, p->a_colptr, p->b_rowptr,
-                                                                                   sp, npieces));
-            TRY(scan_excl(p, npieces, ndom, p->piece_off, s, "piece_scan"));
-            CK(cudaMemcpyAsync(&p->n_split_pieces, p->piece_off + ndom, 8, cudaMemcpyDeviceToHost, s));
-            CK(cudaStreamSynchronize(s));  // sync 2b: #pieces
-        }
-        TRY(palloc(p, &p->pieces, p->n_split_pieces + p->n_whole, s));
-        if (ndom > 0) {
-            const int32_t *dom = p->pair_order + p->pair_starts[kPairBucketSplit];
-            LAUNCH("piece_fill", s, k_piece_fill<<<(unsigned)cdiv(ndom * 32, 256), 256, 0, s>>>(
-                dom, ndom, p->a_colptr, p->b_rowptr, sp, p->piece_off, p->pieces));
-        }
-        if (p->n_whole > 0)
-            LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_whole, 256), 256, 0, s>>>(
-                p->pair_order + p->pair_starts[kPairBucketPiece], p->n_whole, p->a_colptr, p->b_rowptr,
-                p->pieces + p->n_split_pieces));
+        CK(cudaMemcpyAsync(&p->n_split_pieces, p->piece_off + K, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&p->h_scal, p->scal, sizeof(PlanScalars), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));  // sync 2: bin populations, #pieces, limited-row sizes
     }
+    const int64_t ndom = p->pair_starts[kPairBucketSplit + 1] - p->pair_starts[kPairBucketSplit];
+    p->n_whole = p->pair_starts[kPairBucketPiece + 1] - p->pair_starts[kPairBucketPiece];
+    TRY(palloc(p, &p->pieces, p->n_split_pieces + p->n_whole, s));
+    if (ndom > 0) {
+        const int32_t *dom = p->pair_order + p->pair_starts[kPairBucketSplit];
+        LAUNCH("piece_fill", s, k_piece_fill<<<(unsigned)cdiv(ndom * 32, 256), 256, 0, s>>>(
+            dom, ndom, p->a_colptr, p->b_rowptr, sp, p->piece_off, p->pieces));
+    }
+    if (p->n_whole > 0)
+        LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_whole, 256), 256, 0, s>>>(
+            p->pair_order + p->pair_starts[kPairBucketPiece], p->n_whole, p->a_colptr, p->b_rowptr,
+            p->pieces + p->n_split_pieces));
     // limited rows: index map, run lists, B-Limited scratch
     p->nlim = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketLim0];
     if (p->nlim > 0) {
@@ -493,13 +487,9 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
                                                                                   nruns));
             TRY(scan_excl(p, nruns, p->nlim, p->run_start, s, "lim_scan"));
         }
-        // sizes for the run lists and the per-block scratch (sync 3, small)
-        int64_t h[1];
-        CK(cudaMemcpyAsync(h, p->run_start + p->nlim, 8, cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
-        p->lim_runs = h[0];
-        p->lim_max_deg = (int64_t)p->h_scal.max_deg;
-        p->lim_max_L = (int64_t)p->h_scal.max_rowwork;
+        p->lim_runs = (int64_t)p->h_scal.lim_runs;
+        p->lim_max_deg = (int64_t)p->h_scal.lim_max_deg;
+        p->lim_max_L = (int64_t)p->h_scal.lim_max_L;
         TRY(palloc(p, &p->run_base, p->lim_runs, s));
         TRY(palloc(p, &p->run_len, p->lim_runs, s));
         LAUNCH("lim_runs", s, k_lim_runs<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
@@ -507,9 +497,9 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
             p->run_base, p->run_len));
         p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
         p->stage_cap = std::min<int64_t>(p->lim_max_L, p->n);
-        TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * p->lim_max_deg, s));
-        p->lim_max_deg += 1;   // cnt[] holds R+1 offsets
-        TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * p->lim_max_deg, s));
+        TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
+        TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
+        p->lim_max_deg += 1;   // per-block stride of the cursor / cnt scratch (cnt holds R+1 offsets)
         TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
         TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
         TRY(palloc(p, &p->row_counter, 1, s));
