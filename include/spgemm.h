@@ -96,9 +96,10 @@ typedef struct {
  * Paper parameters keep the paper's names (α, β); DESIGN.md §2 R1-R8 gives the readings. */
 typedef struct {
     double alpha;             /* >0: Dominator threshold nnz(Ĉ)/(#pair blocks × α) (L309-L311 R);
-                                 0: B200 default max(dom_min_work, nnz(Ĉ)/(#SMs × dom_waves))   */
+                                 0: B200 default clamp(nnz(Ĉ)/(#SMs × dom_waves),
+                                    dom_min_work, piece_work)                                   */
     int32_t dom_waves;        /* B200 default: fair-share divisor per SM (default 16)           */
-    int64_t dom_min_work;     /* lower bound of the B200 Dominator threshold (default 32768)    */
+    int64_t dom_min_work;     /* lower bound of the B200 Dominator threshold (default 4096)     */
     int32_t split_ca_max;     /* max computations per thread nnz(a_*k) of a piece (default 256) */
     int64_t piece_work;       /* max products of one B-Splitting piece (default 16384)          */
     int32_t split_b_tile;     /* max B-row entries per piece (default 4096)                     */

@@ -53,14 +53,15 @@ def chat_row_offsets(rowwork):
 # --- (2) categorisation (L304-L318 R) ------------------------------------------------------
 
 def dominator_threshold(nnz_chat: int, k_nonempty: int, alpha: float, num_sms: int,
-                        dom_waves: int, dom_min_work: int) -> int:
+                        dom_waves: int, dom_min_work: int, piece_work: int) -> int:
     """threshold = nnz(Ĉ)/(#blocks × α)  (L309-L311 R) when α > 0, with #blocks the number
-    of non-empty pair blocks (R1).  α = 0 selects the B200 re-derivation (R2):
-    max(dom_min_work, ceil(nnz(Ĉ) / (#SMs × dom_waves)))."""
+    of non-empty pair blocks (R1).  α = 0 selects the B200 re-derivation (R2): a block is
+    overloaded when it exceeds the per-SM fair share ceil(nnz(Ĉ)/(#SMs × dom_waves)), clamped
+    to [dom_min_work, piece_work] so that no unsplit block is larger than a split piece."""
     if alpha > 0:
         return int(math.floor(float(nnz_chat) / (float(max(k_nonempty, 1)) * alpha)))
     share = -(-int(nnz_chat) // int(num_sms * dom_waves))
-    return int(max(dom_min_work, share))
+    return int(min(piece_work, max(dom_min_work, share)))
 
 
 def classify_pairs(ca, rb, work, t_dom: int, split_ca_max: int):

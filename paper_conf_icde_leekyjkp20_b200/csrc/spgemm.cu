@@ -254,7 +254,7 @@ void spgemm_default_options(spgemm_options_t *o) {
     memset(o, 0, sizeof(*o));
     o->alpha = 0.0;
     o->dom_waves = 16;
-    o->dom_min_work = 32768;
+    o->dom_min_work = 4096;
     o->split_ca_max = 256;
     o->piece_work = 16384;
     o->split_b_tile = 4096;
@@ -417,7 +417,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     if (o.alpha > 0)
         p->t_dom = (int64_t)std::floor((double)p->nnz_chat / ((double)std::max<uint64_t>(p->h_scal.k_nonempty, 1) * o.alpha));
     else
-        p->t_dom = std::max<int64_t>(o.dom_min_work, cdiv(p->nnz_chat, (int64_t)p->num_sms * o.dom_waves));
+        p->t_dom = std::min<int64_t>(o.piece_work, std::max<int64_t>(o.dom_min_work,
+                                                                     cdiv(p->nnz_chat, (int64_t)p->num_sms * o.dom_waves)));
     const int64_t cap = 4096;
     if (o.beta > 0)
         p->t_lim = std::min<int64_t>(cap, (int64_t)std::floor((double)p->nnz_chat /

@@ -94,7 +94,7 @@ def test_stage2_reorganizer(name, opts):
     st = p.stats()
     ca, rb, work = stages.pair_workload(inp)
     t_dom = stages.dominator_threshold(int(work.sum()), int((work > 0).sum()), o.alpha, _sms(), o.dom_waves,
-                                       o.dom_min_work)
+                                       o.dom_min_work, o.piece_work)
     assert st["t_dom"] == t_dom
     cls = stages.classify_pairs(ca, rb, work, t_dom, o.split_ca_max)
     np.testing.assert_array_equal(p.inspect(spg.VIEW_PAIR_CLASS, np.int8), cls)

@@ -248,7 +248,7 @@ def test_identity_special_case():
 def test_pieces_tile_dominators_exactly(piece_work, b_tile, ca_max):
     inp = synth.make_inputs("C1", seed=4)
     ca, rb, work = stages.pair_workload(inp)
-    t = stages.dominator_threshold(int(work.sum()), int((work > 0).sum()), 0.0, 148, 4, 2000)
+    t = stages.dominator_threshold(int(work.sum()), int((work > 0).sum()), 0.0, 148, 4, 2000, 16384)
     cls = stages.classify_pairs(ca, rb, work, t, ca_max)
     pieces = stages.split_pieces(inp, cls, piece_work, b_tile, ca_max)
     doms = np.nonzero(cls == stages.DOMINATOR)[0]
@@ -292,8 +292,10 @@ def test_balanced_row_partition():
 
 def test_thresholds_formulas():
     # paper form: nnz(Ĉ)/(#blocks × α)  (L309-L311 R),  nnz(Ĉ)/(#blocks × β) with β = 10 (L475-L477 L)
-    assert stages.dominator_threshold(1000, 10, 2.0, 148, 4, 0) == 50
-    assert stages.dominator_threshold(10 ** 9, 10, 0.0, 148, 4, 0) == -(-10 ** 9 // 592)
+    assert stages.dominator_threshold(1000, 10, 2.0, 148, 4, 0, 16384) == 50
+    assert stages.dominator_threshold(10 ** 7, 10, 0.0, 148, 4, 0, 10 ** 9) == -(-10 ** 7 // 592)
+    assert stages.dominator_threshold(10 ** 9, 10, 0.0, 148, 4, 0, 16384) == 16384      # clamped to a piece
+    assert stages.dominator_threshold(10 ** 3, 10, 0.0, 148, 4, 4096, 16384) == 4096    # floor
     assert stages.limiting_threshold(100000, 100, 10.0, 4096) == 100
     assert stages.limiting_threshold(10 ** 9, 100, 10.0, 4096) == 4096
     assert stages.limiting_threshold(10 ** 9, 100, 0.0, 4096) == 4096
