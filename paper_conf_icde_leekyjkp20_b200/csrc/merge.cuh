@@ -294,8 +294,8 @@ __device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const
 
 template <int NW, int GROUPS, int EPT>
 __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
-                                                  int L, int32_t *dk, float *dv, int *hist, int32_t *out_col,
-                                                  float *out_val, int *sc) {
+                                                  int L, int32_t *dk, float *dv, int32_t *dk2, float *dv2,
+                                                  int *hist, int32_t *out_col, float *out_val, int *sc) {
     constexpr int T = NW * 32;
     int32_t key[EPT];
     float val[EPT];
@@ -331,57 +331,64 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     int tot;
     int ex = g.excl_sum(cnt, sc, &tot);
     if (g.reduce_max(mxc, sc) > kBucketMax) return -1;
-    const int my_start = ex;
     for (int b = b0; b < b1; ++b) {
         const int c = hist[b];
         hist[b] = ex;
         ex += c;
     }
     g.sync();
+    // 1. scatter by atomic rank (unordered inside a bucket)
+    int pos[EPT];
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
+        pos[e] = -1;
         if (g.gtid + e * T < L) {
-            const int pos = atomicAdd(&hist[(key[e] - mn) >> sh], 1);
-            dk[pos] = key[e];
-            dv[pos] = val[e];
+            pos[e] = atomicAdd(&hist[(key[e] - mn) >> sh], 1);
+            dk[pos[e]] = key[e];
         }
     }
     g.sync();
-    // hist[b] now = end of bucket b.  Sort + reduce my buckets, compacting in place.
-    int w = my_start;
-    int start = my_start;
-    for (int b = b0; b < b1; ++b) {
-        const int end = hist[b];
-        for (int q = start + 1; q < end; ++q) {       // insertion sort (buckets are tiny)
-            const int32_t kk = dk[q];
-            const float vv = dv[q];
-            int j = q;
-            while (j > start && dk[j - 1] > kk) {
-                dk[j] = dk[j - 1];
-                dv[j] = dv[j - 1];
-                --j;
+    // 2. hist[b] = end of bucket b.  Every element counts the keys of its bucket that sort
+    //    before it (smaller, or equal and scattered earlier) and moves to its sorted slot.
+#pragma unroll
+    for (int e = 0; e < EPT; ++e) {
+        if (pos[e] >= 0) {
+            const int b = (key[e] - mn) >> sh;
+            const int bs = b ? hist[b - 1] : 0, be = hist[b];
+            const int32_t kk = key[e];
+            int rank = 0;
+            for (int q = bs; q < be; ++q) {
+                const int32_t kq = dk[q];
+                rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
             }
-            dk[j] = kk;
-            dv[j] = vv;
+            dk2[bs + rank] = kk;
+            dv2[bs + rank] = val[e];
         }
-        int q = start;
-        while (q < end) {
-            const int32_t kk = dk[q];
-            double acc = (double)dv[q];
-            ++q;
-            while (q < end && dk[q] == kk) acc += (double)dv[q++];
-            dk[w] = kk;
-            dv[w] = (float)acc;
-            ++w;
-        }
-        start = end;
     }
-    const int u = w - my_start;
+    g.sync();
+    // 3. segmented reduction over contiguous slices (fp64), compacted into (dk, dv)
+    const int E = (L + T - 1) / T;
+    const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
+    int nh = 0;
+    for (int p = p0; p < p1; ++p) nh += (p == 0 || dk2[p] != dk2[p - 1]);
     int U;
-    const int off = g.excl_sum(u, sc, &U);
-    __syncwarp();
-    const int64_t wbase = __shfl_sync(kFull, off, 0);
-    warp_copy_out(my_start, u, wbase, dk, dv, out_col, out_val);
+    int o = g.excl_sum(nh, sc, &U);
+    for (int p = p0; p < p1; ++p) {
+        if (p == 0 || dk2[p] != dk2[p - 1]) {
+            const int32_t kk = dk2[p];
+            double acc = (double)dv2[p];
+            for (int q = p + 1; q < L && dk2[q] == kk; ++q) acc += (double)dv2[q];
+            dk[o] = kk;
+            dv[o] = (float)acc;
+            ++o;
+        }
+    }
+    g.sync();
+    // 4. coalesced copy of the merged row
+    for (int q = g.gtid; q < U; q += T) {
+        out_col[q] = dk[q];
+        out_val[q] = dv[q];
+    }
     return U;
 }
 
@@ -391,12 +398,12 @@ template <int NW, int EPT>
 struct BucketSmem {
     static constexpr int kCap = NW * 32 * EPT;
     static constexpr int kNb = ceil_pow2(kCap);
-    static constexpr int kBytes = kCap * 8 + kNb * 4;
+    static constexpr int kBytes = kCap * 16 + kNb * 4;
 };
 
 // Rows of one bin: bucket sort per row; rows whose buckets overflow go to a fallback list.
 template <int NW, int GROUPS, int EPT>
-__global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_bucket(const int32_t *__restrict__ rows, int64_t nrows,
+__global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k_merge_bucket(const int32_t *__restrict__ rows, int64_t nrows,
                                                                   const int64_t *__restrict__ rowoff,
                                                                   int32_t *__restrict__ chat_col,
                                                                   float *__restrict__ chat_val,
@@ -410,12 +417,14 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_bucket(const int32_t
     unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
     int32_t *dk = (int32_t *)slice;
     float *dv = (float *)(slice + S::kCap * 4);
-    int *hist = (int *)(slice + S::kCap * 8);
+    int32_t *dk2 = (int32_t *)(slice + S::kCap * 8);
+    float *dv2 = (float *)(slice + S::kCap * 12);
+    int *hist = (int *)(slice + S::kCap * 16);
     for (int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
         const int i = rows[r];
         const int64_t s = rowoff[i];
         const int L = (int)(rowoff[i + 1] - s);
-        const int U = bucket_sort_reduce<NW, GROUPS, EPT>(g, chat_col + s, chat_val + s, L, dk, dv, hist,
+        const int U = bucket_sort_reduce<NW, GROUPS, EPT>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
                                                           chat_col + s, chat_val + s, sc_all[g.gid]);
         if (g.gtid == 0) {
             if (U >= 0) ccount[i] = U;
@@ -490,9 +499,10 @@ constexpr int kLimNW = kLimThreads / 32;
 constexpr int kLimCap = 9216;
 constexpr int kLimEPT = kLimCap / kLimThreads;   // 18
 constexpr int kLimWindow = 16384;
-constexpr int kLimSmem = SortSmem<kLimCap>::kBytes > kLimWindow * 8 + (kLimWindow / 32) * 4
-                             ? SortSmem<kLimCap>::kBytes
-                             : kLimWindow * 8 + (kLimWindow / 32) * 4;
+constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
+constexpr int kLimSmem = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
+                               kLimCap * 16 + ceil_pow2(kLimCap) * 4,     // bucket sort
+                               kLimWindow * 8 + (kLimWindow / 32) * 4);   // dense window
 
 struct LimitedArgs {
     const int32_t *rows;          // limited rows, longest first
@@ -557,9 +567,11 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         if (L <= kLimCap) {
             int32_t *dk = (int32_t *)smem_raw;
             float *dv = (float *)(smem_raw + kLimCap * 4);
-            int *hist = (int *)(smem_raw + kLimCap * 8);
-            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)L, dk, dv, hist,
-                                                            g.chat_col + s, g.chat_val + s, sc);
+            int32_t *dk2 = (int32_t *)(smem_raw + kLimCap * 8);
+            float *dv2 = (float *)(smem_raw + kLimCap * 12);
+            int *hist = (int *)(smem_raw + kLimCap * 16);
+            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)L, dk, dv, dk2, dv2,
+                                                            hist, g.chat_col + s, g.chat_val + s, sc);
             if (U < 0)
                 U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)L,
                                                           g.chat_col + s, g.chat_val + s);
@@ -731,8 +743,11 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 cp_async_wait_all();
                 __syncthreads();
-                int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, k0, v0, total, k0, v0, (int *)(smem_raw + kLimCap * 8),
-                                                                st_col + nout, st_val + nout, sc);
+                int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, k0, v0, total, k0, v0,
+                                                                (int32_t *)(smem_raw + kLimCap * 8),
+                                                                (float *)(smem_raw + kLimCap * 12),
+                                                                (int *)(smem_raw + kLimCap * 16), st_col + nout,
+                                                                st_val + nout, sc);
                 if (U < 0) {
                     int32_t *k1 = (int32_t *)(smem_raw + kLimCap * 8);
                     float *v1 = (float *)(smem_raw + kLimCap * 12);
