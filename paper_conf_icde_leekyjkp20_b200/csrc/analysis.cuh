@@ -30,8 +30,13 @@ constexpr int kRowBucketLim0 = 5;      // 5 + (39 - floor(log2 L)): longest rows
 constexpr int kRowBucketEmpty = 45;
 constexpr int kNumRowBuckets = 46;
 constexpr int kWarpRowMax = 32;
+// Ĉ runs are padded to multiples of kRunAlign slots (16 B) with sentinel entries
+// (col = INT32_MAX, val = 0) so that every run starts 16-byte aligned (vector stores).
+constexpr int kRunAlign = 4;
+__host__ __device__ __forceinline__ int64_t pad_run(int64_t x) { return (x + kRunAlign - 1) & ~(int64_t)(kRunAlign - 1); }
 constexpr int kSort256Max = 256;
 constexpr int kSort1KMax = 1024;
+constexpr int64_t kLimitCapacity = 4096;   // largest bucket length of the non-limited merge bins
 
 struct PlanScalars {
     unsigned long long nnz_chat;     // sum_k work[k]
@@ -39,6 +44,7 @@ struct PlanScalars {
     unsigned long long m_nonempty;   // #rows with rowwork > 0
     unsigned long long max_rowwork;
     unsigned long long max_deg;      // max runs (A entries with nnz(b_k*) > 0) in a row
+    unsigned long long rowwise_sum;  // sum_i rowwork[i] (nnz(Ĉ) counted row-wise)
     unsigned long long lim_runs;     // sum of runs over limited rows
     unsigned long long lim_max_deg;  // max runs of a limited row
     unsigned long long lim_max_L;    // max products of a limited row
@@ -108,7 +114,8 @@ __global__ void __launch_bounds__(256) k_pair_work(const int64_t *__restrict__ a
 __global__ void __launch_bounds__(256) k_row_work(const int64_t *__restrict__ a_colptr,
                                                   const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
                                                   const int64_t *__restrict__ b_rowptr,
-                                                  unsigned long long *__restrict__ rowwork, int32_t *__restrict__ deg) {
+                                                  unsigned long long *__restrict__ rowwork, int32_t *__restrict__ deg,
+                                                  unsigned long long *__restrict__ rowcap) {
     int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
     if (e0 >= nnz_a) return;
     int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
@@ -124,28 +131,32 @@ __global__ void __launch_bounds__(256) k_row_work(const int64_t *__restrict__ a_
             int32_t i = a_rowidx[e];
             atomicAdd(rowwork + i, (unsigned long long)rb);
             atomicAdd(deg + i, 1);
+            if (rowcap) atomicAdd(rowcap + i, (unsigned long long)pad_run(rb));
         }
     }
 }
 
 __global__ void __launch_bounds__(256) k_row_reduce(const int64_t *__restrict__ rowwork,
                                                     const int32_t *__restrict__ deg, int64_t M, PlanScalars *sc) {
-    __shared__ unsigned long long sm[3][8];
-    unsigned long long ne = 0, mx = 0, md = 0;
+    __shared__ unsigned long long sm[4][8];
+    unsigned long long ne = 0, mx = 0, md = 0, sum = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
         int64_t w = rowwork[i];
+        sum += (unsigned long long)w;
         ne += w > 0;
         mx = max(mx, (unsigned long long)w);
         md = max(md, (unsigned long long)deg[i]);
     }
     ne = warp_sum(ne);
+    sum = warp_sum(sum);
     mx = warp_max(mx);
     md = warp_max(md);
-    if (lane_id() == 0) { sm[0][warp_id()] = ne; sm[1][warp_id()] = mx; sm[2][warp_id()] = md; }
+    if (lane_id() == 0) { sm[0][warp_id()] = ne; sm[1][warp_id()] = mx; sm[2][warp_id()] = md; sm[3][warp_id()] = sum; }
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned long long a = 0, b = 0, c = 0;
-        for (int w = 0; w < 8; ++w) { a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); }
+        unsigned long long a = 0, b = 0, c = 0, d = 0;
+        for (int w = 0; w < 8; ++w) { a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); d += sm[3][w]; }
+        atomicAdd(&sc->rowwise_sum, d);
         atomicAdd(&sc->m_nonempty, a);
         atomicMax(&sc->max_rowwork, b);
         atomicMax(&sc->max_deg, c);
@@ -153,7 +164,8 @@ __global__ void __launch_bounds__(256) k_row_reduce(const int64_t *__restrict__ 
 }
 
 // Run bases: the run of products of A entry e = (i, k) occupies Ĉ positions
-// [base[e], base[e] + nnz(b_k*)) inside row i's bucket (cursor starts at rowoff[i]).
+// [base[e], base[e] + nnz(b_k*)) inside row i's bucket (cursor starts at rowoff[i]), followed
+// by pad_run(nnz(b_k*)) - nnz(b_k*) sentinel slots.
 __global__ void __launch_bounds__(256) k_run_base(const int64_t *__restrict__ a_colptr,
                                                   const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
                                                   const int64_t *__restrict__ b_rowptr,
@@ -169,7 +181,7 @@ __global__ void __launch_bounds__(256) k_run_base(const int64_t *__restrict__ a_
             kend = __ldg(a_colptr + k + 1);
             rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
         }
-        base[e] = rb > 0 ? (int64_t)atomicAdd(cursor + a_rowidx[e], (unsigned long long)rb) : -1;
+        base[e] = rb > 0 ? (int64_t)atomicAdd(cursor + a_rowidx[e], (unsigned long long)pad_run(rb)) : -1;
     }
 }
 
@@ -310,27 +322,30 @@ __global__ void k_piece_whole(const int32_t *__restrict__ list, int64_t n, const
 // Merge row classes.  Limited rows (L > t_lim, L452-L477 L) get B-Limited merge blocks;
 // a row made of a single run (one A entry) is already sorted and duplicate-free.
 __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict__ rowwork,
+                                                      const int64_t *__restrict__ rowoff,
                                                       const int32_t *__restrict__ deg, int64_t M, int64_t t_lim,
-                                                      int8_t *__restrict__ rcls, uint8_t *__restrict__ bucket,
-                                                      PlanScalars *sc) {
+                                                      int64_t cap_max, int8_t *__restrict__ rcls,
+                                                      uint8_t *__restrict__ bucket, PlanScalars *sc) {
     __shared__ unsigned long long sm[3][8];
     unsigned long long runs = 0, mdeg = 0, mlen = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
-        int64_t L = rowwork[i];
+        // L = products of the row (paper class); cap = its padded bucket length (kernel capacity)
+        const int64_t L = rowwork[i];
+        const int64_t cap = rowoff[i + 1] - rowoff[i];
         int8_t c;
         int b;
         if (L == 0) { c = RC_EMPTY; b = kRowBucketEmpty; }
         else if (deg[i] == 1) { c = RC_PASS; b = kRowBucketPass; }
-        else if (L > t_lim) {
+        else if (L > t_lim || cap > cap_max) {
             c = RC_LIMITED;
             b = kRowBucketLim0 + (39 - min(39, ilog2_floor((uint64_t)L)));
             runs += (unsigned long long)deg[i];
             mdeg = max(mdeg, (unsigned long long)deg[i]);
-            mlen = max(mlen, (unsigned long long)L);
+            mlen = max(mlen, (unsigned long long)cap);
         }
-        else if (L <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
-        else if (L <= kSort256Max) { c = RC_WARP_SORT; b = kRowBucketSort256; }
-        else if (L <= kSort1KMax) { c = RC_WARP_SORT; b = kRowBucketSort1K; }
+        else if (cap <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
+        else if (cap <= kSort256Max) { c = RC_WARP_SORT; b = kRowBucketSort256; }
+        else if (cap <= kSort1KMax) { c = RC_WARP_SORT; b = kRowBucketSort1K; }
         else { c = RC_GROUP_SORT; b = kRowBucketSort4K; }
         rcls[i] = c;
         bucket[i] = (uint8_t)b;

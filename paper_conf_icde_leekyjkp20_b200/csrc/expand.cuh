@@ -19,20 +19,46 @@ constexpr int kPieceAChunk = 256;   // A entries staged per round (= default spl
 
 // B-Split pieces and whole blocks (Normal pairs).  One CTA per piece.  The paper's block has
 // nnz(b_k*) effective threads, each looping over the A column (L385-L386 R, L411-L415 L).
-// Wide pieces (b_len >= 32): a warp holds a 128-entry chunk of the B sub-row in registers and
-// streams it to every A entry of the piece (4 coalesced stores per lane and array).
-// Thin pieces (b_len < 32): micro-blocks of w = 2^ceil(log2 b_len) lanes, 32/w A entries per
-// warp step, so thin blocks do not idle lanes (block compaction, L406-L409 R).
+// Runs start 16-byte aligned (kRunAlign padding), so a lane owns 4 consecutive slots and
+// writes them with one 16-byte store per array.
+// Wide pieces (b_len >= 32): a warp holds a 128-slot chunk of the B sub-row in registers and
+// streams it to every A entry of the piece (one int4 + one float4 store per lane and entry).
+// Thin pieces (b_len < 32): micro-blocks of v lanes (v vectors cover the padded run) and 32/v
+// A entries per warp step, so thin blocks do not idle lanes (block compaction, L406-L409 R).
+// The slots after the run's last product (up to the padded length) get sentinel entries.
+__device__ __forceinline__ void load_b4(const int32_t *__restrict__ bc, const float *__restrict__ bv, int j, int n,
+                                        int4 &c4, float4 &v4) {
+    c4.x = j + 0 < n ? __ldg(bc + j + 0) : 0x7fffffff;
+    c4.y = j + 1 < n ? __ldg(bc + j + 1) : 0x7fffffff;
+    c4.z = j + 2 < n ? __ldg(bc + j + 2) : 0x7fffffff;
+    c4.w = j + 3 < n ? __ldg(bc + j + 3) : 0x7fffffff;
+    v4.x = j + 0 < n ? __ldg(bv + j + 0) : 0.f;
+    v4.y = j + 1 < n ? __ldg(bv + j + 1) : 0.f;
+    v4.z = j + 2 < n ? __ldg(bv + j + 2) : 0.f;
+    v4.w = j + 3 < n ? __ldg(bv + j + 3) : 0.f;
+}
+
+__device__ __forceinline__ void store_run4(int32_t *__restrict__ chat_col, float *__restrict__ chat_val, int64_t dst,
+                                           const int4 &c4, const float4 &v4, float a) {
+    *reinterpret_cast<int4 *>(chat_col + dst) = c4;
+    *reinterpret_cast<float4 *>(chat_val + dst) = make_float4(a * v4.x, a * v4.y, a * v4.z, a * v4.w);
+}
+
 __global__ void __launch_bounds__(kPieceThreads) k_expand_pieces(
-    const Piece *__restrict__ pieces, const float *__restrict__ a_val, const int32_t *__restrict__ b_colidx,
-    const float *__restrict__ b_val, const int64_t *__restrict__ base, int32_t *__restrict__ chat_col,
-    float *__restrict__ chat_val) {
+    const Piece *__restrict__ pieces, const float *__restrict__ a_val, const int64_t *__restrict__ b_rowptr,
+    const int32_t *__restrict__ b_colidx, const float *__restrict__ b_val, const int64_t *__restrict__ base,
+    int32_t *__restrict__ chat_col, float *__restrict__ chat_val) {
     __shared__ float s_a[kPieceAChunk];
     __shared__ int64_t s_dst[kPieceAChunk];
     const Piece pc = pieces[blockIdx.x];
     const int lane = lane_id(), w = warp_id();
     const int32_t *__restrict__ bc = b_colidx + pc.b_lo;
     const float *__restrict__ bv = b_val + pc.b_lo;
+    // slots this piece writes: its B sub-row, plus the run's padding if it holds the last tile
+    const int rb = (int)(__ldg(b_rowptr + pc.k + 1) - __ldg(b_rowptr + pc.k));
+    const bool last = pc.b_off + pc.b_len == rb;
+    const int nslots = last ? (int)pad_run(rb) - pc.b_off : pc.b_len;
+    const bool vec = (pc.b_off % kRunAlign) == 0 && (nslots % kRunAlign) == 0;
     for (int a0 = 0; a0 < pc.a_len; a0 += kPieceAChunk) {
         const int na = min(kPieceAChunk, pc.a_len - a0);
         for (int t = threadIdx.x; t < na; t += kPieceThreads) {
@@ -40,75 +66,67 @@ __global__ void __launch_bounds__(kPieceThreads) k_expand_pieces(
             s_dst[t] = __ldg(base + pc.a_lo + a0 + t) + pc.b_off;
         }
         __syncthreads();
-        if (pc.b_len >= 32) {
-            const int nchunks = (pc.b_len + 127) >> 7;
+        if (!vec) {
+            // B tiles not multiples of kRunAlign (a user split_b_tile): scalar stores
+            for (int a = w; a < na; a += kPieceWarps)
+                for (int j = lane; j < nslots; j += 32) {
+                    const bool real = j < pc.b_len;
+                    chat_col[s_dst[a] + j] = real ? __ldg(bc + j) : 0x7fffffff;
+                    chat_val[s_dst[a] + j] = real ? s_a[a] * __ldg(bv + j) : 0.f;
+                }
+        } else if (pc.b_len >= 32) {
+            const int nchunks = (nslots + 127) >> 7;
             const int slices = nchunks >= kPieceWarps ? 1 : kPieceWarps / nchunks;   // A slices per chunk
             for (int u = w; u < nchunks * slices; u += kPieceWarps) {
-                const int c0 = (u / slices) << 7;
+                const int j = ((u / slices) << 7) + 4 * lane;
                 const int sl = u % slices;
-                int32_t cb[4];
-                float vb[4];
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const int j = c0 + q * 32 + lane;
-                    cb[q] = j < pc.b_len ? __ldg(bc + j) : 0;
-                    vb[q] = j < pc.b_len ? __ldg(bv + j) : 0.f;
-                }
-                const int lim = min(128, pc.b_len - c0);
-                for (int a = sl; a < na; a += slices) {
-                    const int64_t dst = s_dst[a] + c0;
-                    const float av = s_a[a];
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        const int j = q * 32 + lane;
-                        if (j < lim) {
-                            chat_col[dst + j] = cb[q];
-                            chat_val[dst + j] = av * vb[q];
-                        }
-                    }
-                }
+                int4 c4;
+                float4 v4;
+                load_b4(bc, bv, j, pc.b_len, c4, v4);
+                if (j < nslots)
+                    for (int a = sl; a < na; a += slices) store_run4(chat_col, chat_val, s_dst[a] + j, c4, v4, s_a[a]);
             }
         } else {
-            const int shift = ilog2_ceil((uint64_t)pc.b_len);
+            const int nvec = nslots >> 2;                       // 1..8 vectors per run
+            const int shift = ilog2_ceil((uint64_t)nvec);       // micro-block of 2^shift lanes
             const int mb = lane >> shift;
             const int sub = lane & ((1 << shift) - 1);
             const int g = 32 >> shift;
-            const bool act = sub < pc.b_len;
-            const int32_t cb = act ? __ldg(bc + sub) : 0;
-            const float vb = act ? __ldg(bv + sub) : 0.f;
-            if (act) {
-                for (int a = w * g + mb; a < na; a += kPieceWarps * g) {
-                    const int64_t dst = s_dst[a] + sub;
-                    chat_col[dst] = cb;
-                    chat_val[dst] = s_a[a] * vb;
-                }
-            }
+            int4 c4;
+            float4 v4;
+            load_b4(bc, bv, 4 * sub, pc.b_len, c4, v4);
+            if (sub < nvec)
+                for (int a = w * g + mb; a < na; a += kPieceWarps * g)
+                    store_run4(chat_col, chat_val, s_dst[a] + 4 * sub, c4, v4, s_a[a]);
         }
         __syncthreads();
     }
 }
 
-// B-Gathering (L369-L450): low performers with 2^(N-1) < nnz(b_k*) <= 2^N are packed
-// 32/2^N per warp ("gathering factor 32/2^n", L438-L441 L); each micro-block of 2^N lanes
-// keeps its B row in registers and loops over its A column, four entries per step with the
-// (value, base) loads issued together.
+// B-Gathering (L369-L450): low performers with 2^(N-1) < nnz(b_k*) <= 2^N are packed into
+// combined blocks ("gathering factor 32/2^n", L438-L441 L).  With 16-byte slots a lane covers
+// 4 effective threads, so a micro-block is V = max(1, 2^N / 4) lanes and a warp packs 32 / V
+// pairs; each micro-block keeps its B row in registers and loops over its A column, four A
+// entries per step with their (value, base) loads issued together.
 template <int N>
 __global__ void __launch_bounds__(256) k_expand_gathered(
     const int32_t *__restrict__ list, int64_t count, const int64_t *__restrict__ a_colptr,
     const float *__restrict__ a_val, const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ b_colidx,
     const float *__restrict__ b_val, const int64_t *__restrict__ base, int32_t *__restrict__ chat_col,
     float *__restrict__ chat_val) {
-    constexpr int W = 1 << N;
-    const int64_t slot = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> N;
-    const int sub = threadIdx.x & (W - 1);
+    constexpr int V = (1 << N) >= 4 ? (1 << N) / 4 : 1;
+    constexpr int SH = V == 1 ? 0 : (V == 2 ? 1 : (V == 4 ? 2 : 3));
+    const int64_t slot = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> SH;
+    const int sub = threadIdx.x & (V - 1);
     if (slot >= count) return;
     const int k = __ldg(list + slot);
     const int64_t a0 = __ldg(a_colptr + k), a1 = __ldg(a_colptr + k + 1);
     const int64_t b0 = __ldg(b_rowptr + k);
     const int rb = (int)(__ldg(b_rowptr + k + 1) - b0);
-    if (sub >= rb) return;
-    const int32_t col = __ldg(b_colidx + b0 + sub);
-    const float bv = __ldg(b_val + b0 + sub);
+    if (4 * sub >= rb) return;
+    int4 c4;
+    float4 v4;
+    load_b4(b_colidx + b0, b_val + b0, 4 * sub, rb, c4, v4);
     int64_t e = a0;
     for (; e + 4 <= a1; e += 4) {
         int64_t d[4];
@@ -119,16 +137,9 @@ __global__ void __launch_bounds__(256) k_expand_gathered(
             av[q] = __ldg(a_val + e + q);
         }
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            chat_col[d[q] + sub] = col;
-            chat_val[d[q] + sub] = av[q] * bv;
-        }
+        for (int q = 0; q < 4; ++q) store_run4(chat_col, chat_val, d[q] + 4 * sub, c4, v4, av[q]);
     }
-    for (; e < a1; ++e) {
-        const int64_t d = __ldg(base + e) + sub;
-        chat_col[d] = col;
-        chat_val[d] = __ldg(a_val + e) * bv;
-    }
+    for (; e < a1; ++e) store_run4(chat_col, chat_val, __ldg(base + e) + 4 * sub, c4, v4, __ldg(a_val + e));
 }
 
 }  // namespace spg

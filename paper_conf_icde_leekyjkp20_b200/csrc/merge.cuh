@@ -303,9 +303,9 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
         const int p = g.gtid + e * T;
-        key[e] = p < L ? sk[p] : kKeyPad;
+        key[e] = p < L ? sk[p] : kKeyPad;       // sentinel (padding) entries stay kKeyPad
         val[e] = p < L ? sv[p] : 0.f;
-        if (p < L) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
+        if (key[e] != kKeyPad) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
     }
     mn = g.reduce_min(mn, sc);
     mx = g.reduce_max(mx, sc);
@@ -318,7 +318,7 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     g.sync();
 #pragma unroll
     for (int e = 0; e < EPT; ++e)
-        if (g.gtid + e * T < L) atomicAdd(&hist[(key[e] - mn) >> sh], 1);
+        if (key[e] != kKeyPad) atomicAdd(&hist[(key[e] - mn) >> sh], 1);
     g.sync();
     const int bpt = (nb + T - 1) / T;
     const int b0 = min(nb, g.gtid * bpt), b1 = min(nb, b0 + bpt);
@@ -342,7 +342,7 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
         pos[e] = -1;
-        if (g.gtid + e * T < L) {
+        if (key[e] != kKeyPad) {
             pos[e] = atomicAdd(&hist[(key[e] - mn) >> sh], 1);
             dk[pos[e]] = key[e];
         }
@@ -367,6 +367,7 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     }
     g.sync();
     // 3. segmented reduction over contiguous slices (fp64), compacted into (dk, dv)
+    L = tot;   // valid (non-sentinel) entries
     const int E = (L + T - 1) / T;
     const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
     int nh = 0;
@@ -438,7 +439,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
 template <int NW, int GROUPS, int CAP>
 __device__ __forceinline__ int merge_row_in_smem(const Group<NW, GROUPS> &g, unsigned char *slice, int *sc,
                                                  int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
-                                                 int64_t s, int L, int32_t *__restrict__ out_col,
+                                                 int64_t s, int L, int Lval, int32_t *__restrict__ out_col,
                                                  float *__restrict__ out_val) {
     constexpr int T = NW * 32;
     int32_t *k0 = (int32_t *)slice;
@@ -454,7 +455,8 @@ __device__ __forceinline__ int merge_row_in_smem(const Group<NW, GROUPS> &g, uns
     cp_async_wait_all();
     g.sync();
     const int which = natural_merge_sort<NW, GROUPS, CAP>(g, k0, v0, k1, v1, bA, bB, L, sc);
-    const int U = segmented_reduce_out<NW, GROUPS>(g, which ? k1 : k0, which ? v1 : v0, L, out_col, out_val, sc);
+    // sentinel (padding) keys sort last: the first Lval entries are the row's products
+    const int U = segmented_reduce_out<NW, GROUPS>(g, which ? k1 : k0, which ? v1 : v0, Lval, out_col, out_val, sc);
     g.sync();
     return U;
 }
@@ -462,6 +464,7 @@ __device__ __forceinline__ int merge_row_in_smem(const Group<NW, GROUPS> &g, uns
 template <int NW, int GROUPS, int CAP>
 __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *__restrict__ rows, int64_t nrows,
                                                                 const int64_t *__restrict__ rowoff,
+                                                                const int64_t *__restrict__ rowwork,
                                                                 int32_t *__restrict__ chat_col,
                                                                 float *__restrict__ chat_val,
                                                                 int64_t *__restrict__ ccount,
@@ -476,7 +479,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
         const int64_t s = rowoff[i];
         const int L = (int)(rowoff[i + 1] - s);
         const int U = merge_row_in_smem<NW, GROUPS, CAP>(g, slice, sc_all[g.gid], chat_col, chat_val, s, L,
-                                                         chat_col + s, chat_val + s);
+                                                         (int)rowwork[i], chat_col + s, chat_val + s);
         if (g.gtid == 0) ccount[i] = U;
     }
 }
@@ -508,6 +511,7 @@ struct LimitedArgs {
     const int32_t *rows;          // limited rows, longest first
     int64_t nrows;
     const int64_t *rowoff;
+    const int64_t *rowwork;
     const int64_t *run_start;     // [nrows+1]
     const int64_t *run_base;
     const int32_t *run_len;
@@ -563,17 +567,18 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         if (r >= g.nrows) break;
         const int i = g.rows[r];
         const int64_t s = g.rowoff[i];
-        const int64_t L = g.rowoff[i + 1] - s;
-        if (L <= kLimCap) {
+        const int64_t cap = g.rowoff[i + 1] - s;   // padded bucket length
+        const int64_t L = g.rowwork[i];             // products
+        if (cap <= kLimCap) {
             int32_t *dk = (int32_t *)smem_raw;
             float *dv = (float *)(smem_raw + kLimCap * 4);
             int32_t *dk2 = (int32_t *)(smem_raw + kLimCap * 8);
             float *dv2 = (float *)(smem_raw + kLimCap * 12);
             int *hist = (int *)(smem_raw + kLimCap * 16);
-            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)L, dk, dv, dk2, dv2,
-                                                            hist, g.chat_col + s, g.chat_val + s, sc);
+            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
+                                                            dv2, hist, g.chat_col + s, g.chat_val + s, sc);
             if (U < 0)
-                U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)L,
+                U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
                                                           g.chat_col + s, g.chat_val + s);
             if (threadIdx.x == 0) g.ccount[i] = U;
             __syncthreads();
@@ -774,11 +779,11 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
 }
 
 // Single-run rows: already sorted and duplicate-free; merged length = bucket length.
-__global__ void k_merge_pass(const int32_t *__restrict__ rows, int64_t nrows, const int64_t *__restrict__ rowoff,
+__global__ void k_merge_pass(const int32_t *__restrict__ rows, int64_t nrows, const int64_t *__restrict__ rowwork,
                              int64_t *__restrict__ ccount) {
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < nrows; q += (int64_t)gridDim.x * blockDim.x) {
         const int i = rows[q];
-        ccount[i] = rowoff[i + 1] - rowoff[i];
+        ccount[i] = rowwork[i];   // the run's sentinel padding trails its products
     }
 }
 

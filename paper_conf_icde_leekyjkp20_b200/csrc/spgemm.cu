@@ -128,7 +128,7 @@ struct spgemm_plan_s {
     int32_t *deg = nullptr;
     PlanScalars *scal = nullptr;
     PlanScalars h_scal{};
-    int64_t nnz_chat = 0, nnz_chat_rowwise = 0, t_dom = 0, t_lim = 0;
+    int64_t nnz_chat = 0, nnz_chat_rowwise = 0, chat_cap = 0, t_dom = 0, t_lim = 0;
     // stage 2
     int8_t *pair_cls = nullptr, *row_cls = nullptr;
     int32_t *pair_order = nullptr, *row_order = nullptr;
@@ -390,10 +390,17 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     if (K > 0)
         LAUNCH("pair_work", s, k_pair_work<<<grid_for(K, 256, p->num_sms * 8), 256, 0, s>>>(p->a_colptr, p->b_rowptr, K,
                                                                                      p->work, p->scal));
-    if (p->nnz_a > 0)
-        LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
-            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg));
-    TRY(scan_excl(p, p->rowwork, M, p->rowoff, s, "row_offsets"));
+    {
+        Temp tcap(s);
+        int64_t *rowcap;
+        TRY(talloc(p, tcap, &rowcap, M));
+        if (M > 0) CK(cudaMemsetAsync(rowcap, 0, M * 8, s));
+        if (p->nnz_a > 0)
+            LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+                p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg,
+                (unsigned long long *)rowcap));
+        TRY(scan_excl(p, rowcap, M, p->rowoff, s, "row_offsets"));   // padded bucket offsets
+    }
     if (M > 0)
         LAUNCH("row_reduce", s, k_row_reduce<<<grid_for(M, 256, p->num_sms * 8), 256, 0, s>>>(p->rowwork, p->deg, M, p->scal));
     if (p->nnz_a > 0) {
@@ -405,10 +412,11 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
             p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, cursor, p->base));
     }
     CK(cudaMemcpyAsync(&p->h_scal, p->scal, sizeof(PlanScalars), cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(&p->nnz_chat_rowwise, p->rowoff + M, 8, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));  // sync 1: nnz(Ĉ) both ways, #non-empty blocks
+    CK(cudaMemcpyAsync(&p->chat_cap, p->rowoff + M, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));  // sync 1: nnz(Ĉ) both ways, Ĉ capacity, #non-empty blocks
     if (p->h_scal.invalid) return fail(SPGEMM_ERR_INVALID_INPUT, "malformed indices (range / order) in A or B");
     p->nnz_chat = (int64_t)p->h_scal.nnz_chat;
+    p->nnz_chat_rowwise = (int64_t)p->h_scal.rowwise_sum;
     if (p->nnz_chat != p->nnz_chat_rowwise)
         return fail(SPGEMM_ERR_CUDA, "internal: block-wise and row-wise nnz(Ĉ) disagree");
 
@@ -449,8 +457,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         TRY(scan_excl(p, npieces, K, p->piece_off, s, "piece_scan"));
         TRY(partition(p, pb, K, kNumPairBuckets, p->pair_order, d_starts, s, "pair_partition"));
         if (M > 0)
-            LAUNCH("row_classify", s, k_row_classify<<<grid_for(M, 256), 256, 0, s>>>(p->rowwork, p->deg, M, p->t_lim,
-                                                                                  p->row_cls, rbk, p->scal));
+            LAUNCH("row_classify", s, k_row_classify<<<grid_for(M, 256), 256, 0, s>>>(
+                p->rowwork, p->rowoff, p->deg, M, p->t_lim, kLimitCapacity, p->row_cls, rbk, p->scal));
         TRY(partition(p, rbk, M, kNumRowBuckets, p->row_order, d_starts + kNumPairBuckets + 1, s, "row_partition"));
         CK(cudaMemcpyAsync(p->pair_starts, d_starts, sizeof(int64_t) * (kNumPairBuckets + 1), cudaMemcpyDeviceToHost, s));
         CK(cudaMemcpyAsync(p->row_starts, d_starts + kNumPairBuckets + 1, sizeof(int64_t) * (kNumRowBuckets + 1),
@@ -506,8 +514,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         TRY(palloc(p, &p->row_counter, 1, s));
     }
     // Ĉ and merge state
-    TRY(palloc(p, &p->chat_col, p->nnz_chat, s));
-    TRY(palloc(p, &p->chat_val, p->nnz_chat, s));
+    TRY(palloc(p, &p->chat_col, p->chat_cap, s));
+    TRY(palloc(p, &p->chat_val, p->chat_cap, s));
     TRY(palloc(p, &p->ccount, M, s));
     TRY(palloc(p, &p->fb_rows, M, s));
     TRY(palloc(p, &p->fb_count, 1, s));
@@ -525,13 +533,14 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     const int64_t np = p->n_split_pieces + p->n_whole;
     if (np > 0)
         LAUNCH("expand_pieces", s, k_expand_pieces<<<(unsigned)np, kPieceThreads, 0, s>>>(
-            p->pieces, p->a_val, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
+            p->pieces, p->a_val, p->b_rowptr, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
     for (int nb = 0; nb < 6; ++nb) {
         const int64_t lo = p->pair_starts[kPairBucketGather0 + nb * 16];
         const int64_t cnt = p->pair_starts[kPairBucketGather0 + nb * 16 + 16] - lo;
         if (cnt == 0) continue;
         const int32_t *list = p->pair_order + lo;
-        const unsigned grid = (unsigned)cdiv(cnt << nb, 256);
+        const int lanes = nb >= 2 ? (1 << nb) / 4 : 1;   // lanes per gathered pair (k_expand_gathered<N>::V)
+        const unsigned grid = (unsigned)cdiv(cnt * lanes, 256);
 #define GATHER_CASE(N)                                                                                      \
     case N:                                                                                                 \
         LAUNCH("expand_gathered", s, k_expand_gathered<N><<<grid, 256, 0, s>>>(                             \
@@ -567,7 +576,7 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     int64_t cnt;
     const int32_t *rows = rows_of(kRowBucketPass, kRowBucketPass + 1, &cnt);
     if (cnt > 0)
-        LAUNCH("merge_pass", s, k_merge_pass<<<grid_for(cnt, 256), 256, 0, s>>>(rows, cnt, p->rowoff, p->ccount));
+        LAUNCH("merge_pass", s, k_merge_pass<<<grid_for(cnt, 256), 256, 0, s>>>(rows, cnt, p->rowwork, p->ccount));
     rows = rows_of(kRowBucketWarp, kRowBucketWarp + 1, &cnt);
     if (cnt > 0)
         LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
@@ -584,7 +593,7 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         const int smem = SortSmem<CAP>::kBytes;
         CK(cudaFuncSetAttribute(k_merge_rows<8, 1, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
-            p->fb_rows, 0, p->rowoff, p->chat_col, p->chat_val, p->ccount, p->fb_count));
+            p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count));
     }
     if (p->nlim > 0) {
         CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
@@ -592,6 +601,7 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         g.rows = p->row_order + p->row_starts[kRowBucketLim0];
         g.nrows = p->nlim;
         g.rowoff = p->rowoff;
+        g.rowwork = p->rowwork;
         g.run_start = p->run_start;
         g.run_base = p->run_base;
         g.run_len = p->run_len;
@@ -718,10 +728,10 @@ int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_
         case SPGEMM_VIEW_ROW_CLASS: src = p->row_cls; bytes = p->m; break;
         case SPGEMM_VIEW_CHAT_COL:
             if (p->state != 2) return fail(SPGEMM_ERR_STATE, "Ĉ is only inspectable between expand and merge");
-            src = p->chat_col; bytes = p->nnz_chat * 4; break;
+            src = p->chat_col; bytes = p->chat_cap * 4; break;
         case SPGEMM_VIEW_CHAT_VAL:
             if (p->state != 2) return fail(SPGEMM_ERR_STATE, "Ĉ is only inspectable between expand and merge");
-            src = p->chat_val; bytes = p->nnz_chat * 4; break;
+            src = p->chat_val; bytes = p->chat_cap * 4; break;
         case SPGEMM_VIEW_CROWPTR:
             if (p->state < 3) return fail(SPGEMM_ERR_STATE, "C row pointers exist after merge");
             src = p->crowptr; bytes = (p->m + 1) * 8; break;
@@ -785,7 +795,7 @@ int spgemm_row_partition(const spgemm_csc_t *A, const spgemm_csr_t *B, int32_t p
         }
         if (A->nnz > 0)
             LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(A->nnz, 8), 256), 256, 0, s>>>(
-                p->a_colptr, p->a_rowidx, K, A->nnz, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg));
+                p->a_colptr, p->a_rowidx, K, A->nnz, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg, nullptr));
         TRY(scan_excl(p, p->rowwork, M, p->rowoff, s, "row_offsets"));
         LAUNCH("partition_bounds", s, k_partition_bounds<<<(unsigned)cdiv(parts + 1, 128), 128, 0, s>>>(p->rowoff, M, parts, bounds));
         CK(cudaMemcpyAsync(bounds_host, bounds, (parts + 1) * 8, cudaMemcpyDeviceToHost, s));
