@@ -435,6 +435,290 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
     }
 }
 
+// --------------------------------------------------------- batched multi-row bucket sort ---
+// Rows of a bin are short (C2: 100-1000 products, 4-18 runs), so per-row fixed costs dominate a
+// one-row-per-group sort.  A CTA claims kBatchRows rows of its bin list and packs them, in list
+// order, into sub-batches of at most CAPN bucket slots; each sub-batch is sorted as ONE problem
+// whose buckets are row-major: row r owns buckets [bbase[r], bbase[r] + nb[r]), nb[r] =
+// 2^ceil(log2 L_r), covering its column span.  Ordering buckets by row makes the sorted array
+// row-major, so the segmented reduction and the copy-out of every row follow directly.
+//   load   : thread t owns CAPN/T consecutive slots (int4 loads; runs are 16-byte aligned and
+//            bucket lengths multiples of 4, so a 4-slot group never straddles two rows)
+//   min/max: per-row span by shared-memory atomicMin/Max (one per row segment of a thread)
+//   sort   : histogram -> scan -> atomic-rank scatter -> in-bucket ranking by counting
+//   reduce : fp64 over equal (row, col) runs, compacted in order; row r's output starts at uoff[r]
+//   store  : one warp per row copies its merged entries to the head of its Ĉ bucket
+constexpr int kBatchRows = 64;
+
+template <int THREADS, int CAPN>
+struct BatchSmem {
+    static constexpr int kNbMax = 2 * CAPN;     // sum of per-row bucket counts <= 2 * slots
+    static constexpr int kBytes = CAPN * 16 + kNbMax * 4;
+};
+
+template <int THREADS, int CAPN>
+__global__ void __launch_bounds__(THREADS) k_merge_batch(const int32_t *__restrict__ rows, int64_t nrows,
+                                                         const int64_t *__restrict__ rowoff,
+                                                         const int64_t *__restrict__ rowwork,
+                                                         int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
+                                                         int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows,
+                                                         unsigned *__restrict__ fb_count) {
+    constexpr int NW = THREADS / 32;
+    constexpr int EPT = CAPN / THREADS;                    // slots per thread (multiple of 4)
+    static_assert(EPT % 4 == 0, "EPT must be a multiple of 4");
+    using S = BatchSmem<THREADS, CAPN>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    int32_t *dk = (int32_t *)smem_raw;
+    float *dv = (float *)(smem_raw + CAPN * 4);
+    int32_t *dk2 = (int32_t *)(smem_raw + CAPN * 8);
+    float *dv2 = (float *)(smem_raw + CAPN * 12);
+    int *hist = (int *)(smem_raw + CAPN * 16);
+    __shared__ int r_row[kBatchRows], r_cap[kBatchRows + 1], r_len[kBatchRows + 1];
+    __shared__ int r_min[kBatchRows], r_max[kBatchRows], r_sh[kBatchRows], r_bb[kBatchRows + 1];
+    __shared__ int r_uoff[kBatchRows + 1];
+    __shared__ int64_t r_src[kBatchRows];
+    __shared__ int sc[NW + 1];
+    __shared__ int s_nsub, s_overflow;
+    const Group<NW, 1> g;
+    const int lane = lane_id(), w = warp_id();
+    for (int64_t c0 = (int64_t)blockIdx.x * kBatchRows; c0 < nrows; c0 += (int64_t)gridDim.x * kBatchRows) {
+        const int nchunk = (int)min((int64_t)kBatchRows, nrows - c0);
+        int done = 0;
+        while (done < nchunk) {
+            // ---- form the next sub-batch: rows [done, done + nsub) of the chunk, caps <= CAPN
+            if (threadIdx.x < 32) {
+                int cap = 0, len = 0, row = 0;
+                int64_t src = 0;
+                int nsub = 0, acc = 0;
+                for (int base = done; base < nchunk; base += 32) {
+                    const int q = base + lane;
+                    if (q < nchunk) {
+                        row = rows[c0 + q];
+                        src = rowoff[row];
+                        cap = (int)(rowoff[row + 1] - src);
+                        len = (int)rowwork[row];
+                    } else {
+                        cap = CAPN + 1;
+                    }
+                    const int inc = warp_incl_sum(cap);
+                    const unsigned fit = __ballot_sync(kFull, acc + inc <= CAPN);
+                    const int take = __popc(fit);            // prefix of lanes that fit
+                    if (lane < take) {
+                        const int r = base - done + lane;
+                        r_row[r] = row;
+                        r_src[r] = src;
+                        r_cap[r] = acc + inc - cap;            // exclusive slot offset
+                        r_len[r] = len;
+                    }
+                    acc += __shfl_sync(kFull, inc, max(take - 1, 0)) * (take > 0);
+                    nsub += take;
+                    if (take < 32) break;
+                }
+                if (lane == 0) {
+                    r_cap[nsub] = acc;
+                    s_nsub = nsub;
+                    s_overflow = 0;
+                }
+            }
+            __syncthreads();
+            const int nsub = s_nsub;
+            const int N = r_cap[nsub];
+            // per-row prefix of product counts (sorted row starts) and init of row spans
+            if (threadIdx.x < 32) {
+                int run = 0;
+                for (int base = 0; base < nsub; base += 32) {
+                    const int q = base + lane;
+                    const int l = q < nsub ? r_len[q] : 0;
+                    const int inc = warp_incl_sum(l);
+                    if (q < nsub) {
+                        r_len[q] = run + inc - l;   // now: sorted start of row q
+                        r_min[q] = kKeyPad;
+                        r_max[q] = 0;
+                    }
+                    run += __shfl_sync(kFull, inc, 31);
+                }
+                if (lane == 0) r_len[nsub] = run;
+            }
+            __syncthreads();
+            // ---- load: thread owns slots [t*EPT, t*EPT + EPT)
+            int32_t key[EPT];
+            float val[EPT];
+            int rid[EPT / 4];
+            const int p0 = threadIdx.x * EPT;
+            {
+                int lo = 0, hi = nsub;     // row of slot p0: last r with r_cap[r] <= p0
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (r_cap[mid] <= p0) lo = mid; else hi = mid;
+                }
+                int r = lo;
+                int32_t mn = kKeyPad, mx = 0;
+#pragma unroll
+                for (int v = 0; v < EPT / 4; ++v) {
+                    const int p = p0 + 4 * v;
+                    if (p < N) {
+                        while (r_cap[r + 1] <= p) {
+                            if (mn != kKeyPad) { atomicMin(&r_min[r], mn); atomicMax(&r_max[r], mx); }
+                            mn = kKeyPad;
+                            mx = 0;
+                            ++r;
+                        }
+                        const int64_t src = r_src[r] + (p - r_cap[r]);
+                        const int4 c4 = *reinterpret_cast<const int4 *>(chat_col + src);
+                        const float4 v4 = *reinterpret_cast<const float4 *>(chat_val + src);
+                        key[4 * v + 0] = c4.x; key[4 * v + 1] = c4.y; key[4 * v + 2] = c4.z; key[4 * v + 3] = c4.w;
+                        val[4 * v + 0] = v4.x; val[4 * v + 1] = v4.y; val[4 * v + 2] = v4.z; val[4 * v + 3] = v4.w;
+                        rid[v] = r;
+#pragma unroll
+                        for (int u = 0; u < 4; ++u)
+                            if (key[4 * v + u] != kKeyPad) { mn = min(mn, key[4 * v + u]); mx = max(mx, key[4 * v + u]); }
+                    } else {
+                        key[4 * v + 0] = key[4 * v + 1] = key[4 * v + 2] = key[4 * v + 3] = kKeyPad;
+                        rid[v] = -1;
+                    }
+                }
+                if (mn != kKeyPad && r < nsub) { atomicMin(&r_min[r], mn); atomicMax(&r_max[r], mx); }
+            }
+            __syncthreads();
+            // ---- per-row bucket ranges
+            if (threadIdx.x < 32) {
+                int run = 0;
+                for (int base = 0; base < nsub; base += 32) {
+                    const int q = base + lane;
+                    int nb = 0;
+                    if (q < nsub) {
+                        const int lq = r_len[q + 1] - r_len[q];
+                        const int lognb = nextpow2_log(max(lq, 1));
+                        nb = 1 << lognb;
+                        const uint32_t span = (uint32_t)(r_max[q] - r_min[q]);
+                        const int bits = span ? 32 - __clz(span) : 0;
+                        r_sh[q] = max(0, bits - lognb);
+                    }
+                    const int inc = warp_incl_sum(nb);
+                    if (q < nsub) r_bb[q] = run + inc - nb;
+                    run += __shfl_sync(kFull, inc, 31);
+                }
+                if (lane == 0) r_bb[nsub] = run;
+            }
+            __syncthreads();
+            const int NB = r_bb[nsub];
+            for (int b = threadIdx.x; b < NB; b += THREADS) hist[b] = 0;
+            __syncthreads();
+            int bkt[EPT];
+#pragma unroll
+            for (int e = 0; e < EPT; ++e) {
+                bkt[e] = -1;
+                if (key[e] != kKeyPad) {
+                    const int r = rid[e / 4];
+                    bkt[e] = r_bb[r] + ((key[e] - r_min[r]) >> r_sh[r]);
+                    atomicAdd(&hist[bkt[e]], 1);
+                }
+            }
+            __syncthreads();
+            // scan of the histogram (thread owns a contiguous bucket range) + overflow check
+            const int bpt = (NB + THREADS - 1) / THREADS;
+            const int b0 = min(NB, (int)threadIdx.x * bpt), b1 = min(NB, b0 + bpt);
+            int cnt = 0, mxc = 0;
+            for (int b = b0; b < b1; ++b) {
+                const int c = hist[b];
+                cnt += c;
+                mxc = max(mxc, c);
+            }
+            if (mxc > kBucketMax) s_overflow = 1;
+            int tot;
+            int ex = g.excl_sum(cnt, sc, &tot);   // (contains barriers: s_overflow visible after)
+            if (s_overflow) {
+                // a bucket too full for the in-bucket ranking: these rows take the merge-path fallback
+                for (int q = threadIdx.x; q < nsub; q += THREADS) fb_rows[atomicAdd(fb_count, 1u)] = r_row[q];
+                done += nsub;
+                __syncthreads();
+                continue;
+            }
+            for (int b = b0; b < b1; ++b) {
+                const int c = hist[b];
+                hist[b] = ex;
+                ex += c;
+            }
+            __syncthreads();
+            int pos[EPT];
+#pragma unroll
+            for (int e = 0; e < EPT; ++e) {
+                pos[e] = -1;
+                if (bkt[e] >= 0) {
+                    pos[e] = atomicAdd(&hist[bkt[e]], 1);
+                    dk[pos[e]] = key[e];
+                }
+            }
+            __syncthreads();
+#pragma unroll
+            for (int e = 0; e < EPT; ++e) {
+                if (pos[e] >= 0) {
+                    const int bs = bkt[e] ? hist[bkt[e] - 1] : 0, be = hist[bkt[e]];
+                    const int32_t kk = key[e];
+                    int rank = 0;
+                    for (int q = bs; q < be; ++q) {
+                        const int32_t kq = dk[q];
+                        rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
+                    }
+                    dk2[bs + rank] = kk;
+                    dv2[bs + rank] = val[e];
+                }
+            }
+            __syncthreads();
+            // ---- reduce: contiguous slices of the sorted array [0, tot); heads at row starts too
+            const int L = tot;
+            const int E = (L + THREADS - 1) / THREADS;
+            const int q0 = min(L, (int)threadIdx.x * E), q1 = min(L, q0 + E);
+            int r;
+            {
+                int lo = 0, hi = nsub;     // row of sorted position q0
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (r_len[mid] <= q0) lo = mid; else hi = mid;
+                }
+                r = lo;
+            }
+            int nh = 0;
+            {
+                int rr = r;
+                for (int q = q0; q < q1; ++q) {
+                    while (r_len[rr + 1] <= q) ++rr;
+                    nh += (q == r_len[rr] || dk2[q] != dk2[q - 1]);
+                }
+            }
+            int U;
+            int o = g.excl_sum(nh, sc, &U);
+            for (int q = q0; q < q1; ++q) {
+                while (r_len[r + 1] <= q) ++r;
+                const bool rs = q == r_len[r];
+                if (rs || dk2[q] != dk2[q - 1]) {
+                    if (rs) r_uoff[r] = o;
+                    const int32_t kk = dk2[q];
+                    double acc = (double)dv2[q];
+                    for (int t2 = q + 1; t2 < r_len[r + 1] && dk2[t2] == kk; ++t2) acc += (double)dv2[t2];
+                    dk[o] = kk;
+                    dv[o] = (float)acc;
+                    ++o;
+                }
+            }
+            if (threadIdx.x == 0) r_uoff[nsub] = U;
+            __syncthreads();
+            // ---- store: warp per row, merged entries to the head of the row's bucket
+            for (int q = w; q < nsub; q += NW) {
+                const int u0 = r_uoff[q], u1 = r_uoff[q + 1];
+                const int64_t dst = r_src[q];
+                for (int t2 = u0 + lane; t2 < u1; t2 += 32) {
+                    chat_col[dst + t2 - u0] = dk[t2];
+                    chat_val[dst + t2 - u0] = dv[t2];
+                }
+                if (lane == 0) ccount[r_row[q]] = u1 - u0;
+            }
+            done += nsub;
+            __syncthreads();
+        }
+    }
+}
+
 // Load Ĉ[s, s+L) into smem (cp.async), sort, reduce, write the merged row back to Ĉ[s, ...).
 template <int NW, int GROUPS, int CAP>
 __device__ __forceinline__ int merge_row_in_smem(const Group<NW, GROUPS> &g, unsigned char *slice, int *sc,

@@ -242,6 +242,18 @@ static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *ro
     return SPGEMM_OK;
 }
 
+template <int THREADS, int CAPN>
+static int launch_batch_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
+                            int ctas_per_sm) {
+    if (cnt == 0) return SPGEMM_OK;
+    const int smem = BatchSmem<THREADS, CAPN>::kBytes;
+    CK(cudaFuncSetAttribute(k_merge_batch<THREADS, CAPN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    const int64_t grid = std::min<int64_t>(cdiv(cnt, kBatchRows), (int64_t)p->num_sms * ctas_per_sm * 4);
+    LAUNCH(name, s, k_merge_batch<THREADS, CAPN><<<(unsigned)grid, THREADS, smem, s>>>(
+        rows, cnt, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
+    return SPGEMM_OK;
+}
+
 // ------------------------------------------------------------------ ABI ------------------
 extern "C" {
 
@@ -582,12 +594,10 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
                                                                                       p->chat_col, p->chat_val, p->ccount));
     CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
-    rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-    TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
-    rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-    TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
-    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-    TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    rows = rows_of(kRowBucketSort256, kRowBucketSort1K + 1, &cnt);       // rows of <= 1024 slots
+    TRY(launch_batch_bin<256, 2048>(p, s, rows, cnt, "merge_batch2k", 4));
+    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);        // rows of <= 4096 slots
+    TRY(launch_batch_bin<512, 4096>(p, s, rows, cnt, "merge_batch4k", 2));
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
