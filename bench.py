@@ -162,6 +162,9 @@ def main():
         inp, A, B = inp_full, A_full, B_full
     stream = torch.cuda.current_stream(dev)
     opts = dict(validate=0)
+    if os.environ.get("SPGEMM_MERGE_VARIANT"):
+        v = (0,) * 16
+        opts["reserved"] = tuple([int(os.environ["SPGEMM_MERGE_VARIANT"])] + [0] * 15)
     flush = torch.zeros(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
 
     def step():

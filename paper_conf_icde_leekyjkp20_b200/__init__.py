@@ -151,6 +151,10 @@ def options(**kw) -> Options:
     for k, v in kw.items():
         if not hasattr(o, k):
             raise KeyError(k)
+        if k == "reserved":
+            for q, x in enumerate(v):
+                o.reserved[q] = x
+            continue
         setattr(o, k, v)
     return o
 

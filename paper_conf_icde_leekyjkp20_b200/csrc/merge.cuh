@@ -435,6 +435,187 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
     }
 }
 
+// ------------------------------------------------------------ warp natural merge (WNM) ---
+// One warp per row of at most CAP slots.  Elements are packed as u64 = (col << 32) | val bits,
+// so ascending u64 order is ascending column order and a merge step is one 64-bit compare.
+// The row's runs (one per a_ik, padded with INT32_MAX sentinels that sort last) are detected
+// as strictly-descending steps, then merged pairwise level by level (merge path per lane);
+// bounds live in a per-warp array of <= 33 entries (rows with more runs go to the fallback).
+__device__ __forceinline__ unsigned long long lds64(unsigned a) {
+    unsigned long long v;
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts64(unsigned a, unsigned long long v) {
+    asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+__device__ __forceinline__ int lds32(unsigned a) {
+    int v;
+    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts32(unsigned a, int v) { asm volatile("st.shared.s32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
+__device__ __forceinline__ unsigned long long pack_kv(int32_t k, float v) {
+    return ((unsigned long long)(uint32_t)k << 32) | (unsigned long long)__float_as_uint(v);
+}
+__device__ __forceinline__ int32_t pk_key(unsigned long long x) { return (int32_t)(x >> 32); }
+__device__ __forceinline__ float pk_val(unsigned long long x) { return __uint_as_float((unsigned)x); }
+
+constexpr int kWnmMaxRuns = 32;
+
+template <int CAP, int WARPS>
+struct WnmSmem {
+    static constexpr int kWarpBytes = CAP * 16 + 2 * (kWnmMaxRuns + 2) * 4;
+    static constexpr int kBytes = kWarpBytes * WARPS;
+};
+
+template <int CAP, int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) k_merge_wnm(const int32_t *__restrict__ rows, int64_t nrows,
+                                                         const int64_t *__restrict__ rowoff,
+                                                         const int64_t *__restrict__ rowwork,
+                                                         int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
+                                                         int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows,
+                                                         unsigned *__restrict__ fb_count) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int lane = lane_id(), w = warp_id();
+    const unsigned base = (unsigned)__cvta_generic_to_shared(smem_raw) + w * WnmSmem<CAP, WARPS>::kWarpBytes;
+    const unsigned bufA = base, bufB = base + CAP * 8;
+    const unsigned bndA = base + CAP * 16, bndB = bndA + (kWnmMaxRuns + 2) * 4;
+    for (int64_t r = (int64_t)blockIdx.x * WARPS + w; r < nrows; r += (int64_t)gridDim.x * WARPS) {
+        const int i = rows[r];
+        const int64_t s = rowoff[i];
+        const int Lc = (int)(rowoff[i + 1] - s);   // slots (multiple of 4)
+        const int Lv = (int)rowwork[i];            // products
+        // ---- load (16-byte vectors) and pack
+        for (int v = lane; v < (Lc >> 2); v += 32) {
+            const int4 c4 = *reinterpret_cast<const int4 *>(chat_col + s + 4 * v);
+            const float4 x4 = *reinterpret_cast<const float4 *>(chat_val + s + 4 * v);
+            sts64(bufA + 32 * v + 0, pack_kv(c4.x, x4.x));
+            sts64(bufA + 32 * v + 8, pack_kv(c4.y, x4.y));
+            sts64(bufA + 32 * v + 16, pack_kv(c4.z, x4.z));
+            sts64(bufA + 32 * v + 24, pack_kv(c4.w, x4.w));
+        }
+        __syncwarp();
+        // ---- run heads (strict descent), lane owns slots [lane*E, lane*E + E)
+        const int E = (Lc + 31) >> 5;
+        const int p0 = min(Lc, lane * E), p1 = min(Lc, p0 + E);
+        int nh = 0;
+        {
+            unsigned long long prev = p0 > 0 ? lds64(bufA + 8 * (p0 - 1)) : 0ull;
+            for (int p = p0; p < p1; ++p) {
+                const unsigned long long x = lds64(bufA + 8 * p);
+                nh += (p == 0 || pk_key(x) < pk_key(prev));
+                prev = x;
+            }
+        }
+        const int inc = warp_incl_sum(nh);
+        const int R = __shfl_sync(kFull, inc, 31);
+        if (R > kWnmMaxRuns) {
+            if (lane == 0) fb_rows[atomicAdd(fb_count, 1u)] = i;
+            __syncwarp();
+            continue;
+        }
+        {
+            int pos = inc - nh;
+            unsigned long long prev = p0 > 0 ? lds64(bufA + 8 * (p0 - 1)) : 0ull;
+            for (int p = p0; p < p1; ++p) {
+                const unsigned long long x = lds64(bufA + 8 * p);
+                if (p == 0 || pk_key(x) < pk_key(prev)) sts32(bndA + 4 * pos++, p);
+                prev = x;
+            }
+            if (lane == 0) sts32(bndA + 4 * R, Lc);
+        }
+        __syncwarp();
+        unsigned src = bufA, dst = bufB, bs = bndA, bd = bndB;
+        int nr = R;
+        while (nr > 1) {
+            const int npairs = (nr + 1) >> 1;
+            if (p0 < p1) {
+                int lo = 0, hi = npairs;       // pair q: last q with start(2q) <= p0
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (lds32(bs + 8 * mid) <= p0) lo = mid; else hi = mid;
+                }
+                int q = lo, o = p0;
+                while (o < p1) {
+                    const int a0 = lds32(bs + 8 * q);
+                    const int a1 = lds32(bs + 4 * min(2 * q + 1, nr));
+                    const int b1 = lds32(bs + 4 * min(2 * q + 2, nr));
+                    const int na = a1 - a0, nb = b1 - a1;
+                    const int d = o - a0;
+                    int ilo = max(0, d - nb), ihi = min(d, na);
+                    while (ilo < ihi) {         // merge path: first i with A[i] > B[d-i-1]
+                        const int mi = (ilo + ihi) >> 1;
+                        if (lds64(src + 8 * (a0 + mi)) <= lds64(src + 8 * (a1 + d - mi - 1))) ilo = mi + 1;
+                        else ihi = mi;
+                    }
+                    int ia = a0 + ilo, jb = a1 + d - ilo;
+                    unsigned long long xa = ia < a1 ? lds64(src + 8 * ia) : ~0ull;
+                    unsigned long long xb = jb < b1 ? lds64(src + 8 * jb) : ~0ull;
+                    const int oend = min(p1, b1);
+                    for (; o < oend; ++o) {
+                        const bool tA = xa <= xb;
+                        sts64(dst + 8 * o, tA ? xa : xb);
+                        if (tA) {
+                            ++ia;
+                            xa = ia < a1 ? lds64(src + 8 * ia) : ~0ull;
+                        } else {
+                            ++jb;
+                            xb = jb < b1 ? lds64(src + 8 * jb) : ~0ull;
+                        }
+                    }
+                    ++q;
+                }
+            }
+            __syncwarp();
+            for (int q = lane; q <= npairs; q += 32)
+                sts32(bd + 4 * q, q < npairs ? lds32(bs + 8 * q) : Lc);
+            __syncwarp();
+            { const unsigned t = src; src = dst; dst = t; }
+            { const unsigned t = bs; bs = bd; bd = t; }
+            nr = npairs;
+        }
+        // ---- segmented reduction over [0, Lv) (sentinels sorted last), compacted into dst
+        const int Ev = (Lv + 31) >> 5;
+        const int v0 = min(Lv, lane * Ev), v1 = min(Lv, v0 + Ev);
+        int nu = 0;
+        {
+            int32_t pk = v0 > 0 ? pk_key(lds64(src + 8 * (v0 - 1))) : -1;
+            for (int p = v0; p < v1; ++p) {
+                const int32_t k = pk_key(lds64(src + 8 * p));
+                nu += (p == 0 || k != pk);
+                pk = k;
+            }
+        }
+        const int uinc = warp_incl_sum(nu);
+        const int U = __shfl_sync(kFull, uinc, 31);
+        {
+            int o = uinc - nu;
+            for (int p = v0; p < v1; ++p) {
+                const unsigned long long x = lds64(src + 8 * p);
+                if (p == 0 || pk_key(x) != pk_key(lds64(src + 8 * (p - 1)))) {
+                    double acc = (double)pk_val(x);
+                    int q = p + 1;
+                    for (; q < Lv; ++q) {
+                        const unsigned long long y = lds64(src + 8 * q);
+                        if (pk_key(y) != pk_key(x)) break;
+                        acc += (double)pk_val(y);
+                    }
+                    sts64(dst + 8 * o++, pack_kv(pk_key(x), (float)acc));
+                }
+            }
+        }
+        __syncwarp();
+        for (int t = lane; t < U; t += 32) {
+            const unsigned long long x = lds64(dst + 8 * t);
+            chat_col[s + t] = pk_key(x);
+            chat_val[s + t] = pk_val(x);
+        }
+        if (lane == 0) ccount[i] = U;
+        __syncwarp();
+    }
+}
+
 // --------------------------------------------------------- batched multi-row bucket sort ---
 // Rows of a bin are short (C2: 100-1000 products, 4-18 runs), so per-row fixed costs dominate a
 // one-row-per-group sort.  A CTA claims kBatchRows rows of its bin list and packs them, in list

@@ -254,6 +254,18 @@ static int launch_batch_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *row
     return SPGEMM_OK;
 }
 
+template <int CAP, int WARPS>
+static int launch_wnm_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
+                          int ctas_per_sm) {
+    if (cnt == 0) return SPGEMM_OK;
+    const int smem = WnmSmem<CAP, WARPS>::kBytes;
+    CK(cudaFuncSetAttribute(k_merge_wnm<CAP, WARPS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    const int64_t grid = std::min<int64_t>(cdiv(cnt, WARPS), (int64_t)p->num_sms * ctas_per_sm * 8);
+    LAUNCH(name, s, k_merge_wnm<CAP, WARPS><<<(unsigned)grid, WARPS * 32, smem, s>>>(
+        rows, cnt, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
+    return SPGEMM_OK;
+}
+
 // ------------------------------------------------------------------ ABI ------------------
 extern "C" {
 
@@ -594,10 +606,36 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
                                                                                       p->chat_col, p->chat_val, p->ccount));
     CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
-    rows = rows_of(kRowBucketSort256, kRowBucketSort1K + 1, &cnt);       // rows of <= 1024 slots
-    TRY(launch_batch_bin<256, 2048>(p, s, rows, cnt, "merge_batch2k", 4));
-    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);        // rows of <= 4096 slots
-    TRY(launch_batch_bin<512, 4096>(p, s, rows, cnt, "merge_batch4k", 2));
+    // merge_variant (options.reserved[0], tuning): 0 per-row bucket sort (default),
+    // 1 batched multi-row bucket sort, 2 per-row bucket sort with 16 slots per thread
+    const int variant = p->opt.reserved[0];
+    if (variant == 1) {
+        rows = rows_of(kRowBucketSort256, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_batch_bin<256, 2048>(p, s, rows, cnt, "merge_batch2k", 4));
+        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+        TRY(launch_batch_bin<512, 4096>(p, s, rows, cnt, "merge_batch4k", 2));
+    } else if (variant == 2) {
+        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
+        TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
+        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_bucket_bin<2, 4, 16>(p, s, rows, cnt, "merge_bucket1k", 4));
+        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+        TRY(launch_bucket_bin<8, 1, 16>(p, s, rows, cnt, "merge_bucket4k", 4));
+    } else if (variant == 3) {
+        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
+        TRY(launch_wnm_bin<256, 8>(p, s, rows, cnt, "merge_wnm256", 6));
+        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_wnm_bin<1024, 4>(p, s, rows, cnt, "merge_wnm1k", 3));
+        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    } else {
+        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
+        TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
+        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
+        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    }
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
