@@ -152,7 +152,7 @@ template <int NW, int GROUPS, int CAP>
 __device__ __forceinline__ int natural_merge_sort(const Group<NW, GROUPS> &g, int32_t *k0, float *v0, int32_t *k1,
                                                   float *v1, int *bA, int *bB, int L, int *sc) {
     constexpr int T = NW * 32;
-    const int E = (L + T - 1) / T;
+    const int E = ((L + T - 1) / T) | 1;
     const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
     // run heads: p == 0 or k[p] <= k[p-1]
     int nh = 0;
@@ -229,7 +229,7 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
                                                     int L, int32_t *__restrict__ out_col, float *__restrict__ out_val,
                                                     int *sc) {
     constexpr int T = NW * 32;
-    const int E = (L + T - 1) / T;
+    const int E = ((L + T - 1) / T) | 1;
     const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
     int nh = 0;
     for (int p = p0; p < p1; ++p) nh += (p == 0 || k[p] != k[p - 1]);
@@ -368,7 +368,7 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     g.sync();
     // 3. segmented reduction over contiguous slices (fp64), compacted into (dk, dv)
     L = tot;   // valid (non-sentinel) entries
-    const int E = (L + T - 1) / T;
+    const int E = ((L + T - 1) / T) | 1;     // odd stride between thread slices: no bank conflicts
     const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
     int nh = 0;
     for (int p = p0; p < p1; ++p) nh += (p == 0 || dk2[p] != dk2[p - 1]);
@@ -497,7 +497,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_merge_wnm(const int32_t *__restr
         }
         __syncwarp();
         // ---- run heads (strict descent), lane owns slots [lane*E, lane*E + E)
-        const int E = (Lc + 31) >> 5;
+        const int E = ((Lc + 31) >> 5) | 1;   // odd lane stride: conflict-free smem slices
         const int p0 = min(Lc, lane * E), p1 = min(Lc, p0 + E);
         int nh = 0;
         {
@@ -576,7 +576,7 @@ __global__ void __launch_bounds__(WARPS * 32) k_merge_wnm(const int32_t *__restr
             nr = npairs;
         }
         // ---- segmented reduction over [0, Lv) (sentinels sorted last), compacted into dst
-        const int Ev = (Lv + 31) >> 5;
+        const int Ev = ((Lv + 31) >> 5) | 1;
         const int v0 = min(Lv, lane * Ev), v1 = min(Lv, v0 + Ev);
         int nu = 0;
         {
@@ -848,7 +848,7 @@ __global__ void __launch_bounds__(THREADS) k_merge_batch(const int32_t *__restri
             __syncthreads();
             // ---- reduce: contiguous slices of the sorted array [0, tot); heads at row starts too
             const int L = tot;
-            const int E = (L + THREADS - 1) / THREADS;
+            const int E = ((L + THREADS - 1) / THREADS) | 1;
             const int q0 = min(L, (int)threadIdx.x * E), q1 = min(L, q0 + E);
             int r;
             {
