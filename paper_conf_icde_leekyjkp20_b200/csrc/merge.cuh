@@ -410,7 +410,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
                                                                   float *__restrict__ chat_val,
                                                                   int64_t *__restrict__ ccount,
                                                                   int32_t *__restrict__ fb_rows,
-                                                                  unsigned *__restrict__ fb_count) {
+                                                                  unsigned *__restrict__ fb_count, int64_t cap_skip) {
     using S = BucketSmem<NW, EPT>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ int sc_all[GROUPS][NW + 1];
@@ -425,14 +425,17 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
         const int i = rows[r];
         const int64_t s = rowoff[i];
         const int L = (int)(rowoff[i + 1] - s);
+        if (L > S::kCap) continue;          // (limited list) rows above this kernel's capacity
         const int U = bucket_sort_reduce<NW, GROUPS, EPT>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
                                                           chat_col + s, chat_val + s, sc_all[g.gid]);
         if (g.gtid == 0) {
             if (U >= 0) ccount[i] = U;
-            else fb_rows[atomicAdd(fb_count, 1u)] = i;
+            else if (fb_rows) fb_rows[atomicAdd(fb_count, 1u)] = i;
+            else ccount[i] = -1;   // limited list: k_merge_limited takes the row (merge-path fallback)
         }
         g.sync();
     }
+    (void)cap_skip;
 }
 
 // ------------------------------------------------------------ warp natural merge (WNM) ---
@@ -990,6 +993,7 @@ struct LimitedArgs {
     int64_t max_deg;
     int64_t stage_cap;
     unsigned long long *row_counter;
+    int skip_small;
 };
 
 __device__ __forceinline__ void smem_add_f64(double *addr, double v) {
@@ -1034,6 +1038,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t s = g.rowoff[i];
         const int64_t cap = g.rowoff[i + 1] - s;   // padded bucket length
         const int64_t L = g.rowwork[i];             // products
+        if (cap <= kLimCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
         if (cap <= kLimCap) {
             int32_t *dk = (int32_t *)smem_raw;
             float *dv = (float *)(smem_raw + kLimCap * 4);

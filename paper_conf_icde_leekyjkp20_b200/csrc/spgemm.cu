@@ -232,13 +232,13 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
 
 template <int NW, int GROUPS, int EPT>
 static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
-                             int ctas_per_sm) {
+                             int ctas_per_sm, bool fallback_list = true) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT>::kBytes * GROUPS;
     CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
     LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
-        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
+        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0));
     return SPGEMM_OK;
 }
 
@@ -663,8 +663,12 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         g.max_deg = p->lim_max_deg;
         g.stage_cap = p->stage_cap;
         g.row_counter = p->row_counter;
+        g.skip_small = 1;
+        // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
+        // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
+        TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
         CK(cudaFuncSetAttribute(k_merge_limited, cudaFuncAttributeMaxDynamicSharedMemorySize, kLimSmem));
-        LAUNCH("merge_limited", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
+        LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
     }
     TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
     CK(cudaMemcpyAsync(&p->nnz_c, p->crowptr + M, 8, cudaMemcpyDeviceToHost, s));
