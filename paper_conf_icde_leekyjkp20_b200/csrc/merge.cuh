@@ -971,9 +971,12 @@ constexpr int kLimCap = 9216;
 constexpr int kLimEPT = kLimCap / kLimThreads;   // 18
 constexpr int kLimWindow = 16384;
 constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
-constexpr int kLimSmem = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
-                               kLimCap * 16 + ceil_pow2(kLimCap) * 4,     // bucket sort
-                               kLimWindow * 8 + (kLimWindow / 32) * 4);   // dense window
+constexpr int kLimSortBytes = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
+                                    kLimCap * 16 + ceil_pow2(kLimCap) * 4,     // bucket sort
+                                    kLimWindow * 8 + (kLimWindow / 32) * 4);   // dense window
+constexpr int kCoarseLog = 10;
+constexpr int kCoarseBins = 1 << kCoarseLog;
+constexpr int kLimSmem = kLimSortBytes + (3 * kCoarseBins + 1) * 4;           // + coarse partition tables
 
 struct LimitedArgs {
     const int32_t *rows;          // limited rows, longest first
@@ -994,6 +997,7 @@ struct LimitedArgs {
     int64_t stage_cap;
     unsigned long long *row_counter;
     int skip_small;
+    int64_t coarse_cap;           // rows up to this many slots take the coarse-partition path
 };
 
 __device__ __forceinline__ void smem_add_f64(double *addr, double v) {
@@ -1137,6 +1141,90 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 __syncthreads();
             }
         } else {
+            bool done_coarse = false;
+            if (cap <= g.coarse_cap) {
+                // sparse long row: coarse column partition through global scratch (two coalesced passes)
+                //  1. histogram over kCoarseBins column ranges; greedy groups of <= kLimCap entries
+                //  2. scatter the row into the block's scratch, grouped by column range
+                //  3. per group (ascending): smem bucket sort (merge-path fallback), merged entries
+                //     appended at the head of the row's bucket -- the row now lives in scratch
+                int *fh = (int *)(smem_raw + kLimSortBytes);      // [kCoarseBins] counts -> group id
+                int *gstart = fh + kCoarseBins;                    // [kCoarseBins + 1]
+                int *gcur = gstart + kCoarseBins + 1;              // [kCoarseBins]
+                __shared__ int s_ngroups, s_bad;
+                const uint32_t span32 = (uint32_t)(mx - mn);
+                const int bits = span32 ? 32 - __clz(span32) : 0;
+                const int shc = max(0, bits - kCoarseLog);
+                for (int t = threadIdx.x; t < kCoarseBins; t += kLimThreads) fh[t] = 0;
+                __syncthreads();
+                for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+                    const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
+                    if (c4.x != kKeyPad) atomicAdd(&fh[(c4.x - mn) >> shc], 1);
+                    if (c4.y != kKeyPad) atomicAdd(&fh[(c4.y - mn) >> shc], 1);
+                    if (c4.z != kKeyPad) atomicAdd(&fh[(c4.z - mn) >> shc], 1);
+                    if (c4.w != kKeyPad) atomicAdd(&fh[(c4.w - mn) >> shc], 1);
+                }
+                __syncthreads();
+                if (threadIdx.x == 0) {                            // greedy grouping of consecutive bins
+                    int ng = 0, acc = 0, bad = 0;
+                    gstart[0] = 0;
+                    for (int b = 0; b < kCoarseBins; ++b) {
+                        const int c = fh[b];
+                        if (c > kLimCap) bad = 1;
+                        if (acc + c > kLimCap && acc > 0) {
+                            ++ng;
+                            gstart[ng] = gstart[ng - 1] + acc;
+                            acc = 0;
+                        }
+                        acc += c;
+                        fh[b] = ng;
+                    }
+                    ++ng;
+                    gstart[ng] = gstart[ng - 1] + acc;
+                    s_ngroups = ng;
+                    s_bad = bad;
+                }
+                __syncthreads();
+                if (!s_bad) {   // (a single column range holding > kLimCap products: window path)
+                    const int ng = s_ngroups;
+                    int32_t *sc_col = g.scratch_col + (int64_t)blockIdx.x * g.stage_cap;
+                    float *sc_val = g.scratch_val + (int64_t)blockIdx.x * g.stage_cap;
+                    for (int t = threadIdx.x; t < ng; t += kLimThreads) gcur[t] = gstart[t];
+                    __syncthreads();
+                    for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+                        const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
+                        const float4 v4 = *reinterpret_cast<const float4 *>(g.chat_val + s + 4 * p);
+                        const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
+                        const float vv[4] = {v4.x, v4.y, v4.z, v4.w};
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) {
+                            if (cc[u] == kKeyPad) continue;
+                            const int q = atomicAdd(&gcur[fh[(cc[u] - mn) >> shc]], 1);
+                            sc_col[q] = cc[u];
+                            sc_val[q] = vv[u];
+                        }
+                    }
+                    __syncthreads();
+                    for (int gi = 0; gi < ng; ++gi) {
+                        const int g0 = gstart[gi], n = gstart[gi + 1] - g0;
+                        if (n == 0) continue;
+                        int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(
+                            grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + kLimCap * 4),
+                            (int32_t *)(smem_raw + kLimCap * 8), (float *)(smem_raw + kLimCap * 12),
+                            (int *)(smem_raw + kLimCap * 16), g.chat_col + s + nout, g.chat_val + s + nout, sc);
+                        if (U < 0)
+                            U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, sc_col, sc_val, g0, n, n,
+                                                                      g.chat_col + s + nout, g.chat_val + s + nout);
+                        nout += U;
+                        __syncthreads();
+                    }
+                    if (threadIdx.x == 0) g.ccount[i] = nout;
+                    __syncthreads();
+                    done_coarse = true;
+                }
+                __syncthreads();
+            }
+            if (done_coarse) continue;
             // sparse: windows whose products fit the smem sorter
             int32_t *k0 = (int32_t *)smem_raw;
             float *v0 = (float *)(smem_raw + kLimCap * 4);

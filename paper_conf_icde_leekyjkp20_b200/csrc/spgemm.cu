@@ -664,6 +664,7 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         g.stage_cap = p->stage_cap;
         g.row_counter = p->row_counter;
         g.skip_small = 1;
+        g.coarse_cap = p->stage_cap;
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
