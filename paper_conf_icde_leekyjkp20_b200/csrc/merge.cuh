@@ -1165,24 +1165,46 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     if (c4.w != kKeyPad) atomicAdd(&fh[(c4.w - mn) >> shc], 1);
                 }
                 __syncthreads();
-                if (threadIdx.x == 0) {                            // greedy grouping of consecutive bins
-                    int ng = 0, acc = 0, bad = 0;
-                    gstart[0] = 0;
-                    for (int b = 0; b < kCoarseBins; ++b) {
-                        const int c = fh[b];
-                        if (c > kLimCap) bad = 1;
-                        if (acc + c > kLimCap && acc > 0) {
-                            ++ng;
-                            gstart[ng] = gstart[ng - 1] + acc;
-                            acc = 0;
-                        }
-                        acc += c;
-                        fh[b] = ng;
+                {   // grouping of consecutive bins: group(b) = floor(prefix(b) / (kLimCap/2)); with no bin
+                    // above kLimCap/2 a group holds < kLimCap products.  Bins per thread: 2 (1024 / 512).
+                    constexpr int BPT = kCoarseBins / kLimThreads;
+                    int c[BPT], cnt = 0, mxb = 0;
+#pragma unroll
+                    for (int u = 0; u < BPT; ++u) {
+                        c[u] = fh[threadIdx.x * BPT + u];
+                        cnt += c[u];
+                        mxb = max(mxb, c[u]);
                     }
-                    ++ng;
-                    gstart[ng] = gstart[ng - 1] + acc;
-                    s_ngroups = ng;
-                    s_bad = bad;
+                    int tot;
+                    int ex = grp.excl_sum(cnt, sc, &tot);
+                    mxb = grp.reduce_max(mxb, sc);
+                    constexpr int T = kLimCap / 2;
+#pragma unroll
+                    for (int u = 0; u < BPT; ++u) {
+                        fh[threadIdx.x * BPT + u] = ex / T;     // group id of the bin
+                        ex += c[u];
+                    }
+                    const int ng = (tot + T - 1) / T;
+                    // group start = first prefix value >= gi*T, i.e. prefix of the first bin of group gi
+                    for (int gi = threadIdx.x; gi <= ng; gi += kLimThreads) gstart[gi] = 0x7fffffff;
+                    __syncthreads();
+                    int pre = ex - cnt;
+#pragma unroll
+                    for (int u = 0; u < BPT; ++u) {
+                        atomicMin(&gstart[pre / T], pre);
+                        pre += c[u];
+                    }
+                    if (threadIdx.x == 0) {
+                        s_ngroups = ng;
+                        s_bad = mxb > T;
+                        gstart[ng] = tot;
+                    }
+                    __syncthreads();
+                    // groups with no bin starting inside them cannot exist (bins are contiguous), but
+                    // guard: an untouched start inherits the next group's start (empty group)
+                    if (threadIdx.x == 0)
+                        for (int gi = ng - 1; gi >= 0; --gi)
+                            if (gstart[gi] == 0x7fffffff) gstart[gi] = gstart[gi + 1];
                 }
                 __syncthreads();
                 if (!s_bad) {   // (a single column range holding > kLimCap products: window path)
@@ -1197,11 +1219,18 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                         const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
                         const float vv[4] = {v4.x, v4.y, v4.z, v4.w};
 #pragma unroll
-                        for (int u = 0; u < 4; ++u) {
-                            if (cc[u] == kKeyPad) continue;
-                            const int q = atomicAdd(&gcur[fh[(cc[u] - mn) >> shc]], 1);
-                            sc_col[q] = cc[u];
-                            sc_val[q] = vv[u];
+                        for (int u = 0; u < 4; ++u) {     // warp-aggregated cursor bumps per group
+                            const int gid = cc[u] == kKeyPad ? -1 - lane_id() : fh[(cc[u] - mn) >> shc];
+                            const unsigned peers = __match_any_sync(__activemask(), gid);
+                            if (gid >= 0) {
+                                const int leader = __ffs(peers) - 1;
+                                int q0 = 0;
+                                if (lane_id() == leader) q0 = atomicAdd(&gcur[gid], __popc(peers));
+                                q0 = __shfl_sync(peers, q0, leader);
+                                const int q = q0 + __popc(peers & lanemask_lt());
+                                sc_col[q] = cc[u];
+                                sc_val[q] = vv[u];
+                            }
                         }
                     }
                     __syncthreads();
@@ -1351,6 +1380,32 @@ __global__ void k_merge_pass(const int32_t *__restrict__ rows, int64_t nrows, co
 constexpr int kCompactWarpMax = 8192;
 constexpr int kCompactLongThreads = 512;
 
+// Realign 4-wide vectors for an output shifted by sh (dst mod 4): the aligned output vector of
+// lane m holds source elements [4m - sh, 4m - sh + 4): the last sh of the previous vector and
+// the first 4 - sh of this lane's.  `prev` = the previous lane's vector (lane 0: carried).
+template <typename V>
+__device__ __forceinline__ V realign4(const V &cur, const V &prev, int sh) {
+    V o;
+    switch (sh) {
+        case 0: o = cur; break;
+        case 1: o.x = prev.w; o.y = cur.x; o.z = cur.y; o.w = cur.z; break;
+        case 2: o.x = prev.z; o.y = prev.w; o.z = cur.x; o.w = cur.y; break;
+        default: o.x = prev.y; o.y = prev.z; o.z = prev.w; o.w = cur.x; break;
+    }
+    return o;
+}
+
+template <typename V>
+__device__ __forceinline__ V shfl_up_vec(const V &v, const V &carry) {
+    V p;
+    p.x = __shfl_up_sync(kFull, v.x, 1);
+    p.y = __shfl_up_sync(kFull, v.y, 1);
+    p.z = __shfl_up_sync(kFull, v.z, 1);
+    p.w = __shfl_up_sync(kFull, v.w, 1);
+    if (lane_id() == 0) p = carry;
+    return p;
+}
+
 __global__ void __launch_bounds__(256) k_compact_rows(const int64_t *__restrict__ crowptr, int64_t M,
                                                       const int64_t *__restrict__ rowoff,
                                                       const int32_t *__restrict__ chat_col,
@@ -1362,22 +1417,41 @@ __global__ void __launch_bounds__(256) k_compact_rows(const int64_t *__restrict_
         const int64_t dst = crowptr[i];
         const int64_t cnt = crowptr[i + 1] - dst;
         if (cnt == 0 || cnt > kCompactWarpMax) continue;
-        const int64_t src = rowoff[i];
-        for (int p0 = 0; p0 < cnt; p0 += 128) {
-            int32_t c[4];
-            float v[4];
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                const int p = p0 + q * 32 + lane;
-                c[q] = p < cnt ? chat_col[src + p] : 0;
-                v[q] = p < cnt ? chat_val[src + p] : 0.f;
+        const int64_t src = rowoff[i];               // 16-byte aligned (padded runs)
+        const int sh = (int)(dst & 3);
+        const int64_t dst_a = dst - sh;              // aligned output base
+        // aligned output vector m covers output slots [4m - sh, 4m - sh + 4) of the row
+        const int64_t nvec = (cnt + sh + 3) >> 2;
+        int4 carry_c = make_int4(0, 0, 0, 0);
+        float4 carry_v = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int64_t m0 = 0; m0 < nvec; m0 += 32) {
+            const int64_t m = m0 + lane;
+            int4 c = make_int4(0, 0, 0, 0);
+            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (4 * m < cnt) {
+                c = *reinterpret_cast<const int4 *>(chat_col + src + 4 * m);
+                v = *reinterpret_cast<const float4 *>(chat_val + src + 4 * m);
             }
+            const int4 oc = realign4(c, shfl_up_vec(c, carry_c), sh);
+            const float4 ov = realign4(v, shfl_up_vec(v, carry_v), sh);
+            carry_c.x = __shfl_sync(kFull, c.x, 31); carry_c.y = __shfl_sync(kFull, c.y, 31);
+            carry_c.z = __shfl_sync(kFull, c.z, 31); carry_c.w = __shfl_sync(kFull, c.w, 31);
+            carry_v.x = __shfl_sync(kFull, v.x, 31); carry_v.y = __shfl_sync(kFull, v.y, 31);
+            carry_v.z = __shfl_sync(kFull, v.z, 31); carry_v.w = __shfl_sync(kFull, v.w, 31);
+            if (m < nvec) {
+                const int64_t j0 = 4 * m - sh;       // row slot of the vector's first element
+                if (j0 >= 0 && j0 + 4 <= cnt) {
+                    *reinterpret_cast<int4 *>(out_col + dst_a + 4 * m) = oc;
+                    *reinterpret_cast<float4 *>(out_val + dst_a + 4 * m) = ov;
+                } else {                              // ragged head / tail of the row
+                    const int32_t cc[4] = {oc.x, oc.y, oc.z, oc.w};
+                    const float vv[4] = {ov.x, ov.y, ov.z, ov.w};
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                const int p = p0 + q * 32 + lane;
-                if (p < cnt) {
-                    out_col[dst + p] = c[q];
-                    out_val[dst + p] = v[q];
+                    for (int u = 0; u < 4; ++u)
+                        if (j0 + u >= 0 && j0 + u < cnt) {
+                            out_col[dst_a + 4 * m + u] = cc[u];
+                            out_val[dst_a + 4 * m + u] = vv[u];
+                        }
                 }
             }
         }
