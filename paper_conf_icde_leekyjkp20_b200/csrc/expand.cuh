@@ -142,4 +142,76 @@ __global__ void __launch_bounds__(256) k_expand_gathered(
     for (; e < a1; ++e) store_run4(chat_col, chat_val, __ldg(base + e) + 4 * sub, c4, v4, __ldg(a_val + e));
 }
 
+// B-Gathering, load-balanced: the items of gathering bin n are (pair, A entry) couples, laid out
+// bin list order (pairs sorted by (n, c, k)) with item_off[q] = sum of nnz(a_*k) over earlier
+// pairs of the gather lists.  One lane per item: it writes the pair's whole padded run (<= 8
+// 16-byte vectors) for that A entry, so a warp combines 32 micro-blocks of up to 32 effective
+// threads each and no lane loops over a long A column.
+constexpr int kGatherTile = 512;
+__global__ void __launch_bounds__(256) k_expand_gathered_items(
+    const int32_t *__restrict__ list, const int64_t *__restrict__ item_off, int64_t q_lo, int64_t q_hi,
+    const int64_t *__restrict__ a_colptr, const float *__restrict__ a_val, const int64_t *__restrict__ b_rowptr,
+    const int32_t *__restrict__ b_colidx, const float *__restrict__ b_val, const int64_t *__restrict__ base,
+    int32_t *__restrict__ chat_col, float *__restrict__ chat_val) {
+    __shared__ int64_t s_off[kGatherTile + 1];
+    __shared__ int64_t s_q0;
+    __shared__ int s_n;
+    const int64_t t_beg = item_off[q_lo], t_end = item_off[q_hi];
+    const int64_t ntiles = (t_end - t_beg + kGatherTile - 1) / kGatherTile;
+    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int64_t t0 = t_beg + tile * kGatherTile;
+        if (threadIdx.x == 0) {
+            int64_t lo = q_lo, hi = q_hi;     // pair of item t0: last q with item_off[q] <= t0
+            while (hi - lo > 1) {
+                const int64_t mid = (lo + hi) >> 1;
+                if (item_off[mid] <= t0) lo = mid; else hi = mid;
+            }
+            s_q0 = lo;
+            int64_t lo2 = lo, hi2 = q_hi;     // pairs starting before the tile's end
+            const int64_t t1 = min(t_end, t0 + kGatherTile);
+            while (hi2 - lo2 > 1) {
+                const int64_t mid = (lo2 + hi2) >> 1;
+                if (item_off[mid] < t1) lo2 = mid; else hi2 = mid;
+            }
+            s_n = (int)(lo2 - lo + 1);
+        }
+        __syncthreads();
+        const int64_t q0 = s_q0;
+        const int n = s_n;
+        for (int u = threadIdx.x; u <= n; u += blockDim.x) s_off[u] = item_off[q0 + u];
+        __syncthreads();
+        for (int u = threadIdx.x; u < kGatherTile; u += blockDim.x) {
+            const int64_t t = t0 + u;
+            if (t >= t_end) break;
+            int lo = 0, hi = n;    // pair: last j with s_off[j] <= t
+            while (hi - lo > 1) {
+                const int mid = (lo + hi) >> 1;
+                if (s_off[mid] <= t) lo = mid; else hi = mid;
+            }
+            const int k = __ldg(list + q0 + lo);
+            const int64_t e = __ldg(a_colptr + k) + (t - s_off[lo]);
+            const int64_t b0 = __ldg(b_rowptr + k);
+            const int rb = (int)(__ldg(b_rowptr + k + 1) - b0);
+            const int64_t dst = __ldg(base + e);
+            const float a = __ldg(a_val + e);
+            for (int v = 0; 4 * v < rb; ++v) {
+                int4 c4;
+                float4 v4;
+                load_b4(b_colidx + b0, b_val + b0, 4 * v, rb, c4, v4);
+                store_run4(chat_col, chat_val, dst + 4 * v, c4, v4, a);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// nnz(a_*k) of the gather-list pairs (input of the item prefix scan)
+__global__ void k_gather_item_counts(const int32_t *__restrict__ list, int64_t n, const int64_t *__restrict__ a_colptr,
+                                     int64_t *__restrict__ cnt) {
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
+        const int k = list[q];
+        cnt[q] = a_colptr[k + 1] - a_colptr[k];
+    }
+}
+
 }  // namespace spg

@@ -135,6 +135,8 @@ struct spgemm_plan_s {
     int64_t pair_starts[kNumPairBuckets + 1] = {};
     int64_t row_starts[kNumRowBuckets + 1] = {};
     Piece *pieces = nullptr;
+    int64_t *gather_item_off = nullptr;
+
     int64_t n_split_pieces = 0, n_whole = 0;
     int64_t *piece_off = nullptr;
     int64_t lim_runs = 0, lim_max_deg = 0, lim_max_L = 0, nlim = 0;
@@ -503,6 +505,19 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_whole, 256), 256, 0, s>>>(
             p->pair_order + p->pair_starts[kPairBucketPiece], p->n_whole, p->a_colptr, p->b_rowptr,
             p->pieces + p->n_split_pieces));
+    // B-Gathering items: prefix of nnz(a_*k) over the gather lists (bins are contiguous in it)
+    {
+        const int64_t g_lo = p->pair_starts[kPairBucketGather0], g_hi = p->pair_starts[kPairBucketEmpty];
+        TRY(palloc(p, &p->gather_item_off, g_hi - g_lo + 1, s));
+        if (g_hi > g_lo) {
+            Temp tg(s);
+            int64_t *cnt;
+            TRY(talloc(p, tg, &cnt, g_hi - g_lo));
+            LAUNCH("gather_items", s, k_gather_item_counts<<<grid_for(g_hi - g_lo, 256), 256, 0, s>>>(
+                p->pair_order + g_lo, g_hi - g_lo, p->a_colptr, cnt));
+            TRY(scan_excl(p, cnt, g_hi - g_lo, p->gather_item_off, s, "gather_scan"));
+        }
+    }
     // limited rows: index map, run lists, B-Limited scratch
     p->nlim = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketLim0];
     if (p->nlim > 0) {
@@ -558,7 +573,15 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     if (np > 0)
         LAUNCH("expand_pieces", s, k_expand_pieces<<<(unsigned)np, kPieceThreads, 0, s>>>(
             p->pieces, p->a_val, p->b_rowptr, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
-    for (int nb = 0; nb < 6; ++nb) {
+    const bool items = p->opt.reserved[1] == 0;   // load-balanced B-Gathering (default)
+    {
+        const int64_t g_lo = p->pair_starts[kPairBucketGather0], g_hi = p->pair_starts[kPairBucketEmpty];
+        if (items && g_hi > g_lo)
+            LAUNCH("expand_gathered", s, k_expand_gathered_items<<<(unsigned)p->num_sms * 8, 256, 0, s>>>(
+                p->pair_order + g_lo, p->gather_item_off, 0, g_hi - g_lo, p->a_colptr, p->a_val, p->b_rowptr,
+                p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
+    }
+    for (int nb = 0; nb < 6 && !items; ++nb) {
         const int64_t lo = p->pair_starts[kPairBucketGather0 + nb * 16];
         const int64_t cnt = p->pair_starts[kPairBucketGather0 + nb * 16 + 16] - lo;
         if (cnt == 0) continue;
