@@ -29,7 +29,9 @@ constexpr unsigned kFull = 0xffffffffu;
 // ------------------------------------------------------------------------ warp bin ---
 __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ rows, int64_t nrows,
                                                     const int64_t *__restrict__ rowoff, int32_t *__restrict__ chat_col,
-                                                    float *__restrict__ chat_val, int64_t *__restrict__ ccount) {
+                                                    float *__restrict__ chat_val, int64_t *__restrict__ ccount,
+                                                    const int64_t *__restrict__ crowptr, int32_t *__restrict__ out_col,
+                                                    float *__restrict__ out_val) {
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (gw >= nrows) return;
     const int lane = lane_id();
@@ -66,10 +68,16 @@ __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ 
     const unsigned tails = __ballot_sync(kFull, tail);
     if (tail) {
         const int pos = __popc(tails & lanemask_lt());
-        chat_col[s + pos] = key;
-        chat_val[s + pos] = (float)v;
+        if (out_col) {
+            const int64_t o = crowptr[i];
+            out_col[o + pos] = key;
+            out_val[o + pos] = (float)v;
+        } else {
+            chat_col[s + pos] = key;
+            chat_val[s + pos] = (float)v;
+        }
     }
-    if (lane == 0) ccount[i] = __popc(tails);
+    if (lane == 0 && !out_col) ccount[i] = __popc(tails);
 }
 
 // ------------------------------------------------------------------ thread groups ---
@@ -266,6 +274,10 @@ constexpr int kBucketMax = 64;
 
 __device__ __forceinline__ int nextpow2_log(int x) { return x <= 1 ? 0 : 32 - __clz(x - 1); }
 
+// histogram slot of bucket b: one pad word per 32 buckets, so threads walking contiguous bucket
+// ranges (stride = buckets per thread) hit distinct banks
+__host__ __device__ __forceinline__ constexpr int hidx(int b) { return b + (b >> 5); }
+
 // Copy a warp's contiguous output slice: lane l staged u_l entries at (sk, sv)[st_l ..) and
 // they go to out[wbase + ex_l ..), ex_l = exclusive prefix of u over the warp's lanes.
 __device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const int32_t *sk, const float *sv,
@@ -314,17 +326,20 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     const int nb = 1 << lognb;
     const int bits = span ? 32 - __clz(span) : 0;
     const int sh = max(0, bits - lognb);
-    for (int b = g.gtid; b < nb; b += T) hist[b] = 0;
+    for (int b = g.gtid; b <= hidx(nb); b += T) hist[b] = 0;
     g.sync();
+    // one shared atomic per element (spread-address ATOMS cost ~2 cycles per lane): its return
+    // value is the element's rank inside its bucket, reused by the scatter below
+    int rk[EPT];
 #pragma unroll
     for (int e = 0; e < EPT; ++e)
-        if (key[e] != kKeyPad) atomicAdd(&hist[(key[e] - mn) >> sh], 1);
+        rk[e] = key[e] != kKeyPad ? atomicAdd(&hist[hidx((key[e] - mn) >> sh)], 1) : 0;
     g.sync();
     const int bpt = (nb + T - 1) / T;
     const int b0 = min(nb, g.gtid * bpt), b1 = min(nb, b0 + bpt);
     int cnt = 0, mxc = 0;
     for (int b = b0; b < b1; ++b) {
-        const int c = hist[b];
+        const int c = hist[hidx(b)];
         cnt += c;
         mxc = max(mxc, c);
     }
@@ -332,29 +347,30 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     int ex = g.excl_sum(cnt, sc, &tot);
     if (g.reduce_max(mxc, sc) > kBucketMax) return -1;
     for (int b = b0; b < b1; ++b) {
-        const int c = hist[b];
-        hist[b] = ex;
+        const int c = hist[hidx(b)];
+        hist[hidx(b)] = ex;
         ex += c;
     }
+    if (g.gtid == 0) hist[hidx(nb)] = tot;
     g.sync();
-    // 1. scatter by atomic rank (unordered inside a bucket)
+    // 1. scatter: bucket start + atomic rank (unordered inside a bucket)
     int pos[EPT];
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
         pos[e] = -1;
         if (key[e] != kKeyPad) {
-            pos[e] = atomicAdd(&hist[(key[e] - mn) >> sh], 1);
+            pos[e] = hist[hidx((key[e] - mn) >> sh)] + rk[e];
             dk[pos[e]] = key[e];
         }
     }
     g.sync();
-    // 2. hist[b] = end of bucket b.  Every element counts the keys of its bucket that sort
+    // 2. bucket b = [hist[b], hist[b+1]).  Every element counts the keys of its bucket that sort
     //    before it (smaller, or equal and scattered earlier) and moves to its sorted slot.
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
         if (pos[e] >= 0) {
             const int b = (key[e] - mn) >> sh;
-            const int bs = b ? hist[b - 1] : 0, be = hist[b];
+            const int bs = hist[hidx(b)], be = hist[hidx(b + 1)];
             const int32_t kk = key[e];
             int rank = 0;
             for (int q = bs; q < be; ++q) {
@@ -399,7 +415,7 @@ template <int NW, int EPT>
 struct BucketSmem {
     static constexpr int kCap = NW * 32 * EPT;
     static constexpr int kNb = ceil_pow2(kCap);
-    static constexpr int kBytes = kCap * 16 + kNb * 4;
+    static constexpr int kBytes = kCap * 16 + (hidx(kNb) + 4) * 4;
 };
 
 // Rows of one bin: bucket sort per row; rows whose buckets overflow go to a fallback list.
@@ -410,7 +426,10 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
                                                                   float *__restrict__ chat_val,
                                                                   int64_t *__restrict__ ccount,
                                                                   int32_t *__restrict__ fb_rows,
-                                                                  unsigned *__restrict__ fb_count, int64_t cap_skip) {
+                                                                  unsigned *__restrict__ fb_count, int64_t cap_skip,
+                                                                  const int64_t *__restrict__ crowptr,
+                                                                  int32_t *__restrict__ out_col,
+                                                                  float *__restrict__ out_val) {
     using S = BucketSmem<NW, EPT>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ int sc_all[GROUPS][NW + 1];
@@ -426,10 +445,12 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
         const int64_t s = rowoff[i];
         const int L = (int)(rowoff[i + 1] - s);
         if (L > S::kCap) continue;          // (limited list) rows above this kernel's capacity
+        const int64_t o = out_col ? crowptr[i] : s;
         const int U = bucket_sort_reduce<NW, GROUPS, EPT>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
-                                                          chat_col + s, chat_val + s, sc_all[g.gid]);
+                                                          (out_col ? out_col : chat_col) + o,
+                                                          (out_col ? out_val : chat_val) + o, sc_all[g.gid]);
         if (g.gtid == 0) {
-            if (U >= 0) ccount[i] = U;
+            if (U >= 0) { if (!out_col) ccount[i] = U; }
             else if (fb_rows) fb_rows[atomicAdd(fb_count, 1u)] = i;
             else ccount[i] = -1;   // limited list: k_merge_limited takes the row (merge-path fallback)
         }
@@ -438,468 +459,525 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
     (void)cap_skip;
 }
 
-// ------------------------------------------------------------ warp natural merge (WNM) ---
-// One warp per row of at most CAP slots.  Elements are packed as u64 = (col << 32) | val bits,
-// so ascending u64 order is ascending column order and a merge step is one 64-bit compare.
-// The row's runs (one per a_ik, padded with INT32_MAX sentinels that sort last) are detected
-// as strictly-descending steps, then merged pairwise level by level (merge path per lane);
-// bounds live in a per-warp array of <= 33 entries (rows with more runs go to the fallback).
-__device__ __forceinline__ unsigned long long lds64(unsigned a) {
-    unsigned long long v;
-    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ void sts64(unsigned a, unsigned long long v) {
-    asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
-}
-__device__ __forceinline__ int lds32(unsigned a) {
-    int v;
-    asm volatile("ld.shared.s32 %0, [%1];" : "=r"(v) : "r"(a));
-    return v;
-}
-__device__ __forceinline__ void sts32(unsigned a, int v) { asm volatile("st.shared.s32 [%0], %1;" ::"r"(a), "r"(v) : "memory"); }
-__device__ __forceinline__ unsigned long long pack_kv(int32_t k, float v) {
-    return ((unsigned long long)(uint32_t)k << 32) | (unsigned long long)__float_as_uint(v);
-}
-__device__ __forceinline__ int32_t pk_key(unsigned long long x) { return (int32_t)(x >> 32); }
-__device__ __forceinline__ float pk_val(unsigned long long x) { return __uint_as_float((unsigned)x); }
+// ------------------------------------------- register-staged counting sort (WCS) ---
+// One warp per row; the row is held in registers (VPT int4 + float4 vectors per lane, CAP =
+// 128*VPT slots) and shared memory holds only the scattered keys / values, the histogram and a
+// bitmap of bucket starts: ~12.3 B per slot, so CAP = 1024 is 12.4 KB and ~17 rows are in
+// flight per SM.
+//   1. vector loads of the padded row (runs are 16-byte aligned); min / max of its columns;
+//   2. nb = max(32, 2^ceil(log2 L)) buckets over the column span, bucket = (col - min) >> sh;
+//      histogram by shared-memory integer atomics;
+//   3. lane l owns nb/32 consecutive buckets (stored at b + b/32, so the 32 lanes' walks hit
+//      distinct banks): exclusive scan -> bucket starts; non-empty bucket starts are marked in
+//      the bitmap;
+//   4. scatter by atomic cursor (order inside a bucket is arbitrary);
+//   5. warp_merge_buckets: 32 slots at a time, cut at the last bucket start, so a chunk holds
+//      whole buckets; keys of a bucket are compared by shuffles (only chunks with a bucket of
+//      >= 2 keys loop), each distinct key's fp64 sum is written at its sorted output index.
+// Segments never cross buckets (equal keys share a bucket), so each chunk is independent.
+constexpr int kBitsPad = 3;   // bitmap words read past the end by bits64()
 
-constexpr int kWnmMaxRuns = 32;
+// bits [p, p + 64) of the bucket-start bitmap
+__device__ __forceinline__ uint64_t bits64(const uint32_t *bits, int p) {
+    const int w = p >> 5, sh = p & 31;
+    const uint32_t a = bits[w], b = bits[w + 1], c = bits[w + 2];
+    const uint32_t lo = __funnelshift_r(a, b, sh), hi = __funnelshift_r(b, c, sh);
+    return (uint64_t)lo | ((uint64_t)hi << 32);
+}
 
-template <int CAP, int WARPS>
-struct WnmSmem {
-    static constexpr int kWarpBytes = CAP * 16 + 2 * (kWnmMaxRuns + 2) * 4;
-    static constexpr int kBytes = kWarpBytes * WARPS;
-};
-
-template <int CAP, int WARPS>
-__global__ void __launch_bounds__(WARPS * 32) k_merge_wnm(const int32_t *__restrict__ rows, int64_t nrows,
-                                                         const int64_t *__restrict__ rowoff,
-                                                         const int64_t *__restrict__ rowwork,
-                                                         int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
-                                                         int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows,
-                                                         unsigned *__restrict__ fb_count) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int lane = lane_id(), w = warp_id();
-    const unsigned base = (unsigned)__cvta_generic_to_shared(smem_raw) + w * WnmSmem<CAP, WARPS>::kWarpBytes;
-    const unsigned bufA = base, bufB = base + CAP * 8;
-    const unsigned bndA = base + CAP * 16, bndB = bndA + (kWnmMaxRuns + 2) * 4;
-    for (int64_t r = (int64_t)blockIdx.x * WARPS + w; r < nrows; r += (int64_t)gridDim.x * WARPS) {
-        const int i = rows[r];
-        const int64_t s = rowoff[i];
-        const int Lc = (int)(rowoff[i + 1] - s);   // slots (multiple of 4)
-        const int Lv = (int)rowwork[i];            // products
-        // ---- load (16-byte vectors) and pack
-        for (int v = lane; v < (Lc >> 2); v += 32) {
-            const int4 c4 = *reinterpret_cast<const int4 *>(chat_col + s + 4 * v);
-            const float4 x4 = *reinterpret_cast<const float4 *>(chat_val + s + 4 * v);
-            sts64(bufA + 32 * v + 0, pack_kv(c4.x, x4.x));
-            sts64(bufA + 32 * v + 8, pack_kv(c4.y, x4.y));
-            sts64(bufA + 32 * v + 16, pack_kv(c4.z, x4.z));
-            sts64(bufA + 32 * v + 24, pack_kv(c4.w, x4.w));
-        }
-        __syncwarp();
-        // ---- run heads (strict descent), lane owns slots [lane*E, lane*E + E)
-        const int E = ((Lc + 31) >> 5) | 1;   // odd lane stride: conflict-free smem slices
-        const int p0 = min(Lc, lane * E), p1 = min(Lc, p0 + E);
-        int nh = 0;
-        {
-            unsigned long long prev = p0 > 0 ? lds64(bufA + 8 * (p0 - 1)) : 0ull;
-            for (int p = p0; p < p1; ++p) {
-                const unsigned long long x = lds64(bufA + 8 * p);
-                nh += (p == 0 || pk_key(x) < pk_key(prev));
-                prev = x;
+// Ascending bitonic sort of (k, v)[0, n) in shared memory by one warp; indices >= n act as +inf
+// (every comparator puts the minimum at the lower index, so virtual padding never moves).
+__device__ __noinline__ void warp_bitonic_smem(int32_t *k, float *v, int n) {
+    int N = 1;
+    while (N < n) N <<= 1;
+    const int lane = lane_id();
+    auto cmpswap = [&](int i, int j) {
+        if (j < n) {
+            const int32_t ki = k[i], kj = k[j];
+            if (kj < ki) {
+                const float vi = v[i];
+                k[i] = kj; k[j] = ki;
+                v[i] = v[j]; v[j] = vi;
             }
         }
-        const int inc = warp_incl_sum(nh);
-        const int R = __shfl_sync(kFull, inc, 31);
-        if (R > kWnmMaxRuns) {
-            if (lane == 0) fb_rows[atomicAdd(fb_count, 1u)] = i;
+    };
+    for (int size = 2; size <= N; size <<= 1) {
+        const int half = size >> 1;
+        for (int t = lane; t < (N >> 1); t += 32) {     // flip: i <-> mirror in its block
+            const int blk = (t / half) * size, off = t % half;
+            cmpswap(blk + off, blk + size - 1 - off);
+        }
+        __syncwarp();
+        for (int d = half >> 1; d >= 1; d >>= 1) {      // half-cleaners
+            for (int t = lane; t < (N >> 1); t += 32) {
+                const int blk = (t / d) * (2 * d), off = t % d;
+                cmpswap(blk + off, blk + off + d);
+            }
             __syncwarp();
+        }
+    }
+}
+
+// Merge the slots [lo, hi) of a row (or of a tile of rows) whose buckets are contiguous and
+// marked in `bits` (lo is a bucket start): every distinct key of a bucket is emitted once, in
+// ascending key order, with the fp64 sum of its values, through emit(o, key, value) with
+// o = 0, 1, ... (warp-uniform call sites; o is relative to the range).  Returns the count.
+template <typename Emit>
+__device__ __forceinline__ int warp_merge_buckets(int32_t *sk, float *sv, const uint32_t *bits, int lo, int hi,
+                                                  Emit emit) {
+    const int lane = lane_id();
+    int ob = 0;
+    int p0 = lo;
+    while (p0 < hi) {
+        uint64_t m = bits64(bits, p0) | 1ull;
+        const int rem = hi - p0;
+        if (rem < 64) m = (m & ((1ull << rem) - 1)) | (1ull << rem);   // hi is a boundary
+        const uint64_t m33 = m & 0x1FFFFFFFEull;                        // boundaries in [1, 32]
+        if (m33 == 0) {
+            // one bucket of more than 32 keys: find its end, sort it (unless single-valued)
+            int e = p0 + 64;
+            while (e < hi) {
+                const uint64_t mm = bits64(bits, e);
+                if (mm) { e += __ffsll((long long)mm) - 1; break; }
+                e += 64;
+            }
+            e = min(e, hi);
+            int32_t kmin = kKeyPad, kmax = 0;
+            for (int p = p0 + lane; p < e; p += 32) { kmin = min(kmin, sk[p]); kmax = max(kmax, sk[p]); }
+            kmin = __reduce_min_sync(kFull, kmin);
+            kmax = __reduce_max_sync(kFull, kmax);
+            if (kmin != kmax) warp_bitonic_smem(sk + p0, sv + p0, e - p0);
+            __syncwarp();
+            for (int q0 = p0; q0 < e; q0 += 32) {
+                const int p = q0 + lane;
+                const bool in = p < e;
+                const int32_t k = in ? sk[p] : kKeyPad;
+                int32_t prev = __shfl_up_sync(kFull, k, 1);
+                if (lane == 0) prev = q0 > p0 ? sk[q0 - 1] : ~k;
+                const bool head = in && k != prev;
+                double acc = 0.0;
+                if (head) {
+                    acc = (double)sv[p];
+                    for (int q = p + 1; q < e && sk[q] == k; ++q) acc += (double)sv[q];
+                }
+                const unsigned hm = __ballot_sync(kFull, head);
+                __syncwarp();
+                if (head) emit(ob + __popc(hm & lanemask_lt()), k, acc);
+                ob += __popc(hm);
+            }
+            __syncwarp();
+            p0 = e;
             continue;
         }
-        {
-            int pos = inc - nh;
-            unsigned long long prev = p0 > 0 ? lds64(bufA + 8 * (p0 - 1)) : 0ull;
-            for (int p = p0; p < p1; ++p) {
-                const unsigned long long x = lds64(bufA + 8 * p);
-                if (p == 0 || pk_key(x) < pk_key(prev)) sts32(bndA + 4 * pos++, p);
-                prev = x;
+        const int n = 63 - __clzll((long long)m33);   // lanes [0, n) hold whole buckets
+        const bool ok = lane < n;
+        const int p = p0 + lane;
+        const int32_t k = ok ? sk[p] : kKeyPad;
+        const float v = ok ? sv[p] : 0.f;
+        const uint32_t mlo = (uint32_t)m;
+        const int bs = 31 - __clz(mlo & (lane == 31 ? kFull : ((2u << lane) - 1)));   // bucket start lane
+        const uint64_t above = m & ~((2ull << lane) - 1);
+        const int be = __ffsll((long long)above) - 1;                                 // bucket end lane
+        const int c = ok ? be - bs : 0;
+        bool rep = ok;
+        double acc = (double)v;
+        int nless = 0;
+        const int maxc = __reduce_max_sync(kFull, c);
+        if (maxc > 1) {
+            const int myq = lane - bs;
+            acc = 0.0;
+            for (int q = 0; q < maxc; ++q) {
+                const int src = min(bs + q, 31);
+                const int32_t kq = __shfl_sync(kFull, k, src);
+                const float vq = __shfl_sync(kFull, v, src);
+                if (q < c && kq == k) {
+                    acc += (double)vq;
+                    if (q < myq) rep = false;
+                }
             }
-            if (lane == 0) sts32(bndA + 4 * R, Lc);
+            for (int q = 0; q < maxc; ++q) {
+                const int src = min(bs + q, 31);
+                const int32_t kq = __shfl_sync(kFull, k, src);
+                const bool rq = __shfl_sync(kFull, (int)rep, src) != 0;
+                nless += (q < c && rq && kq < k);
+            }
+        }
+        const unsigned rm = __ballot_sync(kFull, rep);
+        __syncwarp();
+        if (rep) emit(ob + __popc(rm & ((1u << bs) - 1)) + nless, k, acc);
+        ob += __popc(rm);
+        p0 += n;
+    }
+    __syncwarp();
+    return ob;
+}
+
+template <int VPT>
+struct WcsSmem {
+    static constexpr int kCap = 32 * VPT * 4;      // power of two
+    static constexpr int kHist = kCap + kCap / 32;
+    static constexpr int kBits = kCap / 32 + kBitsPad;
+    static constexpr int kBytes = kCap * 8 + kHist * 4 + kBits * 4;
+};
+
+__device__ __forceinline__ int wcs_hidx(int b) { return b + (b >> 5); }
+
+template <int GROUPS, int VPT>
+__global__ void __launch_bounds__(32 * GROUPS) k_merge_wcs(const int32_t *__restrict__ rows, int64_t nrows,
+                                                          const int64_t *__restrict__ rowoff,
+                                                          const int64_t *__restrict__ rowwork,
+                                                          int32_t *__restrict__ chat_col,
+                                                          float *__restrict__ chat_val,
+                                                          int64_t *__restrict__ ccount,
+                                                          const int64_t *__restrict__ crowptr,
+                                                          int32_t *__restrict__ out_col_all,
+                                                          float *__restrict__ out_val_all) {
+    using S = WcsSmem<VPT>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int gid = threadIdx.x >> 5;
+    unsigned char *slice = smem_raw + (size_t)gid * S::kBytes;
+    int32_t *sk = (int32_t *)slice;
+    float *sv = (float *)(slice + S::kCap * 4);
+    int *hist = (int *)(slice + S::kCap * 8);
+    uint32_t *bits = (uint32_t *)(slice + S::kCap * 8 + S::kHist * 4);
+    const int lane = lane_id();
+    for (int64_t r = (int64_t)blockIdx.x * GROUPS + gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
+        const int i = rows[r];
+        const int64_t s = rowoff[i];
+        const int nv = (int)((rowoff[i + 1] - s) >> 2);
+        const int L = (int)rowwork[i];
+        int4 kc[VPT];
+        float4 kv[VPT];
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const int v = lane + j * 32;
+            if (v < nv) {
+                kc[j] = __ldcs(reinterpret_cast<const int4 *>(chat_col + s) + v);
+                kv[j] = __ldcs(reinterpret_cast<const float4 *>(chat_val + s) + v);
+            } else {
+                kc[j] = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
+            }
+        }
+        int32_t mn = kKeyPad, mx = 0;
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const int32_t c4[4] = {kc[j].x, kc[j].y, kc[j].z, kc[j].w};
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                if (c4[u] != kKeyPad) { mn = min(mn, c4[u]); mx = max(mx, c4[u]); }
+        }
+        mn = __reduce_min_sync(kFull, mn);
+        mx = __reduce_max_sync(kFull, mx);
+        const int lognb = max(nextpow2_log(L), 5);
+        const int nb = 1 << lognb;
+        const uint32_t span = (uint32_t)(mx - mn);
+        const int bits_span = span ? 32 - __clz(span) : 0;
+        const int sh = max(0, bits_span - lognb);
+        const int nbh = nb + (nb >> 5);
+        for (int b = lane; b < nbh; b += 32) hist[b] = 0;
+        for (int w = lane; w < min(S::kBits, (L >> 5) + kBitsPad); w += 32) bits[w] = 0;
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const int32_t c4[4] = {kc[j].x, kc[j].y, kc[j].z, kc[j].w};
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                if (c4[u] != kKeyPad) atomicAdd(&hist[wcs_hidx((c4[u] - mn) >> sh)], 1);
         }
         __syncwarp();
-        unsigned src = bufA, dst = bufB, bs = bndA, bd = bndB;
-        int nr = R;
-        while (nr > 1) {
-            const int npairs = (nr + 1) >> 1;
-            if (p0 < p1) {
-                int lo = 0, hi = npairs;       // pair q: last q with start(2q) <= p0
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (lds32(bs + 8 * mid) <= p0) lo = mid; else hi = mid;
-                }
-                int q = lo, o = p0;
-                while (o < p1) {
-                    const int a0 = lds32(bs + 8 * q);
-                    const int a1 = lds32(bs + 4 * min(2 * q + 1, nr));
-                    const int b1 = lds32(bs + 4 * min(2 * q + 2, nr));
-                    const int na = a1 - a0, nb = b1 - a1;
-                    const int d = o - a0;
-                    int ilo = max(0, d - nb), ihi = min(d, na);
-                    while (ilo < ihi) {         // merge path: first i with A[i] > B[d-i-1]
-                        const int mi = (ilo + ihi) >> 1;
-                        if (lds64(src + 8 * (a0 + mi)) <= lds64(src + 8 * (a1 + d - mi - 1))) ilo = mi + 1;
-                        else ihi = mi;
-                    }
-                    int ia = a0 + ilo, jb = a1 + d - ilo;
-                    unsigned long long xa = ia < a1 ? lds64(src + 8 * ia) : ~0ull;
-                    unsigned long long xb = jb < b1 ? lds64(src + 8 * jb) : ~0ull;
-                    const int oend = min(p1, b1);
-                    for (; o < oend; ++o) {
-                        const bool tA = xa <= xb;
-                        sts64(dst + 8 * o, tA ? xa : xb);
-                        if (tA) {
-                            ++ia;
-                            xa = ia < a1 ? lds64(src + 8 * ia) : ~0ull;
-                        } else {
-                            ++jb;
-                            xb = jb < b1 ? lds64(src + 8 * jb) : ~0ull;
-                        }
-                    }
-                    ++q;
-                }
-            }
-            __syncwarp();
-            for (int q = lane; q <= npairs; q += 32)
-                sts32(bd + 4 * q, q < npairs ? lds32(bs + 8 * q) : Lc);
-            __syncwarp();
-            { const unsigned t = src; src = dst; dst = t; }
-            { const unsigned t = bs; bs = bd; bd = t; }
-            nr = npairs;
-        }
-        // ---- segmented reduction over [0, Lv) (sentinels sorted last), compacted into dst
-        const int Ev = ((Lv + 31) >> 5) | 1;
-        const int v0 = min(Lv, lane * Ev), v1 = min(Lv, v0 + Ev);
-        int nu = 0;
+        const int bpt = nb >> 5;
+        const int b0 = lane * bpt;
+        int cnt = 0;
+        for (int q = 0; q < bpt; ++q) cnt += hist[wcs_hidx(b0 + q)];
+        const int inc = warp_incl_sum(cnt);
         {
-            int32_t pk = v0 > 0 ? pk_key(lds64(src + 8 * (v0 - 1))) : -1;
-            for (int p = v0; p < v1; ++p) {
-                const int32_t k = pk_key(lds64(src + 8 * p));
-                nu += (p == 0 || k != pk);
-                pk = k;
-            }
-        }
-        const int uinc = warp_incl_sum(nu);
-        const int U = __shfl_sync(kFull, uinc, 31);
-        {
-            int o = uinc - nu;
-            for (int p = v0; p < v1; ++p) {
-                const unsigned long long x = lds64(src + 8 * p);
-                if (p == 0 || pk_key(x) != pk_key(lds64(src + 8 * (p - 1)))) {
-                    double acc = (double)pk_val(x);
-                    int q = p + 1;
-                    for (; q < Lv; ++q) {
-                        const unsigned long long y = lds64(src + 8 * q);
-                        if (pk_key(y) != pk_key(x)) break;
-                        acc += (double)pk_val(y);
-                    }
-                    sts64(dst + 8 * o++, pack_kv(pk_key(x), (float)acc));
-                }
+            int run = inc - cnt;
+            for (int q = 0; q < bpt; ++q) {
+                const int h = wcs_hidx(b0 + q);
+                const int c = hist[h];
+                hist[h] = run;
+                if (c) atomicOr(&bits[run >> 5], 1u << (run & 31));
+                run += c;
             }
         }
         __syncwarp();
-        for (int t = lane; t < U; t += 32) {
-            const unsigned long long x = lds64(dst + 8 * t);
-            chat_col[s + t] = pk_key(x);
-            chat_val[s + t] = pk_val(x);
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const int32_t c4[4] = {kc[j].x, kc[j].y, kc[j].z, kc[j].w};
+            const float v4[4] = {kv[j].x, kv[j].y, kv[j].z, kv[j].w};
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                if (c4[u] != kKeyPad) {
+                    const int p = atomicAdd(&hist[wcs_hidx((c4[u] - mn) >> sh)], 1);
+                    sk[p] = c4[u];
+                    sv[p] = v4[u];
+                }
         }
-        if (lane == 0) ccount[i] = U;
+        __syncwarp();
+        const int64_t o0 = out_col_all ? crowptr[i] : s;
+        int32_t *__restrict__ out_col = (out_col_all ? out_col_all : chat_col) + o0;
+        float *__restrict__ out_val = (out_col_all ? out_val_all : chat_val) + o0;
+        const int U = warp_merge_buckets(sk, sv, bits, 0, L, [&](int o, int32_t k, double acc) {
+            out_col[o] = k;
+            out_val[o] = (float)acc;
+        });
+        if (lane == 0 && !out_col_all) ccount[i] = U;
         __syncwarp();
     }
 }
 
-// --------------------------------------------------------- batched multi-row bucket sort ---
-// Rows of a bin are short (C2: 100-1000 products, 4-18 runs), so per-row fixed costs dominate a
-// one-row-per-group sort.  A CTA claims kBatchRows rows of its bin list and packs them, in list
-// order, into sub-batches of at most CAPN bucket slots; each sub-batch is sorted as ONE problem
-// whose buckets are row-major: row r owns buckets [bbase[r], bbase[r] + nb[r]), nb[r] =
-// 2^ceil(log2 L_r), covering its column span.  Ordering buckets by row makes the sorted array
-// row-major, so the segmented reduction and the copy-out of every row follow directly.
-//   load   : thread t owns CAPN/T consecutive slots (int4 loads; runs are 16-byte aligned and
-//            bucket lengths multiples of 4, so a 4-slot group never straddles two rows)
-//   min/max: per-row span by shared-memory atomicMin/Max (one per row segment of a thread)
-//   sort   : histogram -> scan -> atomic-rank scatter -> in-bucket ranking by counting
-//   reduce : fp64 over equal (row, col) runs, compacted in order; row r's output starts at uoff[r]
-//   store  : one warp per row copies its merged entries to the head of its Ĉ bucket
-constexpr int kBatchRows = 64;
+// -------------------------------------------- warp merge-path natural merge sort (WMP) ---
+// No shared-memory atomics (see k_count_rows).  A row's bucket is a concatenation of runs (one
+// per stored a_ik, ascending, sentinel-padded to 4 slots), so it is sorted by merging them.
+// A group of NW warps (T = 32*NW threads) per row:
+//   1. 16-byte vector loads; (col, val) packed into one u64 (col in the high word) in smem;
+//      runs start at vector boundaries where the column descends (or the previous run ended
+//      in sentinels), found per vector and compacted in order (ballot / group scan);
+//   2. levels of pairwise merges, ping-ponging between two smem buffers: thread t produces the
+//      t-th slice of each level's output, locating its start in the pair by a merge-path search
+//      and merging with a branch-free loop (one predicated LDS per output; keys compared as
+//      32-bit integers, ties taken from the left run);
+//   3. reduction: each warp walks its share of the sorted products 32 at a time (shares start
+//      at segment heads): heads by neighbour compare, fp64 sums of duplicates, ballot-compacted
+//      output, straight to the output (NW = 1) or staged per warp in smem and copied out at the
+//      warp's scanned offset (NW > 1); output = C at crowptr[i] or in place in Ĉ.
+__device__ __forceinline__ uint64_t pack_kv(int32_t k, float v) {
+    return ((uint64_t)(uint32_t)k << 32) | (uint64_t)__float_as_uint(v);
+}
+__device__ __forceinline__ int32_t kv_key(uint64_t x) { return (int32_t)(x >> 32); }
+__device__ __forceinline__ float kv_val(uint64_t x) { return __uint_as_float((uint32_t)x); }
+constexpr uint64_t kKvMax = 0x7fffffffffffffffull;   // key INT32_MAX: after every product
 
-template <int THREADS, int CAPN>
-struct BatchSmem {
-    static constexpr int kNbMax = 2 * CAPN;     // sum of per-row bucket counts <= 2 * slots
-    static constexpr int kBytes = CAPN * 16 + kNbMax * 4;
+template <int CAP>
+struct WmpSmem {
+    static constexpr int kRuns = CAP / 4 + 2;
+    static constexpr int kBytes = CAP * 16 + 2 * kRuns * 4;
 };
 
-template <int THREADS, int CAPN>
-__global__ void __launch_bounds__(THREADS) k_merge_batch(const int32_t *__restrict__ rows, int64_t nrows,
-                                                         const int64_t *__restrict__ rowoff,
-                                                         const int64_t *__restrict__ rowwork,
-                                                         int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
-                                                         int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows,
-                                                         unsigned *__restrict__ fb_count) {
-    constexpr int NW = THREADS / 32;
-    constexpr int EPT = CAPN / THREADS;                    // slots per thread (multiple of 4)
-    static_assert(EPT % 4 == 0, "EPT must be a multiple of 4");
-    using S = BatchSmem<THREADS, CAPN>;
+template <int NW, int GROUPS, int CAP>
+__global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_wmp(const int32_t *__restrict__ rows, int64_t nrows,
+                                                               const int64_t *__restrict__ rowoff,
+                                                               const int64_t *__restrict__ rowwork,
+                                                               int32_t *__restrict__ chat_col,
+                                                               float *__restrict__ chat_val,
+                                                               int64_t *__restrict__ ccount,
+                                                               const int64_t *__restrict__ crowptr,
+                                                               int32_t *__restrict__ out_col_all,
+                                                               float *__restrict__ out_val_all) {
+    using S = WmpSmem<CAP>;
+    constexpr int T = NW * 32;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    int32_t *dk = (int32_t *)smem_raw;
-    float *dv = (float *)(smem_raw + CAPN * 4);
-    int32_t *dk2 = (int32_t *)(smem_raw + CAPN * 8);
-    float *dv2 = (float *)(smem_raw + CAPN * 12);
-    int *hist = (int *)(smem_raw + CAPN * 16);
-    __shared__ int r_row[kBatchRows], r_cap[kBatchRows + 1], r_len[kBatchRows + 1];
-    __shared__ int r_min[kBatchRows], r_max[kBatchRows], r_sh[kBatchRows], r_bb[kBatchRows + 1];
-    __shared__ int r_uoff[kBatchRows + 1];
-    __shared__ int64_t r_src[kBatchRows];
-    __shared__ int sc[NW + 1];
-    __shared__ int s_nsub, s_overflow;
-    const Group<NW, 1> g;
-    const int lane = lane_id(), w = warp_id();
-    for (int64_t c0 = (int64_t)blockIdx.x * kBatchRows; c0 < nrows; c0 += (int64_t)gridDim.x * kBatchRows) {
-        const int nchunk = (int)min((int64_t)kBatchRows, nrows - c0);
-        int done = 0;
-        while (done < nchunk) {
-            // ---- form the next sub-batch: rows [done, done + nsub) of the chunk, caps <= CAPN
-            if (threadIdx.x < 32) {
-                int cap = 0, len = 0, row = 0;
-                int64_t src = 0;
-                int nsub = 0, acc = 0;
-                for (int base = done; base < nchunk; base += 32) {
-                    const int q = base + lane;
-                    if (q < nchunk) {
-                        row = rows[c0 + q];
-                        src = rowoff[row];
-                        cap = (int)(rowoff[row + 1] - src);
-                        len = (int)rowwork[row];
-                    } else {
-                        cap = CAPN + 1;
-                    }
-                    const int inc = warp_incl_sum(cap);
-                    const unsigned fit = __ballot_sync(kFull, acc + inc <= CAPN);
-                    const int take = __popc(fit);            // prefix of lanes that fit
-                    if (lane < take) {
-                        const int r = base - done + lane;
-                        r_row[r] = row;
-                        r_src[r] = src;
-                        r_cap[r] = acc + inc - cap;            // exclusive slot offset
-                        r_len[r] = len;
-                    }
-                    acc += __shfl_sync(kFull, inc, max(take - 1, 0)) * (take > 0);
-                    nsub += take;
-                    if (take < 32) break;
+    __shared__ int sc_all[GROUPS][NW + 1];
+    __shared__ int wcnt_all[GROUPS][NW + 1];
+    const Group<NW, GROUPS> g;
+    int *sc = sc_all[g.gid];
+    int *wcnt = wcnt_all[g.gid];
+    const int lane = lane_id(), wg = g.gtid >> 5;
+    unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
+    uint64_t *bufA = (uint64_t *)slice;
+    uint64_t *bufB = bufA + CAP;
+    int *runsA = (int *)(bufB + CAP);
+    int *runsB = runsA + S::kRuns;
+    const unsigned lt = lanemask_lt();
+    for (int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
+        const int i = rows[r];
+        const int64_t s = rowoff[i];
+        const int Lp = (int)(rowoff[i + 1] - s);
+        const int Lv = (int)rowwork[i];
+        const int nv = Lp >> 2;
+        const int4 *__restrict__ c4p = reinterpret_cast<const int4 *>(chat_col + s);
+        const float4 *__restrict__ v4p = reinterpret_cast<const float4 *>(chat_val + s);
+        // 1. load + pack; run starts
+        int R = 0;
+        if constexpr (NW == 1) {
+            int32_t carry = kKeyPad;
+            for (int v0 = 0; v0 < nv; v0 += 64) {
+                int4 c[2];
+                float4 f[2];
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    const int v = v0 + 32 * u + lane;
+                    if (v < nv) { c[u] = __ldcs(c4p + v); f[u] = __ldcs(v4p + v); }
+                    else c[u] = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
                 }
-                if (lane == 0) {
-                    r_cap[nsub] = acc;
-                    s_nsub = nsub;
-                    s_overflow = 0;
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    const int v = v0 + 32 * u + lane;
+                    int32_t prev = __shfl_up_sync(kFull, c[u].w, 1);
+                    if (lane == 0) prev = carry;
+                    carry = __shfl_sync(kFull, c[u].w, 31);
+                    const bool start = v < nv && (v == 0 || c[u].x < prev);
+                    const unsigned m = __ballot_sync(kFull, start);
+                    if (start) runsA[R + __popc(m & lt)] = 4 * v;
+                    R += __popc(m);
+                    if (v < nv) {
+                        ulonglong2 *d = reinterpret_cast<ulonglong2 *>(bufA + 4 * v);
+                        d[0] = make_ulonglong2(pack_kv(c[u].x, f[u].x), pack_kv(c[u].y, f[u].y));
+                        d[1] = make_ulonglong2(pack_kv(c[u].z, f[u].z), pack_kv(c[u].w, f[u].w));
+                    }
                 }
             }
-            __syncthreads();
-            const int nsub = s_nsub;
-            const int N = r_cap[nsub];
-            // per-row prefix of product counts (sorted row starts) and init of row spans
-            if (threadIdx.x < 32) {
-                int run = 0;
-                for (int base = 0; base < nsub; base += 32) {
-                    const int q = base + lane;
-                    const int l = q < nsub ? r_len[q] : 0;
-                    const int inc = warp_incl_sum(l);
-                    if (q < nsub) {
-                        r_len[q] = run + inc - l;   // now: sorted start of row q
-                        r_min[q] = kKeyPad;
-                        r_max[q] = 0;
-                    }
-                    run += __shfl_sync(kFull, inc, 31);
+            if (lane == 0) runsA[R] = Lp;
+            __syncwarp();
+        } else {
+            for (int v0 = 0; v0 < nv; v0 += 2 * T) {
+                int4 c[2];
+                float4 f[2];
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    const int v = v0 + T * u + g.gtid;
+                    if (v < nv) { c[u] = __ldcs(c4p + v); f[u] = __ldcs(v4p + v); }
                 }
-                if (lane == 0) r_len[nsub] = run;
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    const int v = v0 + T * u + g.gtid;
+                    if (v < nv) {
+                        ulonglong2 *d = reinterpret_cast<ulonglong2 *>(bufA + 4 * v);
+                        d[0] = make_ulonglong2(pack_kv(c[u].x, f[u].x), pack_kv(c[u].y, f[u].y));
+                        d[1] = make_ulonglong2(pack_kv(c[u].z, f[u].z), pack_kv(c[u].w, f[u].w));
+                    }
+                }
             }
-            __syncthreads();
-            // ---- load: thread owns slots [t*EPT, t*EPT + EPT)
-            int32_t key[EPT];
-            float val[EPT];
-            int rid[EPT / 4];
-            const int p0 = threadIdx.x * EPT;
-            {
-                int lo = 0, hi = nsub;     // row of slot p0: last r with r_cap[r] <= p0
+            g.sync();
+            // run starts over contiguous vector ranges per thread, compacted by a group scan
+            const int vpt = (nv + T - 1) / T;
+            const int va = min(nv, g.gtid * vpt), vb = min(nv, va + vpt);
+            int ns = 0;
+            for (int v = va; v < vb; ++v) ns += (v == 0 || kv_key(bufA[4 * v]) < kv_key(bufA[4 * v - 1]));
+            int tot;
+            int pos = g.excl_sum(ns, sc, &tot);
+            for (int v = va; v < vb; ++v)
+                if (v == 0 || kv_key(bufA[4 * v]) < kv_key(bufA[4 * v - 1])) runsA[pos++] = 4 * v;
+            R = tot;
+            if (g.gtid == 0) runsA[R] = Lp;
+            g.sync();
+        }
+        // 2. merge levels
+        uint64_t *src = bufA, *dst = bufB;
+        int *rs = runsA, *rd = runsB;
+        const int E = (Lp + T - 1) / T;
+        while (R > 1) {
+            const int npairs = (R + 1) >> 1;
+            int o = min(Lp, g.gtid * E);
+            const int oend = min(Lp, o + E);
+            if (o < oend) {
+                int lo = 0, hi = npairs;      // pair holding output o: last q with rs[2q] <= o
                 while (hi - lo > 1) {
                     const int mid = (lo + hi) >> 1;
-                    if (r_cap[mid] <= p0) lo = mid; else hi = mid;
+                    if (rs[2 * mid] <= o) lo = mid; else hi = mid;
                 }
-                int r = lo;
-                int32_t mn = kKeyPad, mx = 0;
-#pragma unroll
-                for (int v = 0; v < EPT / 4; ++v) {
-                    const int p = p0 + 4 * v;
-                    if (p < N) {
-                        while (r_cap[r + 1] <= p) {
-                            if (mn != kKeyPad) { atomicMin(&r_min[r], mn); atomicMax(&r_max[r], mx); }
-                            mn = kKeyPad;
-                            mx = 0;
-                            ++r;
-                        }
-                        const int64_t src = r_src[r] + (p - r_cap[r]);
-                        const int4 c4 = *reinterpret_cast<const int4 *>(chat_col + src);
-                        const float4 v4 = *reinterpret_cast<const float4 *>(chat_val + src);
-                        key[4 * v + 0] = c4.x; key[4 * v + 1] = c4.y; key[4 * v + 2] = c4.z; key[4 * v + 3] = c4.w;
-                        val[4 * v + 0] = v4.x; val[4 * v + 1] = v4.y; val[4 * v + 2] = v4.z; val[4 * v + 3] = v4.w;
-                        rid[v] = r;
-#pragma unroll
-                        for (int u = 0; u < 4; ++u)
-                            if (key[4 * v + u] != kKeyPad) { mn = min(mn, key[4 * v + u]); mx = max(mx, key[4 * v + u]); }
-                    } else {
-                        key[4 * v + 0] = key[4 * v + 1] = key[4 * v + 2] = key[4 * v + 3] = kKeyPad;
-                        rid[v] = -1;
+                int q = lo;
+                while (o < oend) {
+                    const int a0 = rs[2 * q], a1 = rs[min(2 * q + 1, R)], b1 = rs[min(2 * q + 2, R)];
+                    const int d = o - a0;
+                    int ilo = max(0, d - (b1 - a1)), ihi = min(d, a1 - a0);
+                    while (ilo < ihi) {        // merge path: first i with A[i] > B[d - i - 1] (keys)
+                        const int mi = (ilo + ihi) >> 1;
+                        if (kv_key(src[a0 + mi]) <= kv_key(src[a1 + d - mi - 1])) ilo = mi + 1; else ihi = mi;
                     }
-                }
-                if (mn != kKeyPad && r < nsub) { atomicMin(&r_min[r], mn); atomicMax(&r_max[r], mx); }
-            }
-            __syncthreads();
-            // ---- per-row bucket ranges
-            if (threadIdx.x < 32) {
-                int run = 0;
-                for (int base = 0; base < nsub; base += 32) {
-                    const int q = base + lane;
-                    int nb = 0;
-                    if (q < nsub) {
-                        const int lq = r_len[q + 1] - r_len[q];
-                        const int lognb = nextpow2_log(max(lq, 1));
-                        nb = 1 << lognb;
-                        const uint32_t span = (uint32_t)(r_max[q] - r_min[q]);
-                        const int bits = span ? 32 - __clz(span) : 0;
-                        r_sh[q] = max(0, bits - lognb);
+                    int ia = a0 + ilo, jb = a1 + d - ilo;
+                    uint64_t xa = ia < a1 ? src[ia] : kKvMax;
+                    uint64_t xb = jb < b1 ? src[jb] : kKvMax;
+                    const int pend = min(oend, b1);
+                    for (; o < pend; ++o) {
+                        const bool tA = kv_key(xa) <= kv_key(xb);
+                        dst[o] = tA ? xa : xb;
+                        const int nxt = tA ? ia + 1 : jb + 1;
+                        const uint64_t y = nxt < (tA ? a1 : b1) ? src[nxt] : kKvMax;
+                        ia = tA ? nxt : ia;
+                        jb = tA ? jb : nxt;
+                        xa = tA ? y : xa;
+                        xb = tA ? xb : y;
                     }
-                    const int inc = warp_incl_sum(nb);
-                    if (q < nsub) r_bb[q] = run + inc - nb;
-                    run += __shfl_sync(kFull, inc, 31);
-                }
-                if (lane == 0) r_bb[nsub] = run;
-            }
-            __syncthreads();
-            const int NB = r_bb[nsub];
-            for (int b = threadIdx.x; b < NB; b += THREADS) hist[b] = 0;
-            __syncthreads();
-            int bkt[EPT];
-#pragma unroll
-            for (int e = 0; e < EPT; ++e) {
-                bkt[e] = -1;
-                if (key[e] != kKeyPad) {
-                    const int r = rid[e / 4];
-                    bkt[e] = r_bb[r] + ((key[e] - r_min[r]) >> r_sh[r]);
-                    atomicAdd(&hist[bkt[e]], 1);
+                    ++q;
                 }
             }
-            __syncthreads();
-            // scan of the histogram (thread owns a contiguous bucket range) + overflow check
-            const int bpt = (NB + THREADS - 1) / THREADS;
-            const int b0 = min(NB, (int)threadIdx.x * bpt), b1 = min(NB, b0 + bpt);
-            int cnt = 0, mxc = 0;
-            for (int b = b0; b < b1; ++b) {
-                const int c = hist[b];
-                cnt += c;
-                mxc = max(mxc, c);
+            for (int q = g.gtid; q <= npairs; q += T) rd[q] = q < npairs ? rs[2 * q] : Lp;
+            g.sync();
+            { uint64_t *t = src; src = dst; dst = t; }
+            { int *t = rs; rs = rd; rd = t; }
+            R = npairs;
+        }
+        // 3. reduction of the sorted products (sentinels sorted last) into C
+        int wlo = 0, whi = Lv;
+        if constexpr (NW > 1) {
+            const int per = (Lv + NW - 1) / NW;
+            wlo = min(Lv, wg * per);
+            whi = min(Lv, wlo + per);
+            // shares start at segment heads
+            if (lane == 0) {
+                while (wlo > 0 && wlo < Lv && kv_key(src[wlo]) == kv_key(src[wlo - 1])) ++wlo;
+                while (whi < Lv && kv_key(src[whi]) == kv_key(src[whi - 1])) ++whi;
             }
-            if (mxc > kBucketMax) s_overflow = 1;
-            int tot;
-            int ex = g.excl_sum(cnt, sc, &tot);   // (contains barriers: s_overflow visible after)
-            if (s_overflow) {
-                // a bucket too full for the in-bucket ranking: these rows take the merge-path fallback
-                for (int q = threadIdx.x; q < nsub; q += THREADS) fb_rows[atomicAdd(fb_count, 1u)] = r_row[q];
-                done += nsub;
-                __syncthreads();
+            wlo = __shfl_sync(kFull, wlo, 0);
+            whi = __shfl_sync(kFull, whi, 0);
+        }
+        // output: C at crowptr[i], or in place at the head of the row's Ĉ bucket (the whole row
+        // is in shared memory by now)
+        const int64_t obase = out_col_all ? crowptr[i] : s;
+        int32_t *__restrict__ out_col = out_col_all ? out_col_all : chat_col;
+        float *__restrict__ out_val = out_col_all ? out_val_all : chat_val;
+        int ob = 0;
+        uint64_t *stage = dst + wlo;   // NW > 1: the free buffer, at the warp's share
+        for (int p0 = wlo; p0 < whi; p0 += 32) {
+            const int p = p0 + lane;
+            const bool in = p < whi;
+            const uint64_t x = in ? src[p] : kKvMax;
+            const int32_t k = kv_key(x);
+            int32_t prev = __shfl_up_sync(kFull, k, 1);
+            if (lane == 0) prev = p0 > wlo ? kv_key(src[p0 - 1]) : ~k;
+            int32_t next = __shfl_down_sync(kFull, k, 1);
+            if (lane == 31) next = p + 1 < whi ? kv_key(src[p + 1]) : kKeyPad;
+            const bool head = in && k != prev;
+            const unsigned hm = __ballot_sync(kFull, head);
+            const bool dup = in && next == k;
+            if (hm == kFull && !__any_sync(kFull, dup)) {         // common case: 32 distinct keys
+                if constexpr (NW == 1) {
+                    out_col[obase + ob + lane] = k;
+                    out_val[obase + ob + lane] = kv_val(x);
+                } else {
+                    stage[ob + lane] = x;
+                }
+                ob += 32;
                 continue;
             }
-            for (int b = b0; b < b1; ++b) {
-                const int c = hist[b];
-                hist[b] = ex;
-                ex += c;
-            }
-            __syncthreads();
-            int pos[EPT];
-#pragma unroll
-            for (int e = 0; e < EPT; ++e) {
-                pos[e] = -1;
-                if (bkt[e] >= 0) {
-                    pos[e] = atomicAdd(&hist[bkt[e]], 1);
-                    dk[pos[e]] = key[e];
+            double acc = (double)kv_val(x);
+            if (head && dup)
+                for (int q = p + 1; q < whi; ++q) {
+                    const uint64_t y = src[q];
+                    if (kv_key(y) != k) break;
+                    acc += (double)kv_val(y);
+                }
+            if (head) {
+                const int o = ob + __popc(hm & lt);
+                if constexpr (NW == 1) {
+                    out_col[obase + o] = k;
+                    out_val[obase + o] = (float)acc;
+                } else {
+                    stage[o] = pack_kv(k, (float)acc);
                 }
             }
-            __syncthreads();
-#pragma unroll
-            for (int e = 0; e < EPT; ++e) {
-                if (pos[e] >= 0) {
-                    const int bs = bkt[e] ? hist[bkt[e] - 1] : 0, be = hist[bkt[e]];
-                    const int32_t kk = key[e];
-                    int rank = 0;
-                    for (int q = bs; q < be; ++q) {
-                        const int32_t kq = dk[q];
-                        rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
-                    }
-                    dk2[bs + rank] = kk;
-                    dv2[bs + rank] = val[e];
-                }
-            }
-            __syncthreads();
-            // ---- reduce: contiguous slices of the sorted array [0, tot); heads at row starts too
-            const int L = tot;
-            const int E = ((L + THREADS - 1) / THREADS) | 1;
-            const int q0 = min(L, (int)threadIdx.x * E), q1 = min(L, q0 + E);
-            int r;
-            {
-                int lo = 0, hi = nsub;     // row of sorted position q0
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (r_len[mid] <= q0) lo = mid; else hi = mid;
-                }
-                r = lo;
-            }
-            int nh = 0;
-            {
-                int rr = r;
-                for (int q = q0; q < q1; ++q) {
-                    while (r_len[rr + 1] <= q) ++rr;
-                    nh += (q == r_len[rr] || dk2[q] != dk2[q - 1]);
-                }
-            }
-            int U;
-            int o = g.excl_sum(nh, sc, &U);
-            for (int q = q0; q < q1; ++q) {
-                while (r_len[r + 1] <= q) ++r;
-                const bool rs = q == r_len[r];
-                if (rs || dk2[q] != dk2[q - 1]) {
-                    if (rs) r_uoff[r] = o;
-                    const int32_t kk = dk2[q];
-                    double acc = (double)dv2[q];
-                    for (int t2 = q + 1; t2 < r_len[r + 1] && dk2[t2] == kk; ++t2) acc += (double)dv2[t2];
-                    dk[o] = kk;
-                    dv[o] = (float)acc;
-                    ++o;
-                }
-            }
-            if (threadIdx.x == 0) r_uoff[nsub] = U;
-            __syncthreads();
-            // ---- store: warp per row, merged entries to the head of the row's bucket
-            for (int q = w; q < nsub; q += NW) {
-                const int u0 = r_uoff[q], u1 = r_uoff[q + 1];
-                const int64_t dst = r_src[q];
-                for (int t2 = u0 + lane; t2 < u1; t2 += 32) {
-                    chat_col[dst + t2 - u0] = dk[t2];
-                    chat_val[dst + t2 - u0] = dv[t2];
-                }
-                if (lane == 0) ccount[r_row[q]] = u1 - u0;
-            }
-            done += nsub;
-            __syncthreads();
+            ob += __popc(hm);
         }
+        if constexpr (NW > 1) {
+            if (lane == 0) wcnt[wg] = ob;
+            g.sync();
+            int wb = 0;
+            for (int w = 0; w < wg; ++w) wb += wcnt[w];
+            for (int q = lane; q < ob; q += 32) {
+                const uint64_t x = stage[q];
+                out_col[obase + wb + q] = kv_key(x);
+                out_val[obase + wb + q] = kv_val(x);
+            }
+            if (g.gtid == 0 && !out_col_all) {
+                int U = 0;
+                for (int w = 0; w < NW; ++w) U += wcnt[w];
+                ccount[i] = U;
+            }
+        } else {
+            if (lane == 0 && !out_col_all) ccount[i] = ob;
+        }
+        g.sync();
     }
 }
 
@@ -936,7 +1014,10 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
                                                                 int32_t *__restrict__ chat_col,
                                                                 float *__restrict__ chat_val,
                                                                 int64_t *__restrict__ ccount,
-                                                                const unsigned *__restrict__ dev_count) {
+                                                                const unsigned *__restrict__ dev_count,
+                                                                const int64_t *__restrict__ crowptr,
+                                                                int32_t *__restrict__ out_col,
+                                                                float *__restrict__ out_val) {
     if (dev_count) nrows = *dev_count;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ int sc_all[GROUPS][NW + 1];
@@ -946,9 +1027,11 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
         const int i = rows[r];
         const int64_t s = rowoff[i];
         const int L = (int)(rowoff[i + 1] - s);
+        const int64_t o = out_col ? crowptr[i] : s;
         const int U = merge_row_in_smem<NW, GROUPS, CAP>(g, slice, sc_all[g.gid], chat_col, chat_val, s, L,
-                                                         (int)rowwork[i], chat_col + s, chat_val + s);
-        if (g.gtid == 0) ccount[i] = U;
+                                                         (int)rowwork[i], (out_col ? out_col : chat_col) + o,
+                                                         (out_col ? out_val : chat_val) + o);
+        if (g.gtid == 0 && !out_col) ccount[i] = U;
     }
 }
 
@@ -972,7 +1055,7 @@ constexpr int kLimEPT = kLimCap / kLimThreads;   // 18
 constexpr int kLimWindow = 16384;
 constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
 constexpr int kLimSortBytes = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
-                                    kLimCap * 16 + ceil_pow2(kLimCap) * 4,     // bucket sort
+                                    kLimCap * 16 + (hidx(ceil_pow2(kLimCap)) + 4) * 4,  // bucket sort
                                     kLimWindow * 8 + (kLimWindow / 32) * 4);   // dense window
 constexpr int kCoarseLog = 10;
 constexpr int kCoarseBins = 1 << kCoarseLog;
@@ -1406,14 +1489,16 @@ __device__ __forceinline__ V shfl_up_vec(const V &v, const V &carry) {
     return p;
 }
 
-__global__ void __launch_bounds__(256) k_compact_rows(const int64_t *__restrict__ crowptr, int64_t M,
+__global__ void __launch_bounds__(256) k_compact_rows(const int32_t *__restrict__ list,
+                                                      const int64_t *__restrict__ crowptr, int64_t M,
                                                       const int64_t *__restrict__ rowoff,
                                                       const int32_t *__restrict__ chat_col,
                                                       const float *__restrict__ chat_val,
                                                       int32_t *__restrict__ out_col, float *__restrict__ out_val) {
     const int lane = lane_id();
-    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < M;
-         i += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < M;
+         q += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t i = list ? list[q] : q;       // M = list length when a list is given
         const int64_t dst = crowptr[i];
         const int64_t cnt = crowptr[i + 1] - dst;
         if (cnt == 0 || cnt > kCompactWarpMax) continue;

@@ -240,31 +240,37 @@ static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *ro
     CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
     LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
-        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0));
+        rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0,
+        nullptr, nullptr, nullptr));
     return SPGEMM_OK;
 }
 
-template <int THREADS, int CAPN>
-static int launch_batch_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
-                            int ctas_per_sm) {
+template <int GROUPS, int VPT>
+static int launch_wcs_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name) {
     if (cnt == 0) return SPGEMM_OK;
-    const int smem = BatchSmem<THREADS, CAPN>::kBytes;
-    CK(cudaFuncSetAttribute(k_merge_batch<THREADS, CAPN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    const int64_t grid = std::min<int64_t>(cdiv(cnt, kBatchRows), (int64_t)p->num_sms * ctas_per_sm * 4);
-    LAUNCH(name, s, k_merge_batch<THREADS, CAPN><<<(unsigned)grid, THREADS, smem, s>>>(
-        rows, cnt, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
+    const int smem = WcsSmem<VPT>::kBytes * GROUPS;
+    auto kern = k_merge_wcs<GROUPS, VPT>;
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * GROUPS, smem));
+    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
+    LAUNCH(name, s, kern<<<(unsigned)grid, 32 * GROUPS, smem, s>>>(rows, cnt, p->rowoff, p->rowwork, p->chat_col,
+                                                                  p->chat_val, p->ccount, nullptr, nullptr, nullptr));
     return SPGEMM_OK;
 }
 
-template <int CAP, int WARPS>
-static int launch_wnm_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
-                          int ctas_per_sm) {
+template <int NW, int GROUPS, int CAP>
+static int launch_wmp_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name) {
     if (cnt == 0) return SPGEMM_OK;
-    const int smem = WnmSmem<CAP, WARPS>::kBytes;
-    CK(cudaFuncSetAttribute(k_merge_wnm<CAP, WARPS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-    const int64_t grid = std::min<int64_t>(cdiv(cnt, WARPS), (int64_t)p->num_sms * ctas_per_sm * 8);
-    LAUNCH(name, s, k_merge_wnm<CAP, WARPS><<<(unsigned)grid, WARPS * 32, smem, s>>>(
-        rows, cnt, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
+    const int smem = WmpSmem<CAP>::kBytes * GROUPS;
+    auto kern = k_merge_wmp<NW, GROUPS, CAP>;
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NW * 32 * GROUPS, smem));
+    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
+    LAUNCH(name, s, kern<<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(rows, cnt, p->rowoff, p->rowwork, p->chat_col,
+                                                                       p->chat_val, p->ccount, nullptr, nullptr,
+                                                                       nullptr));
     return SPGEMM_OK;
 }
 
@@ -626,45 +632,31 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         LAUNCH("merge_pass", s, k_merge_pass<<<grid_for(cnt, 256), 256, 0, s>>>(rows, cnt, p->rowwork, p->ccount));
     rows = rows_of(kRowBucketWarp, kRowBucketWarp + 1, &cnt);
     if (cnt > 0)
-        LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(rows, cnt, p->rowoff,
-                                                                                      p->chat_col, p->chat_val, p->ccount));
+        LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
+            rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, nullptr, nullptr, nullptr));
     CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
-    // merge_variant (options.reserved[0], tuning): 0 per-row bucket sort (default),
-    // 1 batched multi-row bucket sort, 2 per-row bucket sort with 16 slots per thread
+    // merge_variant (options.reserved[0], tuning): 0 default (warp merge-path natural merge sort
+    // for the <= 256 bin, per-row bucket sort for the <= 1024 / <= 4096 bins), 1 register-staged
+    // counting sort for the <= 256 / <= 1024 bins, 2 bucket sort everywhere, 3 merge-path everywhere
     const int variant = p->opt.reserved[0];
-    if (variant == 1) {
-        rows = rows_of(kRowBucketSort256, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_batch_bin<256, 2048>(p, s, rows, cnt, "merge_batch2k", 4));
-        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_batch_bin<512, 4096>(p, s, rows, cnt, "merge_batch4k", 2));
-    } else if (variant == 2) {
-        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-        TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
-        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_bucket_bin<2, 4, 16>(p, s, rows, cnt, "merge_bucket1k", 4));
-        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_bucket_bin<8, 1, 16>(p, s, rows, cnt, "merge_bucket4k", 4));
-    } else if (variant == 3) {
-        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-        TRY(launch_wnm_bin<256, 8>(p, s, rows, cnt, "merge_wnm256", 6));
-        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_wnm_bin<1024, 4>(p, s, rows, cnt, "merge_wnm1k", 3));
-        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
-    } else {
-        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-        TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
-        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
-        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
-    }
+    rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
+    if (variant == 1) TRY(launch_wcs_bin<4, 2>(p, s, rows, cnt, "merge_wcs256"));
+    else if (variant == 2) TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
+    else TRY(launch_wmp_bin<1, 8, 256>(p, s, rows, cnt, "merge_wmp256"));
+    rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
+    if (variant == 1) TRY(launch_wcs_bin<1, 8>(p, s, rows, cnt, "merge_wcs1k"));
+    else if (variant == 3) TRY(launch_wmp_bin<1, 4, 1024>(p, s, rows, cnt, "merge_wmp1k"));
+    else TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
+    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+    if (variant == 3) TRY(launch_wmp_bin<4, 1, 4096>(p, s, rows, cnt, "merge_wmp4k"));
+    else TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
         CK(cudaFuncSetAttribute(k_merge_rows<8, 1, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
-            p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count));
+            p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count, nullptr, nullptr,
+            nullptr));
     }
     if (p->nlim > 0) {
         CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
@@ -722,7 +714,7 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
     }
     if (nnz > 0) {
         LAUNCH("compact", s, k_compact_rows<<<grid_for(p->m * 32, 256, (int64_t)p->num_sms * 16), 256, 0, s>>>(
-            p->crowptr, p->m, p->rowoff, p->chat_col, p->chat_val, dcol, dval));
+            nullptr, p->crowptr, p->m, p->rowoff, p->chat_col, p->chat_val, dcol, dval));
         if (p->nlim > 0)
             LAUNCH("compact", s, k_compact_long<<<(unsigned)std::min<int64_t>(p->nlim, (int64_t)p->num_sms * 4),
                                                    kCompactLongThreads, 0, s>>>(

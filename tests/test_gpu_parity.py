@@ -68,8 +68,9 @@ def _deg(inp):
 
 CASES = [
     ("C1", dict()),
-    ("C1", dict(reserved=(1,) + (0,) * 15)),   # merge variant: batched multi-row bucket sort
-    ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: warp natural merge
+    ("C1", dict(reserved=(1,) + (0,) * 15)),   # merge variant: register-staged counting sort
+    ("C1", dict(reserved=(2,) + (0,) * 15)),   # merge variant: smem bucket sort everywhere
+    ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: merge-path everywhere
     ("C1", dict(reserved=(0, 1) + (0,) * 14)),  # B-Gathering: per-pair micro-block loops
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
@@ -154,7 +155,7 @@ def _rows_sorted(m, rowoff, cols, vals):
     return out
 
 
-@pytest.mark.parametrize("name,opts", CASES[:1] + CASES[3:7])
+@pytest.mark.parametrize("name,opts", CASES[:1] + CASES[4:8])
 def test_stage3_expansion_is_eq2(name, opts):
     inp = _inp(name)
     p, keep = _plan(inp, **opts)
@@ -207,7 +208,8 @@ def test_c_matches_oracle(name, opts):
 def test_random_tiny(shape, dens, seed, skew, values):
     inp = synth.random_tiny(*shape, dens[0], dens[1], seed, values=values, skew=skew)
     A, B = spg.from_inputs(inp, "cuda")
-    for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(3,) + (0,) * 15)):
+    for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(1,) + (0,) * 15),
+                 dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15)):
         C = spg.matmul(A, B, **opts)
         assert_c_matches(C, inp, signed=(values == "signed"))
 
