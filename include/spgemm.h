@@ -123,7 +123,7 @@ typedef struct {
     int64_t t_dom, t_lim;      /* thresholds actually used                                     */
     int64_t n_dominator, n_normal, n_low, n_pieces_split;
     int64_t n_gather_bin[6];   /* low performers per gathering bin n (2^(n-1) < t <= 2^n)      */
-    int64_t n_rows_bin[6];     /* empty, passthrough, warp(<=32), warp-radix, cta-radix, limited */
+    int64_t n_rows_bin[6];     /* empty, single-run, <=32 slots, <=1024 slots, <=4096 slots, limited */
     int64_t bytes_workspace;   /* device bytes held by the plan                                */
 } spgemm_stats_t;
 

@@ -22,20 +22,24 @@ constexpr int kNumPairBuckets = 99;
 // row processing classes (SPGEMM_VIEW_ROW_CLASS) and buckets
 enum : int8_t { RC_EMPTY = 0, RC_PASS = 1, RC_WARP = 2, RC_WARP_SORT = 3, RC_GROUP_SORT = 4, RC_LIMITED = 5 };
 constexpr int kRowBucketPass = 0;
-constexpr int kRowBucketWarp = 1;      // L <= 32: register bitonic
-constexpr int kRowBucketSort256 = 2;   // L <= 256: one warp, smem natural merge sort
-constexpr int kRowBucketSort1K = 3;    // L <= 1024: two warps
-constexpr int kRowBucketSort4K = 4;    // L <= t_lim: eight warps
-constexpr int kRowBucketLim0 = 5;      // 5 + (39 - floor(log2 L)): longest rows first
-constexpr int kRowBucketEmpty = 45;
-constexpr int kNumRowBuckets = 46;
+constexpr int kRowBucketWarp = 1;      // cap <= 32: register bitonic
+constexpr int kRowBucketSort256 = 2;   // cap <= 256: one warp, merge-path natural merge sort
+constexpr int kRowBucketSort512 = 3;   // cap <= 512 / 1K / 2K / 4K: bucket sort, 2 / 4 / 8 / 16 warps
+constexpr int kRowBucketSort1K = 4;
+constexpr int kRowBucketSort2K = 5;
+constexpr int kRowBucketSort4K = 6;
+constexpr int kRowBucketLim0 = 7;      // 7 + (39 - floor(log2 L)): longest rows first
+constexpr int kRowBucketEmpty = 47;
+constexpr int kNumRowBuckets = 48;
 constexpr int kWarpRowMax = 32;
 // Ĉ runs are padded to multiples of kRunAlign slots (16 B) with sentinel entries
 // (col = INT32_MAX, val = 0) so that every run starts 16-byte aligned (vector stores).
 constexpr int kRunAlign = 4;
 __host__ __device__ __forceinline__ int64_t pad_run(int64_t x) { return (x + kRunAlign - 1) & ~(int64_t)(kRunAlign - 1); }
 constexpr int kSort256Max = 256;
+constexpr int kSort512Max = 512;
 constexpr int kSort1KMax = 1024;
+constexpr int kSort2KMax = 2048;
 constexpr int64_t kLimitCapacity = 4096;   // largest bucket length of the non-limited merge bins
 
 struct PlanScalars {
@@ -345,7 +349,9 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
         }
         else if (cap <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
         else if (cap <= kSort256Max) { c = RC_WARP_SORT; b = kRowBucketSort256; }
+        else if (cap <= kSort512Max) { c = RC_WARP_SORT; b = kRowBucketSort512; }
         else if (cap <= kSort1KMax) { c = RC_WARP_SORT; b = kRowBucketSort1K; }
+        else if (cap <= kSort2KMax) { c = RC_GROUP_SORT; b = kRowBucketSort2K; }
         else { c = RC_GROUP_SORT; b = kRowBucketSort4K; }
         rcls[i] = c;
         bucket[i] = (uint8_t)b;

@@ -373,10 +373,11 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
             const int bs = hist[hidx(b)], be = hist[hidx(b + 1)];
             const int32_t kk = key[e];
             int rank = 0;
-            for (int q = bs; q < be; ++q) {
-                const int32_t kq = dk[q];
-                rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
-            }
+            if (be - bs > 1)     // (a bucket of one key is already in place)
+                for (int q = bs; q < be; ++q) {
+                    const int32_t kq = dk[q];
+                    rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
+                }
             dk2[bs + rank] = kk;
             dv2[bs + rank] = val[e];
         }
@@ -386,18 +387,37 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     L = tot;   // valid (non-sentinel) entries
     const int E = ((L + T - 1) / T) | 1;     // odd stride between thread slices: no bank conflicts
     const int p0 = min(L, g.gtid * E), p1 = min(L, p0 + E);
+    const int32_t before = p0 > 0 && p0 < L ? dk2[p0 - 1] : -1;   // (-1 is no column)
     int nh = 0;
-    for (int p = p0; p < p1; ++p) nh += (p == 0 || dk2[p] != dk2[p - 1]);
+    {
+        int32_t prevk = before;
+        for (int p = p0; p < p1; ++p) {
+            const int32_t k = dk2[p];
+            nh += k != prevk;
+            prevk = k;
+        }
+    }
     int U;
     int o = g.excl_sum(nh, sc, &U);
-    for (int p = p0; p < p1; ++p) {
-        if (p == 0 || dk2[p] != dk2[p - 1]) {
-            const int32_t kk = dk2[p];
-            double acc = (double)dv2[p];
-            for (int q = p + 1; q < L && dk2[q] == kk; ++q) acc += (double)dv2[q];
-            dk[o] = kk;
+    {   // a segment continuing from the previous slice is summed by that slice's thread
+        int32_t prevk = before, cur = -1;
+        double acc = 0.0;
+        for (int p = p0; p < p1; ++p) {
+            const int32_t k = dk2[p];
+            const float v = dv2[p];
+            if (k != prevk) {
+                if (cur != -1) { dk[o] = cur; dv[o] = (float)acc; ++o; }
+                cur = k;
+                acc = (double)v;
+            } else if (cur != -1) {
+                acc += (double)v;
+            }
+            prevk = k;
+        }
+        if (cur != -1) {
+            for (int q = p1; q < L && dk2[q] == cur; ++q) acc += (double)dv2[q];
+            dk[o] = cur;
             dv[o] = (float)acc;
-            ++o;
         }
     }
     g.sync();

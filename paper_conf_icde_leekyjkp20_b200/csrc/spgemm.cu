@@ -643,13 +643,27 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     if (variant == 1) TRY(launch_wcs_bin<4, 2>(p, s, rows, cnt, "merge_wcs256"));
     else if (variant == 2) TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
     else TRY(launch_wmp_bin<1, 8, 256>(p, s, rows, cnt, "merge_wmp256"));
-    rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-    if (variant == 1) TRY(launch_wcs_bin<1, 8>(p, s, rows, cnt, "merge_wcs1k"));
-    else if (variant == 3) TRY(launch_wmp_bin<1, 4, 1024>(p, s, rows, cnt, "merge_wmp1k"));
-    else TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
-    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-    if (variant == 3) TRY(launch_wmp_bin<4, 1, 4096>(p, s, rows, cnt, "merge_wmp4k"));
-    else TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    if (variant == 1) {
+        rows = rows_of(kRowBucketSort512, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_wcs_bin<1, 8>(p, s, rows, cnt, "merge_wcs1k"));
+    } else if (variant == 3) {
+        rows = rows_of(kRowBucketSort512, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_wmp_bin<1, 4, 1024>(p, s, rows, cnt, "merge_wmp1k"));
+    } else {
+        rows = rows_of(kRowBucketSort512, kRowBucketSort512 + 1, &cnt);
+        TRY(launch_bucket_bin<2, 4, 8>(p, s, rows, cnt, "merge_bucket512", 8));
+        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
+        TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
+    }
+    if (variant == 3) {
+        rows = rows_of(kRowBucketSort2K, kRowBucketSort4K + 1, &cnt);
+        TRY(launch_wmp_bin<4, 1, 4096>(p, s, rows, cnt, "merge_wmp4k"));
+    } else {
+        rows = rows_of(kRowBucketSort2K, kRowBucketSort2K + 1, &cnt);
+        TRY(launch_bucket_bin<8, 1, 8>(p, s, rows, cnt, "merge_bucket2k", 8));
+        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    }
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
@@ -775,7 +789,7 @@ int spgemm_get_stats(spgemm_plan_t p, spgemm_stats_t *st) {
     st->n_rows_bin[1] = p->row_starts[kRowBucketPass + 1] - p->row_starts[kRowBucketPass];
     st->n_rows_bin[2] = p->row_starts[kRowBucketWarp + 1] - p->row_starts[kRowBucketWarp];
     st->n_rows_bin[3] = p->row_starts[kRowBucketSort1K + 1] - p->row_starts[kRowBucketSort256];
-    st->n_rows_bin[4] = p->row_starts[kRowBucketSort4K + 1] - p->row_starts[kRowBucketSort4K];
+    st->n_rows_bin[4] = p->row_starts[kRowBucketSort4K + 1] - p->row_starts[kRowBucketSort2K];
     st->n_rows_bin[5] = p->nlim;
     st->bytes_workspace = p->bytes;
     return SPGEMM_OK;
