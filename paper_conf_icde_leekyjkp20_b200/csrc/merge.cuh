@@ -304,7 +304,8 @@ __device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const
     return wtot;
 }
 
-template <int NW, int GROUPS, int EPT>
+// LS: buckets = 2^LS x (slots rounded up to a power of two); more buckets, fewer shared ones
+template <int NW, int GROUPS, int EPT, int LS = 0>
 __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
                                                   int L, int32_t *dk, float *dv, int32_t *dk2, float *dv2,
                                                   int *hist, int32_t *out_col, float *out_val, int *sc) {
@@ -322,7 +323,7 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
     mn = g.reduce_min(mn, sc);
     mx = g.reduce_max(mx, sc);
     const uint32_t span = (uint32_t)(mx - mn);
-    const int lognb = nextpow2_log(L);
+    const int lognb = nextpow2_log(L) + LS;
     const int nb = 1 << lognb;
     const int bits = span ? 32 - __clz(span) : 0;
     const int sh = max(0, bits - lognb);
@@ -431,15 +432,15 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
 
 constexpr int ceil_pow2(int x) { return x <= 1 ? 1 : 2 * ceil_pow2((x + 1) / 2); }
 
-template <int NW, int EPT>
+template <int NW, int EPT, int LS = 0>
 struct BucketSmem {
     static constexpr int kCap = NW * 32 * EPT;
-    static constexpr int kNb = ceil_pow2(kCap);
+    static constexpr int kNb = ceil_pow2(kCap) << LS;
     static constexpr int kBytes = kCap * 16 + (hidx(kNb) + 4) * 4;
 };
 
 // Rows of one bin: bucket sort per row; rows whose buckets overflow go to a fallback list.
-template <int NW, int GROUPS, int EPT>
+template <int NW, int GROUPS, int EPT, int LS = 0>
 __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k_merge_bucket(const int32_t *__restrict__ rows, int64_t nrows,
                                                                   const int64_t *__restrict__ rowoff,
                                                                   int32_t *__restrict__ chat_col,
@@ -450,7 +451,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
                                                                   const int64_t *__restrict__ crowptr,
                                                                   int32_t *__restrict__ out_col,
                                                                   float *__restrict__ out_val) {
-    using S = BucketSmem<NW, EPT>;
+    using S = BucketSmem<NW, EPT, LS>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ int sc_all[GROUPS][NW + 1];
     const Group<NW, GROUPS> g;
@@ -466,7 +467,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
         const int L = (int)(rowoff[i + 1] - s);
         if (L > S::kCap) continue;          // (limited list) rows above this kernel's capacity
         const int64_t o = out_col ? crowptr[i] : s;
-        const int U = bucket_sort_reduce<NW, GROUPS, EPT>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
+        const int U = bucket_sort_reduce<NW, GROUPS, EPT, LS>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
                                                           (out_col ? out_col : chat_col) + o,
                                                           (out_col ? out_val : chat_val) + o, sc_all[g.gid]);
         if (g.gtid == 0) {
@@ -1529,14 +1530,7 @@ __global__ void __launch_bounds__(256) k_compact_rows(const int32_t *__restrict_
         const int64_t nvec = (cnt + sh + 3) >> 2;
         int4 carry_c = make_int4(0, 0, 0, 0);
         float4 carry_v = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int64_t m0 = 0; m0 < nvec; m0 += 32) {
-            const int64_t m = m0 + lane;
-            int4 c = make_int4(0, 0, 0, 0);
-            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (4 * m < cnt) {
-                c = *reinterpret_cast<const int4 *>(chat_col + src + 4 * m);
-                v = *reinterpret_cast<const float4 *>(chat_val + src + 4 * m);
-            }
+        auto emit = [&](int64_t m, const int4 &c, const float4 &v) {
             const int4 oc = realign4(c, shfl_up_vec(c, carry_c), sh);
             const float4 ov = realign4(v, shfl_up_vec(v, carry_v), sh);
             carry_c.x = __shfl_sync(kFull, c.x, 31); carry_c.y = __shfl_sync(kFull, c.y, 31);
@@ -1546,8 +1540,8 @@ __global__ void __launch_bounds__(256) k_compact_rows(const int32_t *__restrict_
             if (m < nvec) {
                 const int64_t j0 = 4 * m - sh;       // row slot of the vector's first element
                 if (j0 >= 0 && j0 + 4 <= cnt) {
-                    *reinterpret_cast<int4 *>(out_col + dst_a + 4 * m) = oc;
-                    *reinterpret_cast<float4 *>(out_val + dst_a + 4 * m) = ov;
+                    __stcs(reinterpret_cast<int4 *>(out_col + dst_a + 4 * m), oc);
+                    __stcs(reinterpret_cast<float4 *>(out_val + dst_a + 4 * m), ov);
                 } else {                              // ragged head / tail of the row
                     const int32_t cc[4] = {oc.x, oc.y, oc.z, oc.w};
                     const float vv[4] = {ov.x, ov.y, ov.z, ov.w};
@@ -1559,6 +1553,22 @@ __global__ void __launch_bounds__(256) k_compact_rows(const int32_t *__restrict_
                         }
                 }
             }
+        };
+        for (int64_t m0 = 0; m0 < nvec; m0 += 64) {   // two vectors in flight per lane
+            int4 c[2];
+            float4 v[2];
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+                const int64_t m = m0 + 32 * u + lane;
+                c[u] = make_int4(0, 0, 0, 0);
+                v[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (4 * m < cnt) {
+                    c[u] = __ldcs(reinterpret_cast<const int4 *>(chat_col + src + 4 * m));
+                    v[u] = __ldcs(reinterpret_cast<const float4 *>(chat_val + src + 4 * m));
+                }
+            }
+            emit(m0 + lane, c[0], v[0]);
+            if (m0 + 32 < nvec) emit(m0 + 32 + lane, c[1], v[1]);
         }
     }
 }

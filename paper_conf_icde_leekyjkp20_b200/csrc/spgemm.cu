@@ -232,14 +232,14 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     return SPGEMM_OK;
 }
 
-template <int NW, int GROUPS, int EPT>
+template <int NW, int GROUPS, int EPT, int LS = 0>
 static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
                              int ctas_per_sm, bool fallback_list = true) {
     if (cnt == 0) return SPGEMM_OK;
-    const int smem = BucketSmem<NW, EPT>::kBytes * GROUPS;
-    CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    const int smem = BucketSmem<NW, EPT, LS>::kBytes * GROUPS;
+    CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT, LS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
-    LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
+    LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT, LS><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
         rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0,
         nullptr, nullptr, nullptr));
     return SPGEMM_OK;
