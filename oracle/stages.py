@@ -99,7 +99,9 @@ def split_pieces(inp, cls, piece_work: int, b_tile: int, split_ca_max: int):
     ("several elements from each column vector are shifted to the next vector
     sequentially", L374-L376 L); empty trailing pieces are not emitted (Fig. 5: a
     25-computation block split into three blocks, L386-L388 L).  The B row is cut
-    into tiles of b_tile entries only when it exceeds b_tile (R4)."""
+    into tiles of b_tile entries (rounded up to a multiple of 4) only when it exceeds
+    b_tile (R4)."""
+    b_tile = -(-b_tile // 4) * 4   # R4: a tile is whole 16-byte vectors (4 slots) of the run
     out = []
     for k in np.nonzero(cls == DOMINATOR)[0]:
         a0, a1 = int(inp.a_colptr[k]), int(inp.a_colptr[k + 1])

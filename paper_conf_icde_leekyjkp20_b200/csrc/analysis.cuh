@@ -323,6 +323,12 @@ __global__ void k_piece_whole(const int32_t *__restrict__ list, int64_t n, const
     }
 }
 
+// padded length of every B row (input of the B' row-pointer scan)
+__global__ void k_row_padded_len(const int64_t *__restrict__ b_rowptr, int64_t K, int64_t *__restrict__ out) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x)
+        out[k] = pad_run(b_rowptr[k + 1] - b_rowptr[k]);
+}
+
 // Merge row classes.  Limited rows (L > t_lim, L452-L477 L) get B-Limited merge blocks;
 // a row made of a single run (one A entry) is already sorted and duplicate-free.
 __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict__ rowwork,

@@ -134,8 +134,13 @@ struct spgemm_plan_s {
     int32_t *pair_order = nullptr, *row_order = nullptr;
     int64_t pair_starts[kNumPairBuckets + 1] = {};
     int64_t row_starts[kNumRowBuckets + 1] = {};
-    Piece *pieces = nullptr;
-    int64_t *gather_item_off = nullptr;
+    Piece *pieces = nullptr;       // split pieces, whole Normal blocks, gathered Low-performer blocks
+    int64_t *piece_uoff = nullptr; // unit (16-byte vector) prefix over pieces
+    int64_t *tile_p0 = nullptr;    // first piece of every expansion tile
+    int64_t n_low = 0, n_pieces_all = 0;
+    int64_t *b_prow = nullptr;     // B' (rows padded to 4 slots): row starts, cols, values
+    int32_t *bp_col = nullptr;
+    float *bp_val = nullptr;
 
     int64_t n_split_pieces = 0, n_whole = 0;
     int64_t *piece_off = nullptr;
@@ -348,6 +353,7 @@ int spgemm_plan(const spgemm_csc_t *A, const spgemm_csr_t *B, const spgemm_optio
     if (p->opt.split_ca_max <= 0) p->opt.split_ca_max = d.split_ca_max;
     if (p->opt.piece_work <= 0) p->opt.piece_work = d.piece_work;
     if (p->opt.split_b_tile <= 0) p->opt.split_b_tile = d.split_b_tile;
+    p->opt.split_b_tile = (int32_t)pad_run(p->opt.split_b_tile);   // R4: whole 16-byte vectors
     if (p->opt.limit_ctas_per_sm <= 0) p->opt.limit_ctas_per_sm = d.limit_ctas_per_sm;
     int r = plan_impl(p, A, B, (cudaStream_t)stream);
     if (r != SPGEMM_OK) {
@@ -501,7 +507,11 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     }
     const int64_t ndom = p->pair_starts[kPairBucketSplit + 1] - p->pair_starts[kPairBucketSplit];
     p->n_whole = p->pair_starts[kPairBucketPiece + 1] - p->pair_starts[kPairBucketPiece];
-    TRY(palloc(p, &p->pieces, p->n_split_pieces + p->n_whole, s));
+    // B-Gathering blocks: the Low performers, in gather-list order (bins of 2^(n-1) < nnz(b_k*) <= 2^n)
+    const int64_t g_lo = p->pair_starts[kPairBucketGather0], g_hi = p->pair_starts[kPairBucketEmpty];
+    p->n_low = g_hi - g_lo;
+    p->n_pieces_all = p->n_split_pieces + p->n_whole + p->n_low;
+    TRY(palloc(p, &p->pieces, p->n_pieces_all, s));
     if (ndom > 0) {
         const int32_t *dom = p->pair_order + p->pair_starts[kPairBucketSplit];
         LAUNCH("piece_fill", s, k_piece_fill<<<(unsigned)cdiv(ndom * 32, 256), 256, 0, s>>>(
@@ -511,18 +521,39 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_whole, 256), 256, 0, s>>>(
             p->pair_order + p->pair_starts[kPairBucketPiece], p->n_whole, p->a_colptr, p->b_rowptr,
             p->pieces + p->n_split_pieces));
-    // B-Gathering items: prefix of nnz(a_*k) over the gather lists (bins are contiguous in it)
-    {
-        const int64_t g_lo = p->pair_starts[kPairBucketGather0], g_hi = p->pair_starts[kPairBucketEmpty];
-        TRY(palloc(p, &p->gather_item_off, g_hi - g_lo + 1, s));
-        if (g_hi > g_lo) {
-            Temp tg(s);
-            int64_t *cnt;
-            TRY(talloc(p, tg, &cnt, g_hi - g_lo));
-            LAUNCH("gather_items", s, k_gather_item_counts<<<grid_for(g_hi - g_lo, 256), 256, 0, s>>>(
-                p->pair_order + g_lo, g_hi - g_lo, p->a_colptr, cnt));
-            TRY(scan_excl(p, cnt, g_hi - g_lo, p->gather_item_off, s, "gather_scan"));
-        }
+    if (p->n_low > 0)
+        LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_low, 256), 256, 0, s>>>(
+            p->pair_order + g_lo, p->n_low, p->a_colptr, p->b_rowptr, p->pieces + p->n_split_pieces + p->n_whole));
+    TRY(palloc(p, &p->piece_uoff, p->n_pieces_all + 1, s));
+    if (p->n_pieces_all > 0) {
+        Temp tu(s);
+        int64_t *units;
+        TRY(talloc(p, tu, &units, p->n_pieces_all));
+        LAUNCH("piece_units", s, k_piece_units<<<grid_for(p->n_pieces_all, 256), 256, 0, s>>>(
+            p->pieces, p->n_pieces_all, units));
+        TRY(scan_excl(p, units, p->n_pieces_all, p->piece_uoff, s, "piece_scan"));
+        // (units <= nnz(Ĉ)/4 + #pieces; the tile map is sized for that bound, no host sync)
+        const int64_t ntiles_max = cdiv(p->chat_cap / 4 + p->n_pieces_all, kExpTile);
+        TRY(palloc(p, &p->tile_p0, ntiles_max + 1, s));
+        LAUNCH("piece_scan", s, k_tile_first_piece<<<grid_for(ntiles_max + 1, 256), 256, 0, s>>>(
+            p->piece_uoff, p->n_pieces_all, ntiles_max, p->tile_p0));
+    } else {
+        CK(cudaMemsetAsync(p->piece_uoff, 0, 8, s));
+    }
+    // B' = B with rows padded to 4 slots (16-byte aligned vector loads in the expansion)
+    TRY(palloc(p, &p->b_prow, K + 1, s));
+    TRY(palloc(p, &p->bp_col, p->nnz_b + 3 * K, s));
+    TRY(palloc(p, &p->bp_val, p->nnz_b + 3 * K, s));
+    if (K > 0) {
+        Temp tpl(s);
+        int64_t *plen;
+        TRY(talloc(p, tpl, &plen, K));
+        LAUNCH("pad_b", s, k_row_padded_len<<<grid_for(K, 256), 256, 0, s>>>(p->b_rowptr, K, plen));
+        TRY(scan_excl(p, plen, K, p->b_prow, s, "pad_b"));
+        LAUNCH("pad_b", s, k_pad_b<<<grid_for(K, 256), 256, 0, s>>>(
+            p->b_rowptr, p->b_colidx, p->b_val, K, p->b_prow, p->bp_col, p->bp_val));
+    } else {
+        CK(cudaMemsetAsync(p->b_prow, 0, 8, s));
     }
     // limited rows: index map, run lists, B-Limited scratch
     p->nlim = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketLim0];
@@ -575,40 +606,10 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     cudaStream_t s = (cudaStream_t)stream;
     p->last_stream = s;
     CK(cudaSetDevice(p->dev));
-    const int64_t np = p->n_split_pieces + p->n_whole;
-    if (np > 0)
-        LAUNCH("expand_pieces", s, k_expand_pieces<<<(unsigned)np, kPieceThreads, 0, s>>>(
-            p->pieces, p->a_val, p->b_rowptr, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
-    const bool items = p->opt.reserved[1] == 0;   // load-balanced B-Gathering (default)
-    {
-        const int64_t g_lo = p->pair_starts[kPairBucketGather0], g_hi = p->pair_starts[kPairBucketEmpty];
-        if (items && g_hi > g_lo)
-            LAUNCH("expand_gathered", s, k_expand_gathered_items<<<(unsigned)p->num_sms * 8, 256, 0, s>>>(
-                p->pair_order + g_lo, p->gather_item_off, 0, g_hi - g_lo, p->a_colptr, p->a_val, p->b_rowptr,
-                p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val));
-    }
-    for (int nb = 0; nb < 6 && !items; ++nb) {
-        const int64_t lo = p->pair_starts[kPairBucketGather0 + nb * 16];
-        const int64_t cnt = p->pair_starts[kPairBucketGather0 + nb * 16 + 16] - lo;
-        if (cnt == 0) continue;
-        const int32_t *list = p->pair_order + lo;
-        const int lanes = nb >= 2 ? (1 << nb) / 4 : 1;   // lanes per gathered pair (k_expand_gathered<N>::V)
-        const unsigned grid = (unsigned)cdiv(cnt * lanes, 256);
-#define GATHER_CASE(N)                                                                                      \
-    case N:                                                                                                 \
-        LAUNCH("expand_gathered", s, k_expand_gathered<N><<<grid, 256, 0, s>>>(                             \
-            list, cnt, p->a_colptr, p->a_val, p->b_rowptr, p->b_colidx, p->b_val, p->base, p->chat_col, p->chat_val)); \
-        break;
-        switch (nb) {
-            GATHER_CASE(0)
-            GATHER_CASE(1)
-            GATHER_CASE(2)
-            GATHER_CASE(3)
-            GATHER_CASE(4)
-            GATHER_CASE(5)
-        }
-#undef GATHER_CASE
-    }
+    if (p->n_pieces_all > 0)
+        LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * 8, kExpThreads, 0, s>>>(
+            p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_prow, p->bp_col, p->bp_val, p->a_val,
+            p->base, p->chat_col, p->chat_val));
     p->state = 2;
     return SPGEMM_OK;
 }

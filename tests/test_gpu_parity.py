@@ -71,7 +71,6 @@ CASES = [
     ("C1", dict(reserved=(1,) + (0,) * 15)),   # merge variant: register-staged counting sort
     ("C1", dict(reserved=(2,) + (0,) * 15)),   # merge variant: smem bucket sort everywhere
     ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: merge-path everywhere
-    ("C1", dict(reserved=(0, 1) + (0,) * 14)),  # B-Gathering: per-pair micro-block loops
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
     ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
@@ -155,7 +154,7 @@ def _rows_sorted(m, rowoff, cols, vals):
     return out
 
 
-@pytest.mark.parametrize("name,opts", CASES[:1] + CASES[4:8])
+@pytest.mark.parametrize("name,opts", CASES[:1] + CASES[4:7])
 def test_stage3_expansion_is_eq2(name, opts):
     inp = _inp(name)
     p, keep = _plan(inp, **opts)
