@@ -162,9 +162,12 @@ def main():
         inp, A, B = inp_full, A_full, B_full
     stream = torch.cuda.current_stream(dev)
     opts = dict(validate=0)
-    if os.environ.get("SPGEMM_MERGE_VARIANT"):
-        v = (0,) * 16
-        opts["reserved"] = tuple([int(os.environ["SPGEMM_MERGE_VARIANT"])] + [0] * 15)
+    if os.environ.get("SPGEMM_RESERVED"):   # tuning knobs: "index=value,..."
+        res = [0] * 16
+        for kv in os.environ["SPGEMM_RESERVED"].split(","):
+            q, v = kv.split("=")
+            res[int(q)] = int(v)
+        opts["reserved"] = tuple(res)
     flush = torch.zeros(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
 
     def step():
@@ -196,6 +199,9 @@ def main():
         p = spg.Plan(A, B, stream=stream, **opts)
         C = p.execute()
         st = p.stats()
+        if os.environ.get("SPGEMM_RESERVED", "").find("1=2") >= 0:
+            prof = p.inspect(spg.VIEW_UNIT_PROFILE, np.uint64)
+            print("unit-profile", json.dumps([int(x) for x in prof]), file=sys.stderr)
         p.destroy()
         e1.record(stream)
         e1.synchronize()
@@ -272,6 +278,7 @@ def main():
                           "def": "A + B + 2*Ĉ(8 B/product) + C, per step"},
         "kernel_ms": breakdown,
         "gpu_launches": launches_all,
+        "merge_units": {"units": st.get("n_units"), "fallback": st.get("n_units_fallback")},
         "clocks": clocks,
         "wall_s": round(wall, 3),
     }

@@ -125,6 +125,8 @@ typedef struct {
     int64_t n_gather_bin[6];   /* low performers per gathering bin n (2^(n-1) < t <= 2^n)      */
     int64_t n_rows_bin[6];     /* empty, single-run, <=32 slots, <=1024 slots, <=4096 slots, limited */
     int64_t bytes_workspace;   /* device bytes held by the plan                                */
+    int64_t n_units;           /* merge units (short-row groups + long rows), after spgemm_merge */
+    int64_t n_units_fallback;  /* units merged by the natural-merge-sort fallback               */
 } spgemm_stats_t;
 
 /* spgemm_inspect selectors: copy a plan array to host memory (tests, tooling). */
@@ -139,7 +141,8 @@ typedef enum {
                                                 4 cta-radix, 5 limited                        */
     SPGEMM_VIEW_CHAT_COL = 7,    /* int32[nnz_chat] after spgemm_expand (before merge)       */
     SPGEMM_VIEW_CHAT_VAL = 8,    /* fp32[nnz_chat]                                            */
-    SPGEMM_VIEW_CROWPTR = 9      /* int64[m+1] C row pointers after spgemm_merge             */
+    SPGEMM_VIEW_CROWPTR = 9,     /* int64[m+1] C row pointers after spgemm_merge             */
+    SPGEMM_VIEW_UNIT_PROFILE = 10 /* uint64[16] merge-unit phase clocks (options.reserved[1]=2) */
 } spgemm_view;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;

@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(_HERE, "libspgemm.so")
 
 SPGEMM_DEVICE, SPGEMM_HOST = 0, 1
 VIEW_WORK, VIEW_ROWWORK, VIEW_ROWOFF, VIEW_PAIR_CLASS, VIEW_PIECES, VIEW_GATHER, VIEW_ROW_CLASS, \
-    VIEW_CHAT_COL, VIEW_CHAT_VAL, VIEW_CROWPTR = range(10)
+    VIEW_CHAT_COL, VIEW_CHAT_VAL, VIEW_CROWPTR, VIEW_UNIT_PROFILE = range(11)
 
 EXPORTED = ["spgemm_abi_version", "spgemm_last_error", "spgemm_default_options", "spgemm_plan",
             "spgemm_expand", "spgemm_merge", "spgemm_output", "spgemm_execute", "spgemm_get_stats",
@@ -61,7 +61,7 @@ class Stats(ctypes.Structure):
         "m", "k", "n", "nnz_a", "nnz_b", "nnz_chat", "nnz_chat_rowwise", "nnz_c", "k_nonempty",
         "m_nonempty", "t_dom", "t_lim", "n_dominator", "n_normal", "n_low", "n_pieces_split")] + [
         ("n_gather_bin", ctypes.c_int64 * 6), ("n_rows_bin", ctypes.c_int64 * 6),
-        ("bytes_workspace", ctypes.c_int64)]
+        ("bytes_workspace", ctypes.c_int64), ("n_units", ctypes.c_int64), ("n_units_fallback", ctypes.c_int64)]
 
     def as_dict(self):
         d = {f: getattr(self, f) for f, _ in self._fields_}

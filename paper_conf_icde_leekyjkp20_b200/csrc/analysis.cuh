@@ -41,6 +41,7 @@ constexpr int kSort512Max = 512;
 constexpr int kSort1KMax = 1024;
 constexpr int kSort2KMax = 2048;
 constexpr int64_t kLimitCapacity = 4096;   // largest bucket length of the non-limited merge bins
+constexpr int kUnitRowMax = 2048;          // short rows (merged by the unit kernel): padded bucket <= this
 
 struct PlanScalars {
     unsigned long long nnz_chat;     // sum_k work[k]
@@ -52,6 +53,7 @@ struct PlanScalars {
     unsigned long long lim_runs;     // sum of runs over limited rows
     unsigned long long lim_max_deg;  // max runs of a limited row
     unsigned long long lim_max_L;    // max products of a limited row
+    unsigned long long long_slots;   // padded Ĉ slots of the long rows (side buffer of the merge)
     int invalid;                     // validation failure bits
     int pad;
 };
@@ -336,8 +338,8 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
                                                       const int32_t *__restrict__ deg, int64_t M, int64_t t_lim,
                                                       int64_t cap_max, int8_t *__restrict__ rcls,
                                                       uint8_t *__restrict__ bucket, PlanScalars *sc) {
-    __shared__ unsigned long long sm[3][8];
-    unsigned long long runs = 0, mdeg = 0, mlen = 0;
+    __shared__ unsigned long long sm[4][8];
+    unsigned long long runs = 0, mdeg = 0, mlen = 0, lslots = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
         // L = products of the row (paper class); cap = its padded bucket length (kernel capacity)
         const int64_t L = rowwork[i];
@@ -345,7 +347,7 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
         int8_t c;
         int b;
         if (L == 0) { c = RC_EMPTY; b = kRowBucketEmpty; }
-        else if (deg[i] == 1) { c = RC_PASS; b = kRowBucketPass; }
+        else if (deg[i] == 1 && cap <= kUnitRowMax) { c = RC_PASS; b = kRowBucketPass; }
         else if (L > t_lim || cap > cap_max) {
             c = RC_LIMITED;
             b = kRowBucketLim0 + (39 - min(39, ilog2_floor((uint64_t)L)));
@@ -361,15 +363,20 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
         else { c = RC_GROUP_SORT; b = kRowBucketSort4K; }
         rcls[i] = c;
         bucket[i] = (uint8_t)b;
+        if (cap > kUnitRowMax || c == RC_LIMITED) lslots += (unsigned long long)cap;   // long row (side buffer)
     }
     runs = warp_sum(runs);
     mdeg = warp_max(mdeg);
     mlen = warp_max(mlen);
-    if (lane_id() == 0) { sm[0][warp_id()] = runs; sm[1][warp_id()] = mdeg; sm[2][warp_id()] = mlen; }
+    lslots = warp_sum(lslots);
+    if (lane_id() == 0) {
+        sm[0][warp_id()] = runs; sm[1][warp_id()] = mdeg; sm[2][warp_id()] = mlen; sm[3][warp_id()] = lslots;
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned long long a = 0, b = 0, c = 0;
-        for (int w = 0; w < 8; ++w) { a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); }
+        unsigned long long a = 0, b = 0, c = 0, d = 0;
+        for (int w = 0; w < 8; ++w) { a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); d += sm[3][w]; }
+        if (d) atomicAdd(&sc->long_slots, d);
         if (a) atomicAdd(&sc->lim_runs, a);
         if (b) atomicMax(&sc->lim_max_deg, b);
         if (c) atomicMax(&sc->lim_max_L, c);

@@ -471,7 +471,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
                                                           (out_col ? out_col : chat_col) + o,
                                                           (out_col ? out_val : chat_val) + o, sc_all[g.gid]);
         if (g.gtid == 0) {
-            if (U >= 0) { if (!out_col) ccount[i] = U; }
+            if (U >= 0) ccount[i] = U;
             else if (fb_rows) fb_rows[atomicAdd(fb_count, 1u)] = i;
             else ccount[i] = -1;   // limited list: k_merge_limited takes the row (merge-path fallback)
         }
@@ -1052,7 +1052,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
         const int U = merge_row_in_smem<NW, GROUPS, CAP>(g, slice, sc_all[g.gid], chat_col, chat_val, s, L,
                                                          (int)rowwork[i], (out_col ? out_col : chat_col) + o,
                                                          (out_col ? out_val : chat_val) + o);
-        if (g.gtid == 0 && !out_col) ccount[i] = U;
+        if (g.gtid == 0) ccount[i] = U;
     }
 }
 
@@ -1100,6 +1100,9 @@ struct LimitedArgs {
     int64_t max_deg;
     int64_t stage_cap;
     unsigned long long *row_counter;
+    int32_t *out_col;             // merged rows go to out_col/out_val + out_off[i] (NULL: in place)
+    float *out_val;
+    const int64_t *out_off;
     int skip_small;
     int64_t coarse_cap;           // rows up to this many slots take the coarse-partition path
 };
@@ -1147,6 +1150,8 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t cap = g.rowoff[i + 1] - s;   // padded bucket length
         const int64_t L = g.rowwork[i];             // products
         if (cap <= kLimCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
+        int32_t *const oc = g.out_col ? g.out_col + g.out_off[i] : g.chat_col + s;
+        float *const ov = g.out_col ? g.out_val + g.out_off[i] : g.chat_val + s;
         if (cap <= kLimCap) {
             int32_t *dk = (int32_t *)smem_raw;
             float *dv = (float *)(smem_raw + kLimCap * 4);
@@ -1154,10 +1159,10 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
             float *dv2 = (float *)(smem_raw + kLimCap * 12);
             int *hist = (int *)(smem_raw + kLimCap * 16);
             int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
-                                                            dv2, hist, g.chat_col + s, g.chat_val + s, sc);
+                                                            dv2, hist, oc, ov, sc);
             if (U < 0)
                 U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
-                                                          g.chat_col + s, g.chat_val + s);
+                                                          oc, ov);
             if (threadIdx.x == 0) g.ccount[i] = U;
             __syncthreads();
             continue;
@@ -1344,10 +1349,10 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                         int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(
                             grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + kLimCap * 4),
                             (int32_t *)(smem_raw + kLimCap * 8), (float *)(smem_raw + kLimCap * 12),
-                            (int *)(smem_raw + kLimCap * 16), g.chat_col + s + nout, g.chat_val + s + nout, sc);
+                            (int *)(smem_raw + kLimCap * 16), oc + nout, ov + nout, sc);
                         if (U < 0)
                             U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, sc_col, sc_val, g0, n, n,
-                                                                      g.chat_col + s + nout, g.chat_val + s + nout);
+                                                                      oc + nout, ov + nout);
                         nout += U;
                         __syncthreads();
                     }
@@ -1459,10 +1464,10 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 w0 = wend;
             }
         }
-        // copy the merged row back into the head of its Ĉ bucket
+        // copy the merged row to its output (side buffer, or the head of its Ĉ bucket)
         for (int64_t p = threadIdx.x; p < nout; p += kLimThreads) {
-            g.chat_col[s + p] = st_col[p];
-            g.chat_val[s + p] = st_val[p];
+            oc[p] = st_col[p];
+            ov[p] = st_val[p];
         }
         if (threadIdx.x == 0) g.ccount[i] = nout;
         __syncthreads();

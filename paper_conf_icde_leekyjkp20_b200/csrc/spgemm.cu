@@ -13,6 +13,7 @@
 #include "analysis.cuh"
 #include "expand.cuh"
 #include "merge.cuh"
+#include "merge_units.cuh"
 #include "scan.cuh"
 
 using namespace spg;
@@ -158,6 +159,16 @@ struct spgemm_plan_s {
     int64_t *ccount = nullptr, *crowptr = nullptr;
     int32_t *fb_rows = nullptr;
     unsigned *fb_count = nullptr;
+    bool chat_external = false;
+    bool c_in_chat = false;        // C compact at the head of the Ĉ arrays (fused merge)    // Ĉ lives in the caller's C buffers (spgemm_execute, device C)
+    // merge units (merge_units.cuh): long rows merged into the side buffer, then one unit kernel
+    int64_t long_slots = 0;
+    int32_t *side_col = nullptr;
+    float *side_val = nullptr;
+    int64_t *side_off = nullptr;
+    int32_t *unit_row = nullptr;
+    int64_t *nunits = nullptr;
+    unsigned long long *unit_status = nullptr, *unit_ticket = nullptr;
     int64_t nnz_c = -1;
     int state = 0;  // 1 planned, 2 expanded, 3 merged
 };
@@ -237,16 +248,17 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     return SPGEMM_OK;
 }
 
+// merged rows go to the side buffer (long rows) when `side`, else in place
 template <int NW, int GROUPS, int EPT, int LS = 0>
 static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
-                             int ctas_per_sm, bool fallback_list = true) {
+                             int ctas_per_sm, bool fallback_list = true, bool side = false) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, LS>::kBytes * GROUPS;
     CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT, LS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
     LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT, LS><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
         rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0,
-        nullptr, nullptr, nullptr));
+        side ? p->side_off : nullptr, side ? p->side_col : nullptr, side ? p->side_val : nullptr));
     return SPGEMM_OK;
 }
 
@@ -589,9 +601,31 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
         TRY(palloc(p, &p->row_counter, 1, s));
     }
-    // Ĉ and merge state
-    TRY(palloc(p, &p->chat_col, p->chat_cap, s));
-    TRY(palloc(p, &p->chat_val, p->chat_cap, s));
+    // merge state; Ĉ itself is allocated by spgemm_expand (or is the caller's C, spgemm_execute)
+    const bool fused = p->opt.reserved[0] == kMergeFused;
+    p->long_slots = fused ? (int64_t)p->h_scal.long_slots : 0;
+    TRY(palloc(p, &p->side_col, p->long_slots, s));
+    TRY(palloc(p, &p->side_val, p->long_slots, s));
+    TRY(palloc(p, &p->side_off, M + 1, s));
+    TRY(palloc(p, &p->unit_row, M + 1, s));
+    TRY(palloc(p, &p->nunits, 1, s));
+    TRY(palloc(p, &p->unit_status, M + 1, s));
+    TRY(palloc(p, &p->unit_ticket, 18, s));
+    if (M > 0 && fused) {
+        Temp tf(s), tl(s), tu(s);
+        int32_t *flag;
+        int64_t *longcap, *uoff;
+        TRY(talloc(p, tf, &flag, M));
+        TRY(talloc(p, tl, &longcap, M));
+        TRY(talloc(p, tu, &uoff, M + 1));
+        LAUNCH("units", s, k_unit_flags<<<grid_for(M, 256), 256, 0, s>>>(p->rowoff, p->row_cls, M, kUnitThreads, flag,
+                                                                          longcap));
+        TRY(scan_excl(p, longcap, M, p->side_off, s, "units"));
+        TRY(scan_excl(p, flag, M, uoff, s, "units"));
+        LAUNCH("units", s, k_unit_rows<<<grid_for(M, 256), 256, 0, s>>>(flag, uoff, M, p->unit_row, p->nunits));
+    } else {
+        CK(cudaMemsetAsync(p->nunits, 0, 8, s));
+    }
     TRY(palloc(p, &p->ccount, M, s));
     TRY(palloc(p, &p->fb_rows, M, s));
     TRY(palloc(p, &p->fb_count, 1, s));
@@ -606,6 +640,10 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     cudaStream_t s = (cudaStream_t)stream;
     p->last_stream = s;
     CK(cudaSetDevice(p->dev));
+    if (!p->chat_col) {
+        TRY(palloc(p, &p->chat_col, p->chat_cap, s));
+        TRY(palloc(p, &p->chat_val, p->chat_cap, s));
+    }
     if (p->n_pieces_all > 0)
         LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * 8, kExpThreads, 0, s>>>(
             p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_prow, p->bp_col, p->bp_val, p->a_val,
@@ -614,13 +652,7 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     return SPGEMM_OK;
 }
 
-int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
-    if (!p) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan is NULL");
-    if (p->state < 2) return fail(SPGEMM_ERR_STATE, "spgemm_merge before spgemm_expand");
-    if (p->state >= 3) return fail(SPGEMM_ERR_STATE, "plan already merged (plans are single-use)");
-    cudaStream_t s = (cudaStream_t)stream;
-    p->last_stream = s;
-    CK(cudaSetDevice(p->dev));
+static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     const int64_t M = p->m;
     if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
     auto rows_of = [&](int b0, int b1, int64_t *cnt) {
@@ -693,6 +725,9 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         g.max_deg = p->lim_max_deg;
         g.stage_cap = p->stage_cap;
         g.row_counter = p->row_counter;
+        g.out_col = nullptr;   // merged in place
+        g.out_val = nullptr;
+        g.out_off = nullptr;
         g.skip_small = 1;
         g.coarse_cap = p->stage_cap;
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
@@ -702,6 +737,111 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
         LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
     }
     TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
+    return SPGEMM_OK;
+}
+
+static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
+    const int64_t M = p->m;
+    if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
+    auto rows_of = [&](int b0, int b1, int64_t *cnt) {
+        *cnt = p->row_starts[b1] - p->row_starts[b0];
+        return p->row_order + p->row_starts[b0];
+    };
+    int64_t cnt;
+    CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
+    // (a) long rows (padded bucket > kUnitRowMax, or B-Limited), merged into the side buffer:
+    //     <= 4096 slots by a 16-warp bucket-sort block per row; the limited rows B-Limited
+    const int32_t *rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+    TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_long4k", 4, true, true));
+    {   // rows whose buckets overflowed: natural merge sort (count read on the device)
+        constexpr int CAP = 4096;
+        const int smem = SortSmem<CAP>::kBytes;
+        CK(cudaFuncSetAttribute(k_merge_rows<8, 1, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
+            p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count, p->side_off,
+            p->side_col, p->side_val));
+    }
+    if (p->nlim > 0) {
+        CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
+        LimitedArgs g;
+        g.rows = p->row_order + p->row_starts[kRowBucketLim0];
+        g.nrows = p->nlim;
+        g.rowoff = p->rowoff;
+        g.rowwork = p->rowwork;
+        g.run_start = p->run_start;
+        g.run_base = p->run_base;
+        g.run_len = p->run_len;
+        g.chat_col = p->chat_col;
+        g.chat_val = p->chat_val;
+        g.ccount = p->ccount;
+        g.scratch_cursor = p->scr_cursor;
+        g.scratch_cnt = p->scr_cnt;
+        g.scratch_col = p->scr_col;
+        g.scratch_val = p->scr_val;
+        g.max_deg = p->lim_max_deg;
+        g.stage_cap = p->stage_cap;
+        g.row_counter = p->row_counter;
+        g.out_col = p->side_col;
+        g.out_val = p->side_val;
+        g.out_off = p->side_off;
+        g.skip_small = 1;
+        g.coarse_cap = p->stage_cap;
+        // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
+        // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
+        TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false, true));
+        CK(cudaFuncSetAttribute(k_merge_limited, cudaFuncAttributeMaxDynamicSharedMemorySize, kLimSmem));
+        LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
+    }
+    // (b) every unit of short rows (and the long rows' copies), in row order, straight into C
+    if (M > 0) {
+        CK(cudaMemsetAsync(p->unit_status, 0, (M + 1) * 8, s));
+        CK(cudaMemsetAsync(p->unit_ticket, 0, 18 * 8, s));
+        UnitArgs ua;
+        ua.unit_row = p->unit_row;
+        ua.nunits = p->nunits;
+        ua.rowoff = p->rowoff;
+        ua.rowwork = p->rowwork;
+        ua.rcls = p->row_cls;
+        ua.chat_col = p->chat_col;
+        ua.chat_val = p->chat_val;
+        ua.side_col = p->side_col;
+        ua.side_val = p->side_val;
+        ua.side_off = p->side_off;
+        ua.ccount = p->ccount;
+        ua.crowptr = p->crowptr;
+        ua.M = M;
+        ua.status = p->unit_status;
+        ua.ticket = p->unit_ticket;
+        ua.n_fallback = p->unit_ticket + 1;
+        ua.debug = p->opt.reserved[1];
+        ua.prof = p->unit_ticket + 2;
+        constexpr int smem = UnitSmem<kUnitThreads>::kBytes;
+        CK(cudaFuncSetAttribute(k_merge_units<kUnitThreads>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        int occ = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_merge_units<kUnitThreads>, kUnitThreads, smem));
+        LAUNCH("merge_units", s, k_merge_units<kUnitThreads><<<(unsigned)(p->num_sms * std::max(occ, 1)), kUnitThreads,
+                                                                 smem, s>>>(ua));
+        const int64_t nlong = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketSort4K];
+        if (nlong > 0)
+            LAUNCH("merge_copy_long", s, k_copy_long<<<grid_for(nlong, 1, (int64_t)p->num_sms * 8), kCopyThreads, 0, s>>>(
+                p->row_order + p->row_starts[kRowBucketSort4K], nlong, p->crowptr, p->ccount, p->side_off, p->side_col,
+                p->side_val, p->chat_col, p->chat_val));
+    } else {
+        CK(cudaMemsetAsync(p->crowptr, 0, 8, s));
+    }
+    return SPGEMM_OK;
+}
+
+int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
+    if (!p) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan is NULL");
+    if (p->state < 2) return fail(SPGEMM_ERR_STATE, "spgemm_merge before spgemm_expand");
+    if (p->state >= 3) return fail(SPGEMM_ERR_STATE, "plan already merged (plans are single-use)");
+    cudaStream_t s = (cudaStream_t)stream;
+    p->last_stream = s;
+    CK(cudaSetDevice(p->dev));
+    const int64_t M = p->m;
+    p->c_in_chat = p->opt.reserved[0] == kMergeFused;
+    TRY(p->c_in_chat ? merge_fused(p, s) : merge_bins(p, s));
     CK(cudaMemcpyAsync(&p->nnz_c, p->crowptr + M, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     p->state = 3;
@@ -720,6 +860,18 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
     C->ncols = p->n;
     C->nnz = p->nnz_c;
     const int64_t nnz = p->nnz_c;
+    if (p->c_in_chat) {
+        // fused merge: C is compact at the head of the Ĉ arrays (merge_units.cuh)
+        const cudaMemcpyKind kind = C->where == SPGEMM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+        CK(cudaMemcpyAsync(C->rowptr, p->crowptr, (p->m + 1) * 8, kind, s));
+        if (nnz > 0 && C->colidx != p->chat_col) {
+            CK(cudaMemcpyAsync(C->colidx, p->chat_col, nnz * 4, kind, s));
+            CK(cudaMemcpyAsync(C->val, p->chat_val, nnz * 4, kind, s));
+        }
+        if (C->where == SPGEMM_HOST) CK(cudaStreamSynchronize(s));
+        return SPGEMM_OK;
+    }
+    // per-bin merge: rows merged in place in their Ĉ buckets -> CSR compaction
     int32_t *dcol = C->colidx;
     float *dval = C->val;
     Temp t1(s), t2(s);
@@ -754,10 +906,26 @@ int spgemm_execute(spgemm_plan_t p, spgemm_alloc_fn alloc, void *ctx, int32_t ou
     if (!p || !alloc || !C) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan, alloc or C is NULL");
     if (out_where != SPGEMM_DEVICE && out_where != SPGEMM_HOST)
         return fail(SPGEMM_ERR_INVALID_ARGUMENT, "bad out_where");
+    if (p->state != 1) return fail(SPGEMM_ERR_STATE, "spgemm_execute needs a fresh plan");
+    C->where = out_where;
+    if (out_where == SPGEMM_DEVICE && p->opt.reserved[0] == kMergeFused) {
+        // device C: its column / value arrays (capacity nnz(Ĉ) slots) hold Ĉ during the merge and
+        // C at their head afterwards -- no copy, no second nnz(Ĉ)-sized buffer
+        C->rowptr = (int64_t *)alloc((size_t)(p->m + 1) * 8, out_where, ctx);
+        C->colidx = (int32_t *)alloc((size_t)std::max<int64_t>(p->chat_cap, 1) * 4, out_where, ctx);
+        C->val = (float *)alloc((size_t)std::max<int64_t>(p->chat_cap, 1) * 4, out_where, ctx);
+        if (!C->rowptr || !C->colidx || !C->val) return fail(SPGEMM_ERR_OUT_OF_MEMORY, "C allocation callback failed");
+        p->chat_col = C->colidx;
+        p->chat_val = C->val;
+        p->chat_external = true;
+        TRY(spgemm_expand(p, stream));
+        int64_t nnz;
+        TRY(spgemm_merge(p, stream, &nnz));
+        return spgemm_output(p, C, stream);
+    }
     TRY(spgemm_expand(p, stream));
     int64_t nnz;
     TRY(spgemm_merge(p, stream, &nnz));
-    C->where = out_where;
     C->rowptr = (int64_t *)alloc((size_t)(p->m + 1) * 8, out_where, ctx);
     C->colidx = (int32_t *)alloc((size_t)std::max<int64_t>(nnz, 1) * 4, out_where, ctx);
     C->val = (float *)alloc((size_t)std::max<int64_t>(nnz, 1) * 4, out_where, ctx);
@@ -793,6 +961,13 @@ int spgemm_get_stats(spgemm_plan_t p, spgemm_stats_t *st) {
     st->n_rows_bin[4] = p->row_starts[kRowBucketSort4K + 1] - p->row_starts[kRowBucketSort2K];
     st->n_rows_bin[5] = p->nlim;
     st->bytes_workspace = p->bytes;
+    st->n_units = st->n_units_fallback = -1;
+    if (p->state >= 3 && p->m > 0) {
+        unsigned long long t[2];
+        CK(cudaMemcpy(&st->n_units, p->nunits, 8, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(t, p->unit_ticket, 16, cudaMemcpyDeviceToHost));
+        st->n_units_fallback = (int64_t)t[1];
+    }
     return SPGEMM_OK;
 }
 
@@ -818,6 +993,9 @@ int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_
         case SPGEMM_VIEW_CROWPTR:
             if (p->state < 3) return fail(SPGEMM_ERR_STATE, "C row pointers exist after merge");
             src = p->crowptr; bytes = (p->m + 1) * 8; break;
+        case SPGEMM_VIEW_UNIT_PROFILE:
+            if (p->state < 3) return fail(SPGEMM_ERR_STATE, "the unit profile exists after merge");
+            src = p->unit_ticket + 2; bytes = 16 * 8; break;
         case SPGEMM_VIEW_GATHER: {
             const int64_t lo = p->pair_starts[kPairBucketGather0], hi = p->pair_starts[kPairBucketEmpty];
             src = p->pair_order + lo;

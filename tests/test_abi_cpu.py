@@ -34,7 +34,7 @@ def test_struct_layouts_match_header():
     assert ctypes.sizeof(spg.Options) == 144
     assert spg.Options.piece_work.offset == 32 and spg.Options.beta.offset == 48
     assert spg.Options.reserved.offset == 76
-    assert ctypes.sizeof(spg.Stats) == 29 * 8
+    assert ctypes.sizeof(spg.Stats) == 31 * 8
     o = spg.options()
     assert o.dom_waves == 16 and o.split_ca_max == 256 and o.piece_work == 16384
     assert o.split_b_tile == 4096 and o.limit_ctas_per_sm == 1 and o.validate == 1

@@ -66,8 +66,12 @@ def _deg(inp):
     return d
 
 
+FUSED = dict(reserved=(4,) + (0,) * 15)   # merge variant: fused unit merge + look-back output
+
 CASES = [
     ("C1", dict()),
+    ("C1", FUSED),
+    ("C1", dict(beta=10.0, **FUSED)),
     ("C1", dict(reserved=(1,) + (0,) * 15)),   # merge variant: register-staged counting sort
     ("C1", dict(reserved=(2,) + (0,) * 15)),   # merge variant: smem bucket sort everywhere
     ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: merge-path everywhere
@@ -129,8 +133,10 @@ def test_stage2_reorganizer(name, opts):
     assert st["t_lim"] == t_lim
     want_rows = stages.row_bins(rowwork, t_lim)
     got_rows = p.inspect(spg.VIEW_ROW_CLASS, np.int8)
-    single = (_deg(inp) == 1) & (rowwork > 0)
     cap = _caps(inp)
+    # single-run rows are already merged; short ones (padded bucket <= 2048, the unit kernel's
+    # row bound) are classed apart, long ones go through the long-row bins
+    single = (_deg(inp) == 1) & (rowwork > 0) & (cap <= 2048)
     # processing bins: the paper's limiting rows (B-Limiting) plus rows whose padded bucket
     # exceeds the non-limited kernels' capacity; the others by padded length
     lim = ((want_rows == stages.ROW_LIMITED) | (cap > 4096)) & ~single & (rowwork > 0)
@@ -208,7 +214,8 @@ def test_random_tiny(shape, dens, seed, skew, values):
     inp = synth.random_tiny(*shape, dens[0], dens[1], seed, values=values, skew=skew)
     A, B = spg.from_inputs(inp, "cuda")
     for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(1,) + (0,) * 15),
-                 dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15)):
+                 dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15), FUSED,
+                 dict(beta=1000.0, piece_work=64, split_ca_max=3, **FUSED)):
         C = spg.matmul(A, B, **opts)
         assert_c_matches(C, inp, signed=(values == "signed"))
 
@@ -245,16 +252,22 @@ def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False)
     (16, 100, 30000, 0.3, 2000, False, False),     # dense rows: fp64 column windows
     (2, 10000, 1000000, 1.0, 21, True, False),     # column 0 in 10000 runs: single-column overflow
 ])
-def test_limited_paths(m, k, n, dens, run_len, hub, narrow):
+@pytest.mark.parametrize("fused", [False, True])
+def test_limited_paths(m, k, n, dens, run_len, hub, narrow, fused):
     """B-Limited merge: rows longer than the non-limited capacity, through every sub-path."""
     inp = _wide_inputs(m, k, n, dens, run_len, 3, hub_col=hub, narrow=narrow)
     A, B = spg.from_inputs(inp, "cuda")
-    with spg.Plan(A, B) as p:
+    with spg.Plan(A, B, **(FUSED if fused else {})) as p:
         st = p.stats()
         assert st["n_rows_bin"][5] > 0
         p.expand()
         p.merge()
         C = p.output()
+    assert_c_matches(C, inp)
+    with spg.Plan(A, B, **(FUSED if fused else {})) as p:   # staged path with host output
+        p.expand()
+        p.merge()
+        C = p.output(device="cpu")
     assert_c_matches(C, inp)
 
 
@@ -277,6 +290,11 @@ def test_clustered_columns_fallback(k, cluster, spread):
                          (br, bc, synth.edge_values(br, bc, 2)))
     A, B = spg.from_inputs(inp, "cuda")
     C = spg.matmul(A, B)
+    assert_c_matches(C, inp)
+    with spg.Plan(A, B, **FUSED) as p:
+        C = p.execute()
+        if k * (cluster + spread) <= 2048:           # short rows: the unit merge's fallback ran
+            assert p.stats()["n_units_fallback"] > 0
     assert_c_matches(C, inp)
 
 
@@ -331,13 +349,13 @@ def test_validation_rejects_malformed():
 
 
 # ------------------------------------------------------------------ full sizes -------------
-@pytest.mark.parametrize("name", ["C2"])
-def test_full_size_sampled(name):
+@pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", FUSED)])
+def test_full_size_sampled(name, opts):
     """BASELINE.json configs[1] at full size, in the bench's launch configuration: sampled rows
     compared with the oracle one by one, plus whole-matrix properties."""
     inp = synth.make_inputs(name, seed=1)
     A, B = spg.from_inputs(inp, "cuda")
-    with spg.Plan(A, B) as p:
+    with spg.Plan(A, B, **opts) as p:
         st = p.stats()
         C = p.execute()
     ca, rb, work = stages.pair_workload(inp)
