@@ -29,6 +29,7 @@ namespace spg {
 constexpr int kExpThreads = 256;
 constexpr int kExpTile = 2048;   // units (16-byte vectors) per tile
 constexpr int kExpUnroll = 4;
+constexpr int kExpCtasPerSM = 3;   // 80 registers: 3 x 256 threads resident per SM, one persistent wave
 
 // vectors of one run written by a block: the B sub-row rounded up to 4 slots (B tiles start on
 // 4-slot boundaries, so the last tile of a row also writes the run's sentinel padding)

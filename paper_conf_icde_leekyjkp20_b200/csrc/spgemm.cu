@@ -645,7 +645,7 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
         TRY(palloc(p, &p->chat_val, p->chat_cap, s));
     }
     if (p->n_pieces_all > 0)
-        LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * 8, kExpThreads, 0, s>>>(
+        LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
             p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_prow, p->bp_col, p->bp_val, p->a_val,
             p->base, p->chat_col, p->chat_val));
     p->state = 2;

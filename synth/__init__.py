@@ -64,7 +64,9 @@ def edge_values(rows: np.ndarray, cols: np.ndarray, seed: int, kind: str = "real
 
 
 def _dedupe(src: np.ndarray, dst: np.ndarray, ncols: int):
-    key = np.unique(src.astype(np.int64) * np.int64(ncols) + dst.astype(np.int64))
+    key = np.sort(src.astype(np.int64) * np.int64(ncols) + dst.astype(np.int64))   # == np.unique, without
+    if key.size > 1:                                                             # its slow hash path
+        key = key[np.concatenate([[True], key[1:] != key[:-1]])]
     return (key // ncols).astype(np.int32), (key % ncols).astype(np.int32)
 
 
