@@ -256,9 +256,20 @@ def main():
     top = max(gms, key=lambda g: gms[g])
     top_bytes = groups[top][1]
     achieved = top_bytes / (gms[top] / 1e3) / 1e9 if gms[top] > 0 else 0.0
+    # DRAM bytes of the same kernel group per step, from the committed ncu --set full capture
+    # (scripts/ncu_traffic.py); null when no capture of this config exists
+    traffic, traffic_src = None, None
+    tpath = os.path.join(ROOT, "profiles", f"r1_traffic_{args.config}.json")
+    if os.path.exists(tpath) and ws == 1:
+        try:
+            tj = json.load(open(tpath))
+            traffic = tj["groups"][top]["dram_bytes"]
+            traffic_src = os.path.relpath(tpath, ROOT) + " <- " + tj["report"]
+        except (KeyError, ValueError):
+            pass
     roofline = {"bound": "hbm", "kernel": top, "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
-                "frac": round(achieved / hbm, 4), "traffic": None, "peak_source": peak_src,
-                "ms": round(gms[top], 4), "algorithmic_bytes": int(top_bytes)}
+                "frac": round(achieved / hbm, 4), "traffic": traffic, "traffic_src": traffic_src,
+                "peak_source": peak_src, "ms": round(gms[top], 4), "algorithmic_bytes": int(top_bytes)}
     step_bw = bytes_step / (ms_per_step / 1e3) / 1e9
     breakdown = {nm: round(v, 4) for nm, v in sorted(k_ms.items(), key=lambda x: -x[1])}
 

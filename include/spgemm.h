@@ -106,7 +106,9 @@ typedef struct {
     double beta;              /* >0: limiting threshold min(cap, nnz(Ĉ)/(#rows × β)) (L475-L477 L);
                                  0: B200 default = non-limited merge capacity (4096)            */
     int32_t limit_ctas_per_sm;/* B-Limiting: resident limited-merge blocks per SM (default 1)   */
-    int32_t enable_split;     /* ablation switches (Fig. 10): 0 disables the technique          */
+    int32_t enable_split;     /* ablation switches (Fig. 10): 0 disables the technique; for
+                                 enable_limit = 0 the β threshold is ignored and only rows above
+                                 the non-limited kernels' capacity take the long-row kernels     */
     int32_t enable_gather;
     int32_t enable_limit;
     int32_t validate;         /* check input structure in spgemm_plan (default 1)               */

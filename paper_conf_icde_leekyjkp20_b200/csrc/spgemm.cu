@@ -478,7 +478,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         p->t_dom = std::min<int64_t>(o.piece_work, std::max<int64_t>(o.dom_min_work,
                                                                      cdiv(p->nnz_chat, (int64_t)p->num_sms * o.dom_waves)));
     const int64_t cap = 4096;
-    if (o.beta > 0)
+    if (o.beta > 0 && o.enable_limit)   // enable_limit = 0 (ablation): no Limiting rows by the paper's
         p->t_lim = std::min<int64_t>(cap, (int64_t)std::floor((double)p->nnz_chat /
                                                              ((double)std::max<uint64_t>(p->h_scal.m_nonempty, 1) * o.beta)));
     else

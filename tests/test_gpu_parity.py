@@ -80,6 +80,7 @@ CASES = [
     ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
     ("C1", dict(alpha=2.0)),
     ("C1", dict(beta=10.0)),
+    ("C1", dict(beta=10.0, enable_limit=0)),
 ]
 
 
@@ -129,7 +130,9 @@ def test_stage2_reorganizer(name, opts):
                                       np.concatenate([lists[b] for b in range(6)]))
         assert st["n_gather_bin"] == [len(lists[b]) for b in range(6)]
     rowwork = stages.row_workload(inp)
-    t_lim = stages.limiting_threshold(int(work.sum()), int((rowwork > 0).sum()), o.beta, 4096)
+    # enable_limit = 0 (Fig. 10 ablation): no Limiting rows by the β threshold
+    t_lim = stages.limiting_threshold(int(work.sum()), int((rowwork > 0).sum()), o.beta if o.enable_limit else 0.0,
+                                      4096)
     assert st["t_lim"] == t_lim
     want_rows = stages.row_bins(rowwork, t_lim)
     got_rows = p.inspect(spg.VIEW_ROW_CLASS, np.int8)
