@@ -78,67 +78,106 @@ __global__ void k_tile_first_piece(const int64_t *__restrict__ uoff, int64_t npi
     }
 }
 
+// r / nv for r < 2^22 in fp32 with an exact fix-up (else the 64-bit division)
+__device__ __forceinline__ int64_t div_units(int64_t r, int nv) {
+    if (r < (1 << 22)) {
+        const int ri = (int)r;
+        int ai = __float2int_rz(((float)ri + 0.5f) / (float)nv);
+        ai -= (ai * nv > ri);
+        ai += ((ai + 1) * nv <= ri);
+        return ai;
+    }
+    return r / nv;   // (huge unsplit blocks: enable_split = 0)
+}
+
+// Pieces overlapping one tile are staged in shared memory (unit offset, A start, B' source,
+// vectors per run, B offset), so a unit's only global loads are its A value / run base and its
+// B' vector -- all independent, one memory round trip -- followed by the two 16-byte stores.
+// A tile overlapping more than kExpPieceCache blocks (only gathered 1-unit blocks can do that)
+// searches the block list in global memory instead.
+constexpr int kExpPieceCache = 1024;
+
 __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     const Piece *__restrict__ pieces, const int64_t *__restrict__ uoff, int64_t npieces,
     const int64_t *__restrict__ tile_p0, const int64_t *__restrict__ b_prow, const int32_t *__restrict__ bp_col,
     const float *__restrict__ bp_val, const float *__restrict__ a_val, const int64_t *__restrict__ base,
     int32_t *__restrict__ chat_col, float *__restrict__ chat_val) {
+    __shared__ int64_t s_uoff[kExpPieceCache + 1];
+    __shared__ int64_t s_alo[kExpPieceCache];
+    __shared__ int64_t s_bsrc[kExpPieceCache];
+    __shared__ int32_t s_nv[kExpPieceCache];
+    __shared__ int32_t s_boff[kExpPieceCache];
     const int64_t total = uoff[npieces];
     const int64_t ntiles = (total + kExpTile - 1) / kExpTile;
     for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
         const int64_t f0 = tile * kExpTile, f1 = min(total, f0 + kExpTile);
         const int64_t p0 = tile_p0[tile];
         const int64_t pend = tile_p0[tile + 1] + 1;   // blocks [p0, pend) overlap the tile
-        // kExpUnroll units per thread per step, their loads issued together (memory-level
-        // parallelism: each unit is a short chain block -> A entry -> B vector -> store)
-        int64_t pj = p0;
+        const int np = (int)min(pend - p0, (int64_t)kExpPieceCache + 1);
+        const bool cached = np <= kExpPieceCache;
+        __syncthreads();                               // previous tile's readers are done
+        if (cached) {
+            for (int q = threadIdx.x; q < np; q += kExpThreads) {
+                const Piece pc = pieces[p0 + q];
+                s_uoff[q] = uoff[p0 + q];
+                s_alo[q] = pc.a_lo;
+                s_bsrc[q] = b_prow[pc.k] + pc.b_off;
+                s_nv[q] = piece_nvec(pc);
+                s_boff[q] = pc.b_off;
+            }
+            if (threadIdx.x == 0) s_uoff[np] = INT64_MAX;
+        }
+        __syncthreads();
+        // kExpUnroll units per thread per step, their loads issued together
+        int pj = 0;             // cached: local block index (never decreases)
+        int64_t gj = p0;        // uncached: global block index
         for (int64_t fb = f0 + threadIdx.x; fb < f1; fb += kExpUnroll * kExpThreads) {
-            int64_t dst[kExpUnroll], src[kExpUnroll];
+            int64_t dst[kExpUnroll];
             float av[kExpUnroll];
+            int4 c4[kExpUnroll];
+            float4 w4[kExpUnroll];
             bool ok[kExpUnroll];
 #pragma unroll
             for (int u = 0; u < kExpUnroll; ++u) {
                 const int64_t f = fb + u * kExpThreads;
                 ok[u] = f < f1;
                 if (!ok[u]) continue;
-                int64_t hi = pend;                 // last block with uoff <= f (never decreases)
-                while (hi - pj > 1) {
-                    const int64_t mid = (pj + hi) >> 1;
-                    if (__ldg(uoff + mid) <= f) pj = mid; else hi = mid;
+                int64_t alo, bsrc, uo;
+                int nv, boff;
+                if (cached) {
+                    int hi = np;                   // last block with s_uoff <= f
+                    while (hi - pj > 1) {
+                        const int mid = (pj + hi) >> 1;
+                        if (s_uoff[mid] <= f) pj = mid; else hi = mid;
+                    }
+                    uo = s_uoff[pj]; alo = s_alo[pj]; bsrc = s_bsrc[pj]; nv = s_nv[pj]; boff = s_boff[pj];
+                } else {
+                    int64_t hi = pend;
+                    while (hi - gj > 1) {
+                        const int64_t mid = (gj + hi) >> 1;
+                        if (__ldg(uoff + mid) <= f) gj = mid; else hi = mid;
+                    }
+                    const Piece pc = pieces[gj];
+                    uo = __ldg(uoff + gj); alo = pc.a_lo; bsrc = __ldg(b_prow + pc.k) + pc.b_off;
+                    nv = piece_nvec(pc); boff = pc.b_off;
                 }
-                const Piece pc = pieces[pj];
-                const int nv = piece_nvec(pc);
-                const int64_t r = f - __ldg(uoff + pj);
-                int64_t a;
-                if (r < (1 << 22)) {               // r / nv in fp32, then an exact fix-up
-                    const int ri = (int)r;
-                    int ai = __float2int_rz(((float)ri + 0.5f) / (float)nv);
-                    ai -= (ai * nv > ri);
-                    ai += ((ai + 1) * nv <= ri);
-                    a = ai;
-                } else {                           // (huge unsplit blocks: enable_split = 0)
-                    a = r / nv;
-                }
+                const int64_t r = f - uo;
+                const int64_t a = div_units(r, nv);
                 const int v = (int)(r - a * nv);
-                const int64_t e = pc.a_lo + a;
+                const int64_t e = alo + a;
                 av[u] = __ldg(a_val + e);
-                dst[u] = __ldg(base + e) + pc.b_off + 4 * v;
-                src[u] = __ldg(b_prow + pc.k) + pc.b_off + 4 * v;
+                dst[u] = __ldg(base + e) + boff + 4 * v;
+                c4[u] = __ldg(reinterpret_cast<const int4 *>(bp_col + bsrc + 4 * v));
+                w4[u] = __ldg(reinterpret_cast<const float4 *>(bp_val + bsrc + 4 * v));
             }
-            int4 c4[kExpUnroll];
-            float4 w4[kExpUnroll];
 #pragma unroll
             for (int u = 0; u < kExpUnroll; ++u)
                 if (ok[u]) {
-                    c4[u] = __ldg(reinterpret_cast<const int4 *>(bp_col + src[u]));
-                    w4[u] = __ldg(reinterpret_cast<const float4 *>(bp_val + src[u]));
-                }
-#pragma unroll
-            for (int u = 0; u < kExpUnroll; ++u)
-                if (ok[u]) {
-                    *reinterpret_cast<int4 *>(chat_col + dst[u]) = c4[u];
-                    *reinterpret_cast<float4 *>(chat_val + dst[u]) =
-                        make_float4(av[u] * w4[u].x, av[u] * w4[u].y, av[u] * w4[u].z, av[u] * w4[u].w);
+                    // streaming (evict-first) stores: Ĉ is written once and read by the merge much
+                    // later, so it should not push B' (re-read by every A entry of k) out of L2
+                    __stcs(reinterpret_cast<int4 *>(chat_col + dst[u]), c4[u]);
+                    __stcs(reinterpret_cast<float4 *>(chat_val + dst[u]),
+                           make_float4(av[u] * w4[u].x, av[u] * w4[u].y, av[u] * w4[u].z, av[u] * w4[u].w));
                 }
         }
     }

@@ -1069,11 +1069,14 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
 //     merge-sorted.
 // The merged output of the two windowed paths is staged in the block's global scratch and
 // copied to the head of the row's bucket after the whole row has been read.
+// (measured: 256 threads / 3584 slots at 2 blocks per SM made C3's long rows 8.6x slower -- bins
+// of the coarse partition overflow the smaller sorter and fall back to the window search)
 constexpr int kLimThreads = 512;
-constexpr int kLimNW = kLimThreads / 32;
-constexpr int kLimCap = 9216;
-constexpr int kLimEPT = kLimCap / kLimThreads;   // 18
+constexpr int kLimCap = 9216;                     // 1 limited block per SM (B-Limiting)
 constexpr int kLimWindow = 16384;
+constexpr int kLimNW = kLimThreads / 32;
+constexpr int kLimEPT = kLimCap / kLimThreads;
+constexpr int kLimBucketCap = 9216;               // rows up to this were merged by the bucket launch
 constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
 constexpr int kLimSortBytes = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
                                     kLimCap * 16 + (hidx(ceil_pow2(kLimCap)) + 4) * 4,  // bucket sort
@@ -1081,6 +1084,7 @@ constexpr int kLimSortBytes = cmax3(SortSmem<kLimCap>::kBytes,                 /
 constexpr int kCoarseLog = 10;
 constexpr int kCoarseBins = 1 << kCoarseLog;
 constexpr int kLimSmem = kLimSortBytes + (3 * kCoarseBins + 1) * 4;           // + coarse partition tables
+constexpr int kLimCtasPerSM = 228 * 1024 / (kLimSmem + 1024);   // B-Limiting: limited blocks resident per SM
 
 struct LimitedArgs {
     const int32_t *rows;          // limited rows, longest first
@@ -1149,7 +1153,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t s = g.rowoff[i];
         const int64_t cap = g.rowoff[i + 1] - s;   // padded bucket length
         const int64_t L = g.rowwork[i];             // products
-        if (cap <= kLimCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
+        if (cap <= kLimBucketCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
         int32_t *const oc = g.out_col ? g.out_col + g.out_off[i] : g.chat_col + s;
         float *const ov = g.out_col ? g.out_val + g.out_off[i] : g.chat_val + s;
         if (cap <= kLimCap) {
