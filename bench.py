@@ -141,10 +141,15 @@ def main():
     from paper_conf_icde_leekyjkp20_b200.build import build_library
     if rank == 0:
         build_library()
+    if os.environ.get("SPGEMM_BENCH_SHARE_GPU"):   # test mode: N ranks share the visible GPUs (gloo)
+        local = local % torch.cuda.device_count()
     if ws > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if os.environ.get("SPGEMM_BENCH_SHARE_GPU"):
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         dist.barrier()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
