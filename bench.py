@@ -204,7 +204,7 @@ def main():
         p = spg.Plan(A, B, stream=stream, **opts)
         C = p.execute()
         st = p.stats()
-        if os.environ.get("SPGEMM_RESERVED", "").find("1=2") >= 0:
+        if "1=2" in os.environ.get("SPGEMM_RESERVED", "") or "1=3" in os.environ.get("SPGEMM_RESERVED", ""):
             prof = p.inspect(spg.VIEW_UNIT_PROFILE, np.uint64)
             print("unit-profile", json.dumps([int(x) for x in prof]), file=sys.stderr)
         p.destroy()

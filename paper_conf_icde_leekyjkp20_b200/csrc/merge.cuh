@@ -1071,9 +1071,11 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
 // copied to the head of the row's bucket after the whole row has been read.
 // (measured: 256 threads / 3584 slots at 2 blocks per SM made C3's long rows 8.6x slower -- bins
 // of the coarse partition overflow the smaller sorter and fall back to the window search)
-constexpr int kLimThreads = 512;
+constexpr int kLimThreads = 1024;
 constexpr int kLimCap = 9216;                     // 1 limited block per SM (B-Limiting)
-constexpr int kLimWindow = 16384;
+constexpr int kLimWinLog = 14;
+constexpr int kLimWindow = 1 << kLimWinLog;
+constexpr int kLimWords = kLimWindow / 32;         // touched-column bitmap words of a window
 constexpr int kLimNW = kLimThreads / 32;
 constexpr int kLimEPT = kLimCap / kLimThreads;
 constexpr int kLimBucketCap = 9216;               // rows up to this were merged by the bucket launch
@@ -1108,6 +1110,7 @@ struct LimitedArgs {
     float *out_val;
     const int64_t *out_off;
     int skip_small;
+    unsigned long long *prof;     // NULL, or per-path clock totals [0..10) (tuning)
     int64_t coarse_cap;           // rows up to this many slots take the coarse-partition path
 };
 
@@ -1153,6 +1156,15 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t s = g.rowoff[i];
         const int64_t cap = g.rowoff[i + 1] - s;   // padded bucket length
         const int64_t L = g.rowwork[i];             // products
+        const long long t_row = clock64();
+        auto rec = [&](int path) {   // options.reserved[1] = 3: per-path row clocks (tuning)
+            if (g.prof && threadIdx.x == 0) {
+                const unsigned long long dt = (unsigned long long)(clock64() - t_row);
+                atomicAdd(g.prof + path, dt);
+                atomicAdd(g.prof + 5 + path, 1ull);
+                atomicMax(g.prof + 4, dt);
+            }
+        };
         if (cap <= kLimBucketCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
         int32_t *const oc = g.out_col ? g.out_col + g.out_off[i] : g.chat_col + s;
         float *const ov = g.out_col ? g.out_val + g.out_off[i] : g.chat_val + s;
@@ -1169,6 +1181,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                                                           oc, ov);
             if (threadIdx.x == 0) g.ccount[i] = U;
             __syncthreads();
+            rec(0);
             continue;
         }
         const int64_t rs = g.run_start[r];
@@ -1188,6 +1201,117 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t nwin_dense = (span + kLimWindow - 1) / kLimWindow;
         const bool dense = L * 4 >= span && (int64_t)R * nwin_dense <= 2 * L;
         int64_t nout = 0;
+        const int64_t nwin_pow = (span + kLimWindow - 1) >> kLimWinLog;
+        if (dense && cap <= g.stage_cap && nwin_pow <= kCoarseBins) {
+            // dense row, streamed: (1) histogram of the row's column windows (2^kLimWinLog columns),
+            // (2) scatter into the block's scratch grouped by window, (3) per window, coalesced
+            // sweep of its products into the fp64 shared accumulator + touched bits, extracted in
+            // column order straight to the row's output (the row now lives in scratch).  Every
+            // load is independent (the per-run cursor walk below is one dependent load per run
+            // per window: C3's hub rows, 38K runs x 104 windows, took 250 ms in one block).
+            const int nwin = (int)nwin_pow;
+            int *fh = (int *)(smem_raw + kLimSortBytes);       // [kCoarseBins] counts -> starts
+            int *wst = fh + kCoarseBins;                        // [kCoarseBins + 1]
+            int *wcur = wst + kCoarseBins + 1;                  // [kCoarseBins]
+            int32_t *sc_col = g.scratch_col + (int64_t)blockIdx.x * g.stage_cap;
+            float *sc_val = g.scratch_val + (int64_t)blockIdx.x * g.stage_cap;
+            for (int t = threadIdx.x; t < kCoarseBins; t += kLimThreads) fh[t] = 0;
+            __syncthreads();
+            for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+                const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
+                const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> kLimWinLog;
+                    const unsigned peers = __match_any_sync(__activemask(), wid);
+                    if (wid >= 0 && lane_id() == __ffs(peers) - 1) atomicAdd(&fh[wid], __popc(peers));
+                }
+            }
+            __syncthreads();
+            {
+                constexpr int BPT = kCoarseBins / kLimThreads;
+                int c[BPT], cnt = 0;
+#pragma unroll
+                for (int u = 0; u < BPT; ++u) { c[u] = fh[threadIdx.x * BPT + u]; cnt += c[u]; }
+                int tot;
+                int ex = grp.excl_sum(cnt, sc, &tot);
+#pragma unroll
+                for (int u = 0; u < BPT; ++u) {
+                    wst[threadIdx.x * BPT + u] = ex;
+                    wcur[threadIdx.x * BPT + u] = ex;
+                    ex += c[u];
+                }
+                if (threadIdx.x == 0) wst[kCoarseBins] = tot;
+            }
+            __syncthreads();
+            for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+                const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
+                const float4 v4 = *reinterpret_cast<const float4 *>(g.chat_val + s + 4 * p);
+                const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
+                const float vv[4] = {v4.x, v4.y, v4.z, v4.w};
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {     // warp-aggregated cursor bumps per window
+                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> kLimWinLog;
+                    const unsigned peers = __match_any_sync(__activemask(), wid);
+                    if (wid >= 0) {
+                        const int leader = __ffs(peers) - 1;
+                        int q0 = 0;
+                        if (lane_id() == leader) q0 = atomicAdd(&wcur[wid], __popc(peers));
+                        q0 = __shfl_sync(peers, q0, leader);
+                        const int q = q0 + __popc(peers & lanemask_lt());
+                        sc_col[q] = cc[u];
+                        sc_val[q] = vv[u];
+                    }
+                }
+            }
+            double *acc = (double *)smem_raw;
+            uint32_t *bits = (uint32_t *)(smem_raw + kLimWindow * 8);
+            for (int t = threadIdx.x; t < kLimWindow; t += kLimThreads) acc[t] = 0.0;
+            for (int t = threadIdx.x; t < kLimWindow / 32; t += kLimThreads) bits[t] = 0u;
+            __syncthreads();
+            for (int wi = 0; wi < nwin; ++wi) {
+                const int q0 = wst[wi], q1 = wst[wi + 1];
+                if (q0 == q1) continue;
+                const int32_t wbase = mn + (wi << kLimWinLog);
+                for (int q = q0 + threadIdx.x; q < q1; q += kLimThreads) {
+                    const int x = sc_col[q] - wbase;
+                    smem_add_f64(acc + x, (double)sc_val[q]);
+                    atomicOr(bits + (x >> 5), 1u << (x & 31));
+                }
+                __syncthreads();
+                constexpr int WPT = kLimWords >= kLimThreads ? kLimWords / kLimThreads : 1;
+                const bool own = threadIdx.x * WPT < kLimWords;   // threads past the bitmap: no words
+                int cntw = 0;
+                uint32_t word[WPT];
+#pragma unroll
+                for (int u = 0; u < WPT; ++u) {
+                    word[u] = own ? bits[threadIdx.x * WPT + u] : 0u;
+                    cntw += __popc(word[u]);
+                }
+                int tot;
+                int64_t pos = nout + grp.excl_sum(cntw, sc, &tot);
+#pragma unroll
+                for (int u = 0; u < WPT; ++u) {
+                    uint32_t m = word[u];
+                    while (m) {
+                        const int bpos = __ffs(m) - 1;
+                        m &= m - 1;
+                        const int x = (threadIdx.x * WPT + u) * 32 + bpos;
+                        oc[pos] = wbase + x;
+                        ov[pos] = (float)acc[x];
+                        acc[x] = 0.0;
+                        ++pos;
+                    }
+                    if (own) bits[threadIdx.x * WPT + u] = 0u;
+                }
+                nout += tot;
+                __syncthreads();
+            }
+            if (threadIdx.x == 0) g.ccount[i] = nout;
+            __syncthreads();
+            rec(2);
+            continue;
+        }
         if (dense) {
             double *acc = (double *)smem_raw;
             uint32_t *bits = (uint32_t *)(smem_raw + kLimWindow * 8);
@@ -1196,42 +1320,36 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
             __syncthreads();
             for (int64_t w0 = mn; w0 <= mx; w0 += kLimWindow) {
                 const int32_t wend = (int32_t)min((int64_t)mx + 1, w0 + kLimWindow);
-                for (int q = w; q < R; q += kLimNW) {       // warp per run, 128 products per step
+                // warp per run, 32 products per step: a run contributes L / (R * #windows) < 2
+                // products to a window on average, so a wider probe mostly loads entries of later
+                // windows (measured: 4 vectors per lane made C3's densest rows 4x slower)
+                for (int q = w; q < R; q += kLimNW) {
                     const int64_t b = rbase[q];
                     const int len = rlen[q];
                     int cur = cursor[q];
                     while (cur < len) {
-                        int32_t c[4];
-                        float v[4];
-#pragma unroll
-                        for (int u = 0; u < 4; ++u) {
-                            const int p = cur + u * 32 + lane;
-                            c[u] = p < len ? g.chat_col[b + p] : kKeyPad;
-                            v[u] = p < len ? g.chat_val[b + p] : 0.f;
+                        const int p = cur + lane;
+                        const int32_t c = p < len ? g.chat_col[b + p] : kKeyPad;
+                        const bool in = c < wend;
+                        if (in) {
+                            const int x = c - (int32_t)w0;
+                            smem_add_f64(acc + x, (double)g.chat_val[b + p]);
+                            atomicOr(bits + (x >> 5), 1u << (x & 31));
                         }
-                        int taken = 0;
-#pragma unroll
-                        for (int u = 0; u < 4; ++u) {
-                            const bool in = c[u] < wend;
-                            if (in) {
-                                const int x = c[u] - (int32_t)w0;
-                                smem_add_f64(acc + x, (double)v[u]);
-                                atomicOr(bits + (x >> 5), 1u << (x & 31));
-                            }
-                            taken += __popc(__ballot_sync(kFull, in));
-                        }
+                        const int taken = __popc(__ballot_sync(kFull, in));
                         cur += taken;
-                        if (taken < 128) break;
+                        if (taken < 32) break;
                     }
                     if (lane == 0) cursor[q] = cur;
                 }
                 __syncthreads();
-                constexpr int WPT = (kLimWindow / 32) / kLimThreads;
+                constexpr int WPT = kLimWords >= kLimThreads ? kLimWords / kLimThreads : 1;
+                const bool own = threadIdx.x * WPT < kLimWords;   // threads past the bitmap: no words
                 int cntw = 0;
                 uint32_t word[WPT];
 #pragma unroll
                 for (int u = 0; u < WPT; ++u) {
-                    word[u] = bits[threadIdx.x * WPT + u];
+                    word[u] = own ? bits[threadIdx.x * WPT + u] : 0u;
                     cntw += __popc(word[u]);
                 }
                 int tot;
@@ -1248,7 +1366,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                         acc[x] = 0.0;
                         ++pos;
                     }
-                    bits[threadIdx.x * WPT + u] = 0u;
+                    if (own) bits[threadIdx.x * WPT + u] = 0u;
                 }
                 nout += tot;
                 __syncthreads();
@@ -1366,7 +1484,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 __syncthreads();
             }
-            if (done_coarse) continue;
+            if (done_coarse) { rec(1); continue; }
             // sparse: windows whose products fit the smem sorter
             int32_t *k0 = (int32_t *)smem_raw;
             float *v0 = (float *)(smem_raw + kLimCap * 4);
@@ -1475,6 +1593,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         }
         if (threadIdx.x == 0) g.ccount[i] = nout;
         __syncthreads();
+        rec(dense ? 2 : 3);
     }
 }
 

@@ -593,7 +593,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
             p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->base, p->lim_index, p->run_start, p->run_fill,
             p->run_base, p->run_len));
         p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
-        p->stage_cap = std::min<int64_t>(p->lim_max_L, p->n);
+        p->stage_cap = p->lim_max_L;   // whole-row scratch (dense rows are regrouped by window)
         TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
         TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
         p->lim_max_deg += 1;   // per-block stride of the cursor / cnt scratch (cnt holds R+1 offsets)
@@ -729,7 +729,9 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         g.out_val = nullptr;
         g.out_off = nullptr;
         g.skip_small = 1;
-        g.coarse_cap = p->stage_cap;
+        g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
+        if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
+        g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
@@ -785,7 +787,9 @@ static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
         g.out_val = p->side_val;
         g.out_off = p->side_off;
         g.skip_small = 1;
-        g.coarse_cap = p->stage_cap;
+        g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
+        if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
+        g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false, true));

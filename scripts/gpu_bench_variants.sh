@@ -3,7 +3,7 @@ cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 for v in "$@"; do
-  SPGEMM_RESERVED="$v" timeout 600 python bench.py --steps 3 --warmup 2 --no-e2e --no-cpu-baseline > gpurun_out/bench_v.log 2>&1
+  SPGEMM_RESERVED="$v" timeout 900 python bench.py --config ${CFG:-C2} --steps 3 --warmup 2 --no-e2e --no-cpu-baseline > gpurun_out/bench_v.log 2>&1
   echo "== [$v] exit $?"
   python - <<'PY'
 import json
