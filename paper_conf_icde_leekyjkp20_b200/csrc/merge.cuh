@@ -1735,4 +1735,96 @@ __global__ void __launch_bounds__(kCompactLongThreads) k_compact_long(const int3
     }
 }
 
+// Load-balanced compaction: the output is cut into chunks of kCmpChunk entries (a chunk may
+// hold part of one long row or many short rows); chunk_r0[c] = row of the chunk's first entry.
+// A thread writes aligned 16-byte output vectors; each of its 4 entries is read from its row's
+// bucket head (src = rowoff[r] + (q - crowptr[r]); 4 scalar loads, coalesced across the warp).
+// Every row length gets the same per-entry cost (C3's 60K-entry rows made the warp / CTA per
+// row copy 2.4 TB/s).
+constexpr int kCmpChunk = 8192;
+constexpr int kCmpThreads = 256;
+
+__global__ void k_chunk_first_row(const int64_t *__restrict__ crowptr, int64_t M, int64_t nnz, int64_t nchunks,
+                                  int32_t *__restrict__ chunk_r0) {
+    for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c <= nchunks; c += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t q = min(c * (int64_t)kCmpChunk, nnz - 1);
+        int64_t lo = 0, hi = M;               // last row r with crowptr[r] <= q (a non-empty row)
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (crowptr[mid] <= q) lo = mid; else hi = mid;
+        }
+        chunk_r0[c] = (int32_t)lo;
+    }
+}
+
+__global__ void __launch_bounds__(kCmpThreads) k_compact_flat(const int64_t *__restrict__ crowptr,
+                                                               const int64_t *__restrict__ rowoff,
+                                                               const int32_t *__restrict__ chunk_r0, int64_t nnz,
+                                                               int64_t nchunks, const int32_t *__restrict__ chat_col,
+                                                               const float *__restrict__ chat_val,
+                                                               int32_t *__restrict__ out_col,
+                                                               float *__restrict__ out_val) {
+    for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
+        const int64_t q0 = c * (int64_t)kCmpChunk, q1 = min(nnz, q0 + kCmpChunk);
+        const int r0 = chunk_r0[c], r1 = chunk_r0[c + 1];
+        int rc = r0;                                   // this thread's row cursor (monotone)
+        int64_t cs = __ldg(crowptr + rc), ce = __ldg(crowptr + rc + 1), ro = __ldg(rowoff + rc);
+        auto seek = [&](int64_t q) {                   // row of entry q (q >= cs): cached bounds
+            if (q < ce) return;
+            int lo = rc + 1, hi = r1 + 1;              // last row in (rc, r1] with crowptr <= q
+            while (hi - lo > 1) {
+                const int mid = (lo + hi) >> 1;
+                if (__ldg(crowptr + mid) <= q) lo = mid; else hi = mid;
+            }
+            rc = lo;
+            cs = __ldg(crowptr + rc);
+            ce = __ldg(crowptr + rc + 1);
+            ro = __ldg(rowoff + rc);
+        };
+        for (int64_t qv = q0 + 4 * threadIdx.x; qv < q1; qv += 4 * kCmpThreads) {
+            int32_t cc[4];
+            float vv[4];
+            seek(qv);
+            if (qv + 4 <= q1 && ce >= qv + 4) {
+                // the 4 entries are consecutive in one row: two aligned vectors + realign
+                const int64_t src = ro + (qv - cs);
+                const int sh = (int)(src & 3);
+                const int64_t a = src - sh;
+                // (default caching: the second vector is the next lane's first -- an L1 hit)
+                const int4 c0 = *reinterpret_cast<const int4 *>(chat_col + a);
+                const float4 v0 = *reinterpret_cast<const float4 *>(chat_val + a);
+                int4 oc = c0;
+                float4 ov = v0;
+                if (sh) {
+                    const int4 c1 = *reinterpret_cast<const int4 *>(chat_col + a + 4);
+                    const float4 v1 = *reinterpret_cast<const float4 *>(chat_val + a + 4);
+                    oc = realign4(c1, c0, 4 - sh);
+                    ov = realign4(v1, v0, 4 - sh);
+                }
+                __stcs(reinterpret_cast<int4 *>(out_col + qv), oc);
+                __stcs(reinterpret_cast<float4 *>(out_val + qv), ov);
+                continue;
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int64_t q = qv + u;
+                if (q < q1) {
+                    seek(q);
+                    const int64_t src = ro + (q - cs);
+                    cc[u] = __ldcs(chat_col + src);
+                    vv[u] = __ldcs(chat_val + src);
+                }
+            }
+            if (qv + 4 <= q1) {
+                __stcs(reinterpret_cast<int4 *>(out_col + qv), make_int4(cc[0], cc[1], cc[2], cc[3]));
+                __stcs(reinterpret_cast<float4 *>(out_val + qv), make_float4(vv[0], vv[1], vv[2], vv[3]));
+            } else {
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (qv + u < q1) { out_col[qv + u] = cc[u]; out_val[qv + u] = vv[u]; }
+            }
+        }
+    }
+}
+
 }  // namespace spg

@@ -883,7 +883,20 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
         TRY(talloc(p, t1, &dcol, nnz));
         TRY(talloc(p, t2, &dval, nnz));
     }
-    if (nnz > 0) {
+    const bool aligned = ((uintptr_t)dcol & 15) == 0 && ((uintptr_t)dval & 15) == 0;
+    if (nnz > 0 && aligned && p->opt.reserved[2] != 1) {
+        // load-balanced by output entry (any row-length mix)
+        const int64_t nchunks = cdiv(nnz, kCmpChunk);
+        Temp tc(s);
+        int32_t *chunk_r0;
+        TRY(talloc(p, tc, &chunk_r0, nchunks + 1));
+        LAUNCH("compact", s, k_chunk_first_row<<<grid_for(nchunks + 1, 256), 256, 0, s>>>(p->crowptr, p->m, nnz, nchunks,
+                                                                                          chunk_r0));
+        LAUNCH("compact", s, k_compact_flat<<<(unsigned)std::min<int64_t>(nchunks, (int64_t)p->num_sms * 8), kCmpThreads, 0,
+                                              s>>>(p->crowptr, p->rowoff, chunk_r0, nnz, nchunks, p->chat_col,
+                                                   p->chat_val, dcol, dval));
+    } else if (nnz > 0) {
+        // warp per row (realigned vectors) + CTA per long row (unaligned caller buffers; tuning)
         LAUNCH("compact", s, k_compact_rows<<<grid_for(p->m * 32, 256, (int64_t)p->num_sms * 16), 256, 0, s>>>(
             nullptr, p->crowptr, p->m, p->rowoff, p->chat_col, p->chat_val, dcol, dval));
         if (p->nlim > 0)
