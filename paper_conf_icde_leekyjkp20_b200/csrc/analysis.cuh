@@ -22,15 +22,17 @@ constexpr int kNumPairBuckets = 99;
 // row processing classes (SPGEMM_VIEW_ROW_CLASS) and buckets
 enum : int8_t { RC_EMPTY = 0, RC_PASS = 1, RC_WARP = 2, RC_WARP_SORT = 3, RC_GROUP_SORT = 4, RC_LIMITED = 5 };
 constexpr int kRowBucketPass = 0;
-constexpr int kRowBucketWarp = 1;      // cap <= 32: register bitonic
-constexpr int kRowBucketSort256 = 2;   // cap <= 256: one warp, merge-path natural merge sort
-constexpr int kRowBucketSort512 = 3;   // cap <= 512 / 1K / 2K / 4K: bucket sort, 2 / 4 / 8 / 16 warps
-constexpr int kRowBucketSort1K = 4;
-constexpr int kRowBucketSort2K = 5;
-constexpr int kRowBucketSort4K = 6;
-constexpr int kRowBucketLim0 = 7;      // 7 + (39 - floor(log2 L)): longest rows first
-constexpr int kRowBucketEmpty = 47;
-constexpr int kNumRowBuckets = 48;
+constexpr int kRowBucketWarp = 1;      // cap <= 32: register bitonic, 1 slot per lane
+constexpr int kRowBucketWarp64 = 2;    // cap <= 64 / 128 / 256: register bitonic, 2 / 4 / 8 slots per lane
+constexpr int kRowBucketWarp128 = 3;
+constexpr int kRowBucketSort256 = 4;
+constexpr int kRowBucketSort512 = 5;   // cap <= 512 / 1K / 2K / 4K: bucket sort, 2 / 4 / 8 / 16 warps
+constexpr int kRowBucketSort1K = 6;
+constexpr int kRowBucketSort2K = 7;
+constexpr int kRowBucketSort4K = 8;
+constexpr int kRowBucketLim0 = 9;      // 9 + (39 - floor(log2 L)): longest rows first
+constexpr int kRowBucketEmpty = 49;
+constexpr int kNumRowBuckets = 50;
 constexpr int kWarpRowMax = 32;
 // Ĉ runs are padded to multiples of kRunAlign slots (16 B) with sentinel entries
 // (col = INT32_MAX, val = 0) so that every run starts 16-byte aligned (vector stores).
@@ -356,6 +358,8 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
             mlen = max(mlen, (unsigned long long)cap);
         }
         else if (cap <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
+        else if (cap <= 64) { c = RC_WARP_SORT; b = kRowBucketWarp64; }
+        else if (cap <= 128) { c = RC_WARP_SORT; b = kRowBucketWarp128; }
         else if (cap <= kSort256Max) { c = RC_WARP_SORT; b = kRowBucketSort256; }
         else if (cap <= kSort512Max) { c = RC_WARP_SORT; b = kRowBucketSort512; }
         else if (cap <= kSort1KMax) { c = RC_WARP_SORT; b = kRowBucketSort1K; }

@@ -80,6 +80,126 @@ __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ 
     if (lane == 0 && !out_col) ccount[i] = __popc(tails);
 }
 
+// ------------------------------------------------------------ warp bins, E slots/lane ---
+// One warp per row of <= 32E padded slots, held in registers in blocked order (lane l owns
+// slots [lE, lE + E)): bitonic network over the 32E (col, val) pairs (partners at distance >= E
+// by shuffles, closer ones inside the lane), then an fp64 segmented reduction -- in-lane running
+// sums plus a segmented scan of the lanes' open tails -- and the segment ends are written back
+// in place (the row is in registers).  No shared memory: rows of <= 256 slots with few runs
+// (C4: 8 runs of 8) cost ~log2(32E)^2/2 shuffle stages instead of merge levels in smem.
+template <int E>
+__global__ void __launch_bounds__(256) k_merge_warpE(const int32_t *__restrict__ rows, int64_t nrows,
+                                                     const int64_t *__restrict__ rowoff, int32_t *__restrict__ chat_col,
+                                                     float *__restrict__ chat_val, int64_t *__restrict__ ccount) {
+    constexpr int N = 32 * E;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (gw >= nrows) return;
+    const int lane = lane_id();
+    const int i = rows[gw];
+    const int64_t s = rowoff[i];
+    const int L = (int)(rowoff[i + 1] - s);   // multiple of 4 (padded runs)
+    int32_t k[E];
+    float v[E];
+    if constexpr (E % 4 == 0) {
+#pragma unroll
+        for (int q = 0; q < E / 4; ++q) {
+            const int p = lane * E + 4 * q;
+            int4 c = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
+            float4 f = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (p < L) {
+                c = __ldcs(reinterpret_cast<const int4 *>(chat_col + s + p));
+                f = __ldcs(reinterpret_cast<const float4 *>(chat_val + s + p));
+            }
+            k[4 * q] = c.x; k[4 * q + 1] = c.y; k[4 * q + 2] = c.z; k[4 * q + 3] = c.w;
+            v[4 * q] = f.x; v[4 * q + 1] = f.y; v[4 * q + 2] = f.z; v[4 * q + 3] = f.w;
+        }
+    } else {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+            const int p = lane * E + e;
+            k[e] = p < L ? chat_col[s + p] : kKeyPad;
+            v[e] = p < L ? chat_val[s + p] : 0.f;
+        }
+    }
+#pragma unroll
+    for (int kk = 2; kk <= N; kk <<= 1) {
+#pragma unroll
+        for (int j = kk >> 1; j > 0; j >>= 1) {
+            if (j >= E) {
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    const int idx = lane * E + e;
+                    const int32_t pk = __shfl_xor_sync(kFull, k[e], j / E);
+                    const float pv = __shfl_xor_sync(kFull, v[e], j / E);
+                    const bool up = (idx & kk) == 0, lower = (idx & j) == 0;
+                    if (lower == up ? (pk < k[e]) : (pk > k[e])) { k[e] = pk; v[e] = pv; }
+                }
+            } else {
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    const int f = e ^ j;
+                    if (f > e) {
+                        const bool up = ((lane * E + e) & kk) == 0;
+                        if (up ? (k[f] < k[e]) : (k[f] > k[e])) {
+                            const int32_t tk = k[e]; k[e] = k[f]; k[f] = tk;
+                            const float tv = v[e]; v[e] = v[f]; v[f] = tv;
+                        }
+                    }
+                }
+            }
+        }
+    }
+    // fp64 segmented sums: a segment starts where the key changes
+    const int32_t prev_last = __shfl_up_sync(kFull, k[E - 1], 1);
+    double acc[E];
+    double run = 0.0;
+    bool any_head = false;
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        const bool head = e == 0 ? (lane == 0 || k[0] != prev_last) : (k[e] != k[e - 1]);
+        run = head ? (double)v[e] : run + (double)v[e];
+        any_head |= head;
+        acc[e] = run;
+    }
+    // segmented inclusive scan over lanes of (open tail sum, lane has a head)
+    double sc = run;
+    bool fl = any_head;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const double os = __shfl_up_sync(kFull, sc, d);
+        const bool of = __shfl_up_sync(kFull, (int)fl, d) != 0;
+        if (lane >= d && !fl) { sc += os; fl = of; }
+    }
+    double carry = __shfl_up_sync(kFull, sc, 1);
+    if (lane == 0) carry = 0.0;
+    bool open = true;   // slots before the lane's first head continue the previous lane's segment
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        open &= !(e == 0 ? (lane == 0 || k[0] != prev_last) : (k[e] != k[e - 1]));
+        if (open) acc[e] += carry;
+    }
+    // segment ends (valid keys only) -> in place, in order
+    const int32_t next_first = __shfl_down_sync(kFull, k[0], 1);
+    int nt = 0;
+    bool tail[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+        const int32_t nk = e < E - 1 ? k[e + 1] : (lane == 31 ? kKeyPad : next_first);
+        tail[e] = k[e] != kKeyPad && (nk != k[e] || (e == E - 1 && lane == 31));
+        nt += tail[e];
+    }
+    const int inc = warp_incl_sum(nt);
+    int o = inc - nt;
+#pragma unroll
+    for (int e = 0; e < E; ++e)
+        if (tail[e]) {
+            chat_col[s + o] = k[e];
+            chat_val[s + o] = (float)acc[e];
+            ++o;
+        }
+    if (lane == 31) ccount[i] = inc;
+}
+
 // ------------------------------------------------------------------ thread groups ---
 // A group of NW warps works on one row; GROUPS groups share a CTA.  Groups synchronise with
 // __syncwarp (NW = 1), __syncthreads (one group per CTA) or a named barrier (bar.sync id, n).

@@ -672,8 +672,25 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     // for the <= 256 bin, per-row bucket sort for the <= 1024 / <= 4096 bins), 1 register-staged
     // counting sort for the <= 256 / <= 1024 bins, 2 bucket sort everywhere, 3 merge-path everywhere
     const int variant = p->opt.reserved[0];
-    rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-    if (variant == 1) TRY(launch_wcs_bin<4, 2>(p, s, rows, cnt, "merge_wcs256"));
+    if (variant == 6) {
+        // register bitonic, 2 / 4 / 8 slots per lane (measured slower than the merge-path warp:
+        // C4 2.24 vs 2.11 ms, C2's <= 256 bin 0.80 vs 0.37 ms -- latency-bound, one row per warp)
+        rows = rows_of(kRowBucketWarp64, kRowBucketWarp64 + 1, &cnt);
+        if (cnt > 0)
+            LAUNCH("merge_warp64", s, k_merge_warpE<2><<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
+                rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
+        rows = rows_of(kRowBucketWarp128, kRowBucketWarp128 + 1, &cnt);
+        if (cnt > 0)
+            LAUNCH("merge_warp128", s, k_merge_warpE<4><<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
+                rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
+        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
+        if (cnt > 0)
+            LAUNCH("merge_warp256", s, k_merge_warpE<8><<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
+                rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
+    }
+    rows = rows_of(kRowBucketWarp64, kRowBucketSort256 + 1, &cnt);   // 32 < slots <= 256
+    if (variant == 6) {
+    } else if (variant == 1) TRY(launch_wcs_bin<4, 2>(p, s, rows, cnt, "merge_wcs256"));
     else if (variant == 2) TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
     else TRY(launch_wmp_bin<1, 8, 256>(p, s, rows, cnt, "merge_wmp256"));
     if (variant == 1) {
@@ -974,12 +991,12 @@ int spgemm_get_stats(spgemm_plan_t p, spgemm_stats_t *st) {
     st->n_rows_bin[0] = p->row_starts[kRowBucketEmpty + 1] - p->row_starts[kRowBucketEmpty];
     st->n_rows_bin[1] = p->row_starts[kRowBucketPass + 1] - p->row_starts[kRowBucketPass];
     st->n_rows_bin[2] = p->row_starts[kRowBucketWarp + 1] - p->row_starts[kRowBucketWarp];
-    st->n_rows_bin[3] = p->row_starts[kRowBucketSort1K + 1] - p->row_starts[kRowBucketSort256];
+    st->n_rows_bin[3] = p->row_starts[kRowBucketSort1K + 1] - p->row_starts[kRowBucketWarp64];
     st->n_rows_bin[4] = p->row_starts[kRowBucketSort4K + 1] - p->row_starts[kRowBucketSort2K];
     st->n_rows_bin[5] = p->nlim;
     st->bytes_workspace = p->bytes;
     st->n_units = st->n_units_fallback = -1;
-    if (p->state >= 3 && p->m > 0) {
+    if (p->state >= 3 && p->m > 0 && p->c_in_chat) {
         unsigned long long t[2];
         CK(cudaMemcpy(&st->n_units, p->nunits, 8, cudaMemcpyDeviceToHost));
         CK(cudaMemcpy(t, p->unit_ticket, 16, cudaMemcpyDeviceToHost));

@@ -75,6 +75,7 @@ CASES = [
     ("C1", dict(reserved=(1,) + (0,) * 15)),   # merge variant: register-staged counting sort
     ("C1", dict(reserved=(2,) + (0,) * 15)),   # merge variant: smem bucket sort everywhere
     ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: merge-path everywhere
+    ("C1", dict(reserved=(6,) + (0,) * 15)),   # merge variant: register bitonic for <= 256 slots
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
     ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
@@ -217,7 +218,7 @@ def test_random_tiny(shape, dens, seed, skew, values):
     inp = synth.random_tiny(*shape, dens[0], dens[1], seed, values=values, skew=skew)
     A, B = spg.from_inputs(inp, "cuda")
     for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(1,) + (0,) * 15),
-                 dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15), FUSED,
+                 dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15), FUSED, dict(reserved=(6,) + (0,) * 15),
                  dict(beta=1000.0, piece_work=64, split_ca_max=3, **FUSED)):
         C = spg.matmul(A, B, **opts)
         assert_c_matches(C, inp, signed=(values == "signed"))
