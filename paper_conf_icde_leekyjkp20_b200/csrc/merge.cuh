@@ -424,22 +424,47 @@ __device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const
     return wtot;
 }
 
+// striped load of a row into registers (slot gtid + e*T); sentinel (padding) entries stay kKeyPad
+template <int NW, int GROUPS, int EPT>
+__device__ __forceinline__ void bsr_load(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv, int L,
+                                         int32_t (&key)[EPT], float (&val)[EPT]) {
+    constexpr int T = NW * 32;
+#pragma unroll
+    for (int e = 0; e < EPT; ++e) {
+        const int p = g.gtid + e * T;
+        key[e] = p < L ? sk[p] : kKeyPad;
+        val[e] = p < L ? sv[p] : 0.f;
+    }
+}
+
+template <int NW, int GROUPS, int EPT, int LS = 0>
+__device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
+                                                       float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
+                                                       float *dv2, int *hist, int32_t *out_col, float *out_val,
+                                                       int *sc);
+
 // LS: buckets = 2^LS x (slots rounded up to a power of two); more buckets, fewer shared ones
 template <int NW, int GROUPS, int EPT, int LS = 0>
 __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
                                                   int L, int32_t *dk, float *dv, int32_t *dk2, float *dv2,
                                                   int *hist, int32_t *out_col, float *out_val, int *sc) {
-    constexpr int T = NW * 32;
     int32_t key[EPT];
     float val[EPT];
+    bsr_load<NW, GROUPS, EPT>(g, sk, sv, L, key, val);
+    return bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, L, dk, dv, dk2, dv2, hist, out_col, out_val, sc);
+}
+
+// the row already in registers (bsr_load; software-pipelined callers load the next row early)
+template <int NW, int GROUPS, int EPT, int LS>
+__device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
+                                                       float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
+                                                       float *dv2, int *hist, int32_t *out_col, float *out_val,
+                                                       int *sc) {
+    constexpr int T = NW * 32;
     int32_t mn = kKeyPad, mx = 0;
 #pragma unroll
-    for (int e = 0; e < EPT; ++e) {
-        const int p = g.gtid + e * T;
-        key[e] = p < L ? sk[p] : kKeyPad;       // sentinel (padding) entries stay kKeyPad
-        val[e] = p < L ? sv[p] : 0.f;
+    for (int e = 0; e < EPT; ++e)
         if (key[e] != kKeyPad) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
-    }
     mn = g.reduce_min(mn, sc);
     mx = g.reduce_max(mx, sc);
     const uint32_t span = (uint32_t)(mx - mn);
@@ -598,6 +623,70 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
         g.sync();
     }
     (void)cap_skip;
+}
+
+// Software-pipelined variant (in place): per row r of the bin the group holds row r's slots in
+// registers, loads row r + S (S = groups in the grid) while sorting row r, and row r + 2S's
+// (offset, length, id) from the bin's meta table -- one independent load -- so neither the
+// row data nor its offsets are a dependent memory round trip on the sort's critical path.
+struct RowMeta {
+    int64_t s;    // first slot of the row's Ĉ bucket
+    int32_t L;    // padded length
+    int32_t i;    // row id
+};
+
+__global__ void k_row_meta(const int32_t *__restrict__ order, int64_t n, const int64_t *__restrict__ rowoff,
+                           RowMeta *__restrict__ meta) {
+    for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
+        const int i = order[q];
+        const int64_t s = rowoff[i];
+        meta[q] = RowMeta{s, (int32_t)(rowoff[i + 1] - s), i};
+    }
+}
+
+template <int NW, int GROUPS, int EPT, int LS = 0>
+__global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k_merge_bucket_pipe(
+    const RowMeta *__restrict__ meta, int64_t nrows, int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
+    int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows, unsigned *__restrict__ fb_count) {
+    using S = BucketSmem<NW, EPT, LS>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ int sc_all[GROUPS][NW + 1];
+    const Group<NW, GROUPS> g;
+    unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
+    int32_t *dk = (int32_t *)slice;
+    float *dv = (float *)(slice + S::kCap * 4);
+    int32_t *dk2 = (int32_t *)(slice + S::kCap * 8);
+    float *dv2 = (float *)(slice + S::kCap * 12);
+    int *hist = (int *)(slice + S::kCap * 16);
+    const int64_t stride = (int64_t)gridDim.x * GROUPS;
+    int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid;
+    const RowMeta none{0, 0, -1};
+    RowMeta m0 = r < nrows ? meta[r] : none;
+    RowMeta m1 = r + stride < nrows ? meta[r + stride] : none;
+    int32_t key[EPT];
+    float val[EPT];
+    bsr_load<NW, GROUPS, EPT>(g, chat_col + m0.s, chat_val + m0.s, min(m0.L, S::kCap), key, val);
+    while (r < nrows) {
+        int32_t kn[EPT];
+        float vn[EPT];
+        bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, min(m1.L, S::kCap), kn, vn);
+        const RowMeta m2 = r + 2 * stride < nrows ? meta[r + 2 * stride] : none;
+        if (m0.L <= S::kCap) {
+            const int U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
+                                                                       chat_col + m0.s, chat_val + m0.s,
+                                                                       sc_all[g.gid]);
+            if (g.gtid == 0) {
+                if (U >= 0) ccount[m0.i] = U;
+                else fb_rows[atomicAdd(fb_count, 1u)] = m0.i;
+            }
+        }
+        g.sync();
+#pragma unroll
+        for (int e = 0; e < EPT; ++e) { key[e] = kn[e]; val[e] = vn[e]; }
+        m0 = m1;
+        m1 = m2;
+        r += stride;
+    }
 }
 
 // ------------------------------------------- register-staged counting sort (WCS) ---

@@ -76,6 +76,8 @@ CASES = [
     ("C1", dict(reserved=(2,) + (0,) * 15)),   # merge variant: smem bucket sort everywhere
     ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: merge-path everywhere
     ("C1", dict(reserved=(6,) + (0,) * 15)),   # merge variant: register bitonic for <= 256 slots
+    ("C1", dict(reserved=(7,) + (0,) * 15)),   # merge variant: bucket bins without pipelining
+    ("C1", dict(reserved=(8,) + (0,) * 15)),   # merge variant: all bucket bins pipelined
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
     ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
