@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--opt", action="append", default=[],
+                    help="spgemm option key=value (e.g. enable_split=0: the Fig. 10 ablations)")
     return ap.parse_args()
 
 
@@ -167,6 +169,9 @@ def main():
         inp, A, B = inp_full, A_full, B_full
     stream = torch.cuda.current_stream(dev)
     opts = dict(validate=0)
+    for kv in args.opt:
+        k, v = kv.split("=")
+        opts[k] = float(v) if k in ("alpha", "beta") else int(v)
     if os.environ.get("SPGEMM_RESERVED"):   # tuning knobs: "index=value,..."
         res = [0] * 16
         for kv in os.environ["SPGEMM_RESERVED"].split(","):
@@ -287,7 +292,8 @@ def main():
                    "nnz_a": inp_full.nnz_a, "products": products_all, "nnz_c": nnz_c_all,
                    "parallelism": f"row-partition x{ws}" if ws > 1 else "single GPU",
                    "l2": "flushed between steps (512 MiB write); Ĉ >> L2", "seed": args.seed,
-                   "step": "plan+execute+destroy via C-ABI, device-resident inputs"},
+                   "step": "plan+execute+destroy via C-ABI, device-resident inputs",
+                   **({"options": {k: v for k, v in opts.items() if k != "validate"}} if len(opts) > 1 else {})},
         "roofline": roofline,
         "step_roofline": {"achieved": round(step_bw, 1), "peak": hbm, "unit": "GB/s",
                           "frac": round(step_bw / hbm, 4), "bytes": int(bytes_step),
