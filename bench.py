@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--slice", default=None,
+                    help="N:r -- run only rank r's row block of an N-way partition on this GPU (scaling study)")
     ap.add_argument("--opt", action="append", default=[],
                     help="spgemm option key=value (e.g. enable_split=0: the Fig. 10 ablations)")
     return ap.parse_args()
@@ -157,12 +159,16 @@ def main():
     dev = torch.device("cuda", local)
     inp_full = synth.make_inputs(args.config, seed=args.seed)
     A_full, B_full = spg.from_inputs(inp_full, dev)
-    if ws > 1:
+    nparts, part = (ws, rank)
+    if args.slice:
+        nparts, part = (int(x) for x in args.slice.split(":"))
+    if nparts > 1:
         from paper_conf_icde_leekyjkp20_b200 import dist as pdist
-        bounds = spg.row_partition(A_full, B_full, ws)
-        A = pdist.csc_row_slice(A_full, int(bounds[rank]), int(bounds[rank + 1]))
+        bounds = spg.row_partition(A_full, B_full, nparts)
+        rank_ = part
+        A = pdist.csc_row_slice(A_full, int(bounds[rank_]), int(bounds[rank_ + 1]))
         B = B_full
-        inp = synth.SparseInputs(f"{args.config}[{bounds[rank]}:{bounds[rank + 1]}]", A.nrows, A.ncols, B.ncols,
+        inp = synth.SparseInputs(f"{args.config}[{bounds[rank_]}:{bounds[rank_ + 1]}]", A.nrows, A.ncols, B.ncols,
                                  A.colptr.cpu().numpy(), A.rowidx.cpu().numpy(), A.val.cpu().numpy(),
                                  inp_full.b_rowptr, inp_full.b_colidx, inp_full.b_val)
     else:

@@ -327,11 +327,10 @@ __global__ void k_piece_whole(const int32_t *__restrict__ list, int64_t n, const
     }
 }
 
-// padded length of every B row (input of the B' row-pointer scan)
-__global__ void k_row_padded_len(const int64_t *__restrict__ b_rowptr, int64_t K, int64_t *__restrict__ out) {
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x)
-        out[k] = pad_run(b_rowptr[k + 1] - b_rowptr[k]);
-}
+// B' (B with rows padded to 4 slots) row k starts at bp_start(b_rowptr[k], k) = b_rowptr[k] + 7k
+// rounded up to 4 slots: 16-byte aligned and clear of row k + 1 (row k ends by b_rowptr[k+1] + 7k + 6)
+// without a scan over the padded lengths; B' holds nnz(B) + 7K + 4 slots.
+__host__ __device__ __forceinline__ int64_t bp_start(int64_t rp, int64_t k) { return (rp + 7 * k + 3) & ~(int64_t)3; }
 
 // Merge row classes.  Limited rows (L > t_lim, L452-L477 L) get B-Limited merge blocks;
 // a row made of a single run (one A entry) is already sorted and duplicate-free.

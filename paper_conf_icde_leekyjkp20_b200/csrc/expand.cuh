@@ -43,13 +43,13 @@ __global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64
 }
 
 // B' = B with every row padded to a multiple of 4 slots (col = INT32_MAX, val = 0); one thread
-// per row (rows are short), 16-byte stores
+// per row, 16-byte stores (measured: a warp per 32 rows is 2x slower -- rows are short)
 __global__ void k_pad_b(const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ b_colidx,
-                        const float *__restrict__ b_val, int64_t K, const int64_t *__restrict__ b_prow,
-                        int32_t *__restrict__ bp_col, float *__restrict__ bp_val) {
+                        const float *__restrict__ b_val, int64_t K, int32_t *__restrict__ bp_col,
+                        float *__restrict__ bp_val) {
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x) {
         const int64_t b0 = b_rowptr[k], rb = b_rowptr[k + 1] - b0;
-        const int64_t d0 = b_prow[k];
+        const int64_t d0 = bp_start(b0, k);
         for (int64_t j = 0; j < rb; j += 4) {
             int32_t c[4];
             float v[4];
@@ -99,7 +99,7 @@ constexpr int kExpPieceCache = 1024;
 
 __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     const Piece *__restrict__ pieces, const int64_t *__restrict__ uoff, int64_t npieces,
-    const int64_t *__restrict__ tile_p0, const int64_t *__restrict__ b_prow, const int32_t *__restrict__ bp_col,
+    const int64_t *__restrict__ tile_p0, const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ bp_col,
     const float *__restrict__ bp_val, const float *__restrict__ a_val, const int64_t *__restrict__ base,
     int32_t *__restrict__ chat_col, float *__restrict__ chat_val) {
     __shared__ int64_t s_uoff[kExpPieceCache + 1];
@@ -121,7 +121,7 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
                 const Piece pc = pieces[p0 + q];
                 s_uoff[q] = uoff[p0 + q];
                 s_alo[q] = pc.a_lo;
-                s_bsrc[q] = b_prow[pc.k] + pc.b_off;
+                s_bsrc[q] = bp_start(b_rowptr[pc.k], pc.k) + pc.b_off;
                 s_nv[q] = piece_nvec(pc);
                 s_boff[q] = pc.b_off;
             }
@@ -158,7 +158,7 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
                         if (__ldg(uoff + mid) <= f) gj = mid; else hi = mid;
                     }
                     const Piece pc = pieces[gj];
-                    uo = __ldg(uoff + gj); alo = pc.a_lo; bsrc = __ldg(b_prow + pc.k) + pc.b_off;
+                    uo = __ldg(uoff + gj); alo = pc.a_lo; bsrc = bp_start(__ldg(b_rowptr + pc.k), pc.k) + pc.b_off;
                     nv = piece_nvec(pc); boff = pc.b_off;
                 }
                 const int64_t r = f - uo;

@@ -8,6 +8,9 @@
 #include <cstring>
 #include <string>
 #include <vector>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 #include "../../include/spgemm.h"
 #include "analysis.cuh"
@@ -139,7 +142,7 @@ struct spgemm_plan_s {
     int64_t *piece_uoff = nullptr; // unit (16-byte vector) prefix over pieces
     int64_t *tile_p0 = nullptr;    // first piece of every expansion tile
     int64_t n_low = 0, n_pieces_all = 0;
-    int64_t *b_prow = nullptr;     // B' (rows padded to 4 slots): row starts, cols, values
+    // B' (rows padded to 4 slots, row k at bp_start(b_rowptr[k], k)): cols, values
     int32_t *bp_col = nullptr;
     float *bp_val = nullptr;
 
@@ -212,6 +215,28 @@ static inline unsigned grid_for(int64_t n, int threads, int64_t cap = 148 * 64) 
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(n, threads), cap));
 }
 
+// Large-smem kernels: opt-in shared memory size and resident blocks per SM, queried once per
+// (kernel, device, smem, threads) -- these runtime calls cost host microseconds on every step.
+static int kernel_occupancy(const void *kern, int smem, int threads, int *occ) {
+    static std::mutex mu;
+    static std::map<std::tuple<const void *, int, int, int>, int> cache;
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    const auto key = std::make_tuple(kern, dev, smem, threads);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(key);
+    if (it != cache.end()) {
+        if (occ) *occ = it->second;
+        return SPGEMM_OK;
+    }
+    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    int o = 0;
+    if (threads > 0) CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, threads, smem));
+    cache[key] = o;
+    if (occ) *occ = o;
+    return SPGEMM_OK;
+}
+
 // ------------------------------------------------------------------ primitives -----------
 template <typename Tin>
 static int scan_excl(spgemm_plan_s *p, const Tin *in, int64_t n, int64_t *out, cudaStream_t s, const char *name) {
@@ -255,9 +280,8 @@ static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int6
                               int ctas_per_sm) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, 0>::kBytes * GROUPS;
-    CK(cudaFuncSetAttribute(k_merge_bucket_pipe<NW, GROUPS, EPT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_merge_bucket_pipe<NW, GROUPS, EPT>, NW * 32 * GROUPS, smem));
+    TRY(kernel_occupancy((const void *)k_merge_bucket_pipe<NW, GROUPS, EPT>, smem, NW * 32 * GROUPS, &occ));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
     (void)ctas_per_sm;
     LAUNCH(name, s, k_merge_bucket_pipe<NW, GROUPS, EPT><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
@@ -271,7 +295,7 @@ static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *ro
                              int ctas_per_sm, bool fallback_list = true, bool side = false) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, LS>::kBytes * GROUPS;
-    CK(cudaFuncSetAttribute(k_merge_bucket<NW, GROUPS, EPT, LS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    TRY(kernel_occupancy((const void *)k_merge_bucket<NW, GROUPS, EPT, LS>, smem, 0, nullptr));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
     LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT, LS><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
         rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0,
@@ -284,9 +308,8 @@ static int launch_wcs_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows,
     if (cnt == 0) return SPGEMM_OK;
     const int smem = WcsSmem<VPT>::kBytes * GROUPS;
     auto kern = k_merge_wcs<GROUPS, VPT>;
-    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 32 * GROUPS, smem));
+    TRY(kernel_occupancy((const void *)kern, smem, 32 * GROUPS, &occ));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
     LAUNCH(name, s, kern<<<(unsigned)grid, 32 * GROUPS, smem, s>>>(rows, cnt, p->rowoff, p->rowwork, p->chat_col,
                                                                   p->chat_val, p->ccount, nullptr, nullptr, nullptr));
@@ -298,9 +321,8 @@ static int launch_wmp_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows,
     if (cnt == 0) return SPGEMM_OK;
     const int smem = WmpSmem<CAP>::kBytes * GROUPS;
     auto kern = k_merge_wmp<NW, GROUPS, CAP>;
-    CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
     int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, NW * 32 * GROUPS, smem));
+    TRY(kernel_occupancy((const void *)kern, smem, NW * 32 * GROUPS, &occ));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
     LAUNCH(name, s, kern<<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(rows, cnt, p->rowoff, p->rowwork, p->chat_col,
                                                                        p->chat_val, p->ccount, nullptr, nullptr,
@@ -570,20 +592,11 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         CK(cudaMemsetAsync(p->piece_uoff, 0, 8, s));
     }
     // B' = B with rows padded to 4 slots (16-byte aligned vector loads in the expansion)
-    TRY(palloc(p, &p->b_prow, K + 1, s));
-    TRY(palloc(p, &p->bp_col, p->nnz_b + 3 * K, s));
-    TRY(palloc(p, &p->bp_val, p->nnz_b + 3 * K, s));
-    if (K > 0) {
-        Temp tpl(s);
-        int64_t *plen;
-        TRY(talloc(p, tpl, &plen, K));
-        LAUNCH("pad_b", s, k_row_padded_len<<<grid_for(K, 256), 256, 0, s>>>(p->b_rowptr, K, plen));
-        TRY(scan_excl(p, plen, K, p->b_prow, s, "pad_b"));
-        LAUNCH("pad_b", s, k_pad_b<<<grid_for(K, 256), 256, 0, s>>>(
-            p->b_rowptr, p->b_colidx, p->b_val, K, p->b_prow, p->bp_col, p->bp_val));
-    } else {
-        CK(cudaMemsetAsync(p->b_prow, 0, 8, s));
-    }
+    TRY(palloc(p, &p->bp_col, p->nnz_b + 7 * K + 4, s));
+    TRY(palloc(p, &p->bp_val, p->nnz_b + 7 * K + 4, s));
+    if (K > 0)
+        LAUNCH("pad_b", s, k_pad_b<<<grid_for(K, 256), 256, 0, s>>>(p->b_rowptr, p->b_colidx, p->b_val, K, p->bp_col,
+                                                                    p->bp_val));
     // limited rows: index map, run lists, B-Limited scratch
     p->nlim = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketLim0];
     if (p->nlim > 0) {
@@ -663,7 +676,7 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     }
     if (p->n_pieces_all > 0)
         LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
-            p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_prow, p->bp_col, p->bp_val, p->a_val,
+            p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
             p->base, p->chat_col, p->chat_val));
     p->state = 2;
     return SPGEMM_OK;
@@ -755,7 +768,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
-        CK(cudaFuncSetAttribute(k_merge_rows<8, 1, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        TRY(kernel_occupancy((const void *)k_merge_rows<8, 1, CAP>, smem, 0, nullptr));
         LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
             p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count, nullptr, nullptr,
             nullptr));
@@ -790,7 +803,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
-        CK(cudaFuncSetAttribute(k_merge_limited, cudaFuncAttributeMaxDynamicSharedMemorySize, kLimSmem));
+        TRY(kernel_occupancy((const void *)k_merge_limited, kLimSmem, 0, nullptr));
         LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
     }
     TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
@@ -813,7 +826,7 @@ static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
-        CK(cudaFuncSetAttribute(k_merge_rows<8, 1, CAP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        TRY(kernel_occupancy((const void *)k_merge_rows<8, 1, CAP>, smem, 0, nullptr));
         LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
             p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count, p->side_off,
             p->side_col, p->side_val));
@@ -848,7 +861,7 @@ static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false, true));
-        CK(cudaFuncSetAttribute(k_merge_limited, cudaFuncAttributeMaxDynamicSharedMemorySize, kLimSmem));
+        TRY(kernel_occupancy((const void *)k_merge_limited, kLimSmem, 0, nullptr));
         LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
     }
     // (b) every unit of short rows (and the long rows' copies), in row order, straight into C
@@ -875,9 +888,8 @@ static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
         ua.debug = p->opt.reserved[1];
         ua.prof = p->unit_ticket + 2;
         constexpr int smem = UnitSmem<kUnitThreads>::kBytes;
-        CK(cudaFuncSetAttribute(k_merge_units<kUnitThreads>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
         int occ = 0;
-        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_merge_units<kUnitThreads>, kUnitThreads, smem));
+        TRY(kernel_occupancy((const void *)k_merge_units<kUnitThreads>, smem, kUnitThreads, &occ));
         LAUNCH("merge_units", s, k_merge_units<kUnitThreads><<<(unsigned)(p->num_sms * std::max(occ, 1)), kUnitThreads,
                                                                  smem, s>>>(ua));
         const int64_t nlong = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketSort4K];
