@@ -1618,7 +1618,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     int tot;
                     int ex = grp.excl_sum(cnt, sc, &tot);
                     mxb = grp.reduce_max(mxb, sc);
-                    constexpr int T = kLimCap / 2;
+                    constexpr int T = kLimCap * 3 / 4;   // groups < T + max bin <= kLimCap (7/8: same speed)
 #pragma unroll
                     for (int u = 0; u < BPT; ++u) {
                         fh[threadIdx.x * BPT + u] = ex / T;     // group id of the bin
@@ -1636,7 +1636,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     }
                     if (threadIdx.x == 0) {
                         s_ngroups = ng;
-                        s_bad = mxb > T;
+                        s_bad = mxb > kLimCap - T;
                         gstart[ng] = tot;
                     }
                     __syncthreads();
