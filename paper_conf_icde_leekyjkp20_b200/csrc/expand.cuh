@@ -183,4 +183,82 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     }
 }
 
+// ------------------------------------------------ row-product expansion (comparison) ---
+// The paper's comparison point (row-product / Gustavson order, L476-L478 R): the same Ĉ (every
+// run at base[e]) written row by row -- one warp per row of A walks the row's entries (A in CSR
+// order, built by a counting sort of the CSC entries) and copies nnz(b_k*) scaled B' vectors per
+// entry.  No Block Reorganizer: a row's work is one warp's, whatever its size.  Selected by
+// options.reserved[3] = 1 (bench --opt reserved... / tests); DESIGN.md §5 compares the two.
+__global__ void k_row_entries(const int64_t *__restrict__ a_colptr, int64_t K, int64_t nnz_a,
+                              const int32_t *__restrict__ a_rowidx, const int64_t *__restrict__ b_rowptr,
+                              const int64_t *__restrict__ rptr, unsigned *__restrict__ cursor,
+                              int64_t *__restrict__ list_e, int32_t *__restrict__ list_k) {
+    int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
+    if (e0 >= nnz_a) return;
+    int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
+    int64_t kend = __ldg(a_colptr + k + 1);
+    for (int64_t e = e0; e < e0 + 8 && e < nnz_a; ++e) {
+        while (e >= kend) { ++k; kend = __ldg(a_colptr + k + 1); }
+        if (__ldg(b_rowptr + k + 1) > __ldg(b_rowptr + k)) {
+            const int i = a_rowidx[e];
+            const int64_t q = rptr[i] + atomicAdd(cursor + i, 1u);
+            list_e[q] = e;
+            list_k[q] = (int32_t)k;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_expand_rows(const int64_t *__restrict__ rptr, int64_t M,
+                                                     const int64_t *__restrict__ list_e,
+                                                     const int32_t *__restrict__ list_k,
+                                                     const int64_t *__restrict__ b_rowptr,
+                                                     const int32_t *__restrict__ bp_col,
+                                                     const float *__restrict__ bp_val,
+                                                     const float *__restrict__ a_val,
+                                                     const int64_t *__restrict__ base, int32_t *__restrict__ chat_col,
+                                                     float *__restrict__ chat_val) {
+    const int lane = lane_id();
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < M; i += nw) {
+        const int64_t e_lo = rptr[i], e_hi = rptr[i + 1];
+        for (int64_t c0 = e_lo; c0 < e_hi; c0 += 32) {
+            const int64_t q = c0 + lane;
+            int nv = 0;
+            int64_t src = 0, dst = 0;
+            float av = 0.f;
+            if (q < e_hi) {
+                const int64_t e = list_e[q];
+                const int32_t k = list_k[q];
+                const int64_t b0 = __ldg(b_rowptr + k);
+                nv = (int)((__ldg(b_rowptr + k + 1) - b0 + 3) >> 2);
+                src = bp_start(b0, k);
+                dst = base[e];
+                av = a_val[e];
+            }
+            const int inc = warp_incl_sum(nv);
+            const int off = inc - nv, tot = __shfl_sync(0xffffffffu, inc, 31);
+            for (int u0 = 0; u0 < tot; u0 += 32) {
+                const int u = u0 + lane;
+                int j = 0;               // owner lane: number of lanes with inc <= u
+#pragma unroll
+                for (int step = 16; step > 0; step >>= 1) {
+                    const int probe = __shfl_sync(0xffffffffu, inc, min(j + step - 1, 31));
+                    if (j + step <= 32 && probe <= u) j += step;
+                }
+                j = min(j, 31);
+                const int64_t s_j = __shfl_sync(0xffffffffu, src, j), d_j = __shfl_sync(0xffffffffu, dst, j);
+                const float a_j = __shfl_sync(0xffffffffu, av, j);
+                const int v = u - __shfl_sync(0xffffffffu, off, j);
+                if (u < tot) {
+                    const int4 c4 = __ldg(reinterpret_cast<const int4 *>(bp_col + s_j + 4 * v));
+                    const float4 w4 = __ldg(reinterpret_cast<const float4 *>(bp_val + s_j + 4 * v));
+                    __stcs(reinterpret_cast<int4 *>(chat_col + d_j + 4 * v), c4);
+                    __stcs(reinterpret_cast<float4 *>(chat_val + d_j + 4 * v),
+                           make_float4(a_j * w4.x, a_j * w4.y, a_j * w4.z, a_j * w4.w));
+                }
+            }
+        }
+    }
+}
+
 }  // namespace spg

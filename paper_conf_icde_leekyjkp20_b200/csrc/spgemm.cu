@@ -674,10 +674,28 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
         TRY(palloc(p, &p->chat_col, p->chat_cap, s));
         TRY(palloc(p, &p->chat_val, p->chat_cap, s));
     }
-    if (p->n_pieces_all > 0)
+    if (p->opt.reserved[3] == 1 && p->m > 0 && p->nnz_a > 0) {
+        // row-product expansion (the paper's comparison order): A's entries by row, warp per row
+        const int64_t M = p->m;
+        Temp tr(s), tc(s), te(s), tk(s);
+        int64_t *rptr, *list_e;
+        unsigned *cursor;
+        int32_t *list_k;
+        TRY(talloc(p, tr, &rptr, M + 1));
+        TRY(talloc(p, tc, &cursor, M));
+        TRY(talloc(p, te, &list_e, p->nnz_a));
+        TRY(talloc(p, tk, &list_k, p->nnz_a));
+        TRY(scan_excl(p, p->deg, M, rptr, s, "expand_rows"));
+        CK(cudaMemsetAsync(cursor, 0, M * 4, s));
+        LAUNCH("expand_rows", s, k_row_entries<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+            p->a_colptr, p->k, p->nnz_a, p->a_rowidx, p->b_rowptr, rptr, cursor, list_e, list_k));
+        LAUNCH("expand_rows", s, k_expand_rows<<<grid_for(M * 32, 256, (int64_t)p->num_sms * 8), 256, 0, s>>>(
+            rptr, M, list_e, list_k, p->b_rowptr, p->bp_col, p->bp_val, p->a_val, p->base, p->chat_col, p->chat_val));
+    } else if (p->n_pieces_all > 0) {
         LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
             p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
             p->base, p->chat_col, p->chat_val));
+    }
     p->state = 2;
     return SPGEMM_OK;
 }

@@ -78,6 +78,7 @@ CASES = [
     ("C1", dict(reserved=(6,) + (0,) * 15)),   # merge variant: register bitonic for <= 256 slots
     ("C1", dict(reserved=(7,) + (0,) * 15)),   # merge variant: bucket bins without pipelining
     ("C1", dict(reserved=(8,) + (0,) * 15)),   # merge variant: all bucket bins pipelined
+    ("C1", dict(reserved=(0, 0, 0, 1) + (0,) * 12)),   # row-product expansion (comparison order)
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
     ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
@@ -166,7 +167,11 @@ def _rows_sorted(m, rowoff, cols, vals):
     return out
 
 
-@pytest.mark.parametrize("name,opts", CASES[:1] + CASES[4:7])
+EXPAND_CASES = [c for c in CASES if not c[1] or {"enable_gather", "enable_split", "piece_work"} & set(c[1])
+                or c[1].get("reserved", (0,) * 4)[3] == 1]
+
+
+@pytest.mark.parametrize("name,opts", EXPAND_CASES)
 def test_stage3_expansion_is_eq2(name, opts):
     inp = _inp(name)
     p, keep = _plan(inp, **opts)
