@@ -196,6 +196,12 @@ int spgemm_destroy(spgemm_plan_t plan);
 int spgemm_row_partition(const spgemm_csc_t *A, const spgemm_csr_t *B, int32_t parts, int64_t *bounds_host,
                          void *stream);
 
+/* Plans allocate their workspaces from a per-device stream-ordered pool that keeps freed memory
+ * for the next plan (no OS allocation per step).  spgemm_trim_pool returns the current device's
+ * cached memory to the driver (e.g. before allocating a large C or between very large products).
+ * Synchronises the device. */
+int spgemm_trim_pool(void);
+
 /* Per-kernel device timing of the last spgemm_expand / spgemm_merge (CUDA events on the
  * launch stream; enabled by spgemm_set_timing(1)).  names/ms arrays of capacity n. */
 int spgemm_set_timing(int32_t enable);

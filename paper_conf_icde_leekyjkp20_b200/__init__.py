@@ -28,7 +28,7 @@ VIEW_WORK, VIEW_ROWWORK, VIEW_ROWOFF, VIEW_PAIR_CLASS, VIEW_PIECES, VIEW_GATHER,
 EXPORTED = ["spgemm_abi_version", "spgemm_last_error", "spgemm_default_options", "spgemm_plan",
             "spgemm_expand", "spgemm_merge", "spgemm_output", "spgemm_execute", "spgemm_get_stats",
             "spgemm_inspect", "spgemm_destroy", "spgemm_set_timing", "spgemm_last_timings",
-            "spgemm_row_partition"]
+            "spgemm_row_partition", "spgemm_trim_pool"]
 
 
 class SpgemmError(RuntimeError):
@@ -96,6 +96,7 @@ def lib():
         L.spgemm_destroy.argtypes = [vp]
         L.spgemm_row_partition.argtypes = [ctypes.POINTER(_CSC), ctypes.POINTER(_CSR), i32, vp, vp]
         L.spgemm_set_timing.argtypes = [i32]
+        L.spgemm_trim_pool.argtypes = []
         L.spgemm_last_timings.argtypes = [ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(ctypes.c_float), i32,
                                           ctypes.POINTER(i32)]
         for f in EXPORTED:
@@ -274,6 +275,24 @@ def matmul(A: CSC, B: CSR, device=None, stream=None, **opts) -> CSR:
         return p.execute(device=device)
 
 
+def matmul_chunked(A: CSC, B: CSR, parts: int, device=None, stream=None, **opts) -> CSR:
+    """C = A x B in `parts` balanced row blocks run one after another (north star C5: chunked
+    expansion): the blocks' Ĉ are formed and merged in turn, so the peak intermediate storage is
+    ~nnz(Ĉ)/parts.  Same boundaries as the multi-GPU row partition (R8)."""
+    from . import dist as pdist
+    if parts <= 1:
+        return matmul(A, B, device=device, stream=stream, **opts)
+    bounds = row_partition(A, B, parts, stream=stream)
+    blocks = []
+    for r in range(parts):
+        Ar = pdist.csc_row_slice(A, int(bounds[r]), int(bounds[r + 1]))
+        C = matmul(Ar, B, device=device, stream=stream, **opts)
+        if C.colidx.untyped_storage().nbytes() > C.colidx.numel() * 4 * 1.05:   # release capacity slack
+            C = CSR(C.nrows, C.ncols, C.rowptr, C.colidx.clone(), C.val.clone())
+        blocks.append(C)
+    return pdist.concat_row_blocks(blocks)
+
+
 def row_partition(A: CSC, B: CSR, parts: int, stream=None):
     """Balanced row-block boundaries (parts+1 int64) of C = A x B, computed on the GPU."""
     import numpy as np
@@ -283,6 +302,11 @@ def row_partition(A: CSC, B: CSR, parts: int, stream=None):
     _check(lib().spgemm_row_partition(ctypes.byref(a), ctypes.byref(b), parts,
                                       out.ctypes.data_as(ctypes.c_void_p), _stream(stream)))
     return out
+
+
+def trim_pool():
+    """Return the plans' cached device memory (stream-ordered pool) to the driver."""
+    _check(lib().spgemm_trim_pool())
 
 
 def set_timing(enable: bool):

@@ -354,6 +354,15 @@ void spgemm_default_options(spgemm_options_t *o) {
     o->validate = 1;
 }
 
+int spgemm_trim_pool(void) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    cudaMemPool_t pool = pool_for_device(dev);
+    CK(cudaDeviceSynchronize());
+    if (pool) CK(cudaMemPoolTrimTo(pool, 0));
+    return SPGEMM_OK;
+}
+
 int spgemm_set_timing(int32_t enable) {
     g_timing = enable != 0;
     return SPGEMM_OK;

@@ -324,6 +324,14 @@ def test_row_partition_and_row_blocks():
     assert_c_matches(C, inp)
 
 
+@pytest.mark.parametrize("parts", [1, 3, 8])
+def test_chunked_execution(parts):
+    """Chunked expansion (row blocks one after another on one GPU) gives the oracle's C."""
+    inp = synth.make_inputs("C1", seed=4)
+    A, B = spg.from_inputs(inp, "cuda")
+    assert_c_matches(spg.matmul_chunked(A, B, parts), inp)
+
+
 def test_empty_and_degenerate():
     for shape in [(5, 0, 7), (0, 4, 3), (3, 4, 0)]:
         m, k, n = shape
@@ -360,18 +368,23 @@ def test_validation_rejects_malformed():
 
 
 # ------------------------------------------------------------------ full sizes -------------
-@pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", FUSED), ("C3", {}), ("C4", {}), ("C5", {})])
+@pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", FUSED), ("C3", {}), ("C4", {}), ("C5", {}),
+                                       ("C5", {"chunks": 4})])
 def test_full_size_sampled(name, opts):
     """BASELINE.json configs[1] at full size, in the bench's launch configuration: sampled rows
     compared with the oracle one by one, plus whole-matrix properties."""
     inp = synth.make_inputs(name, seed=1)
     A, B = spg.from_inputs(inp, "cuda")
     torch.cuda.empty_cache()
-    with spg.Plan(A, B, **opts) as p:
-        st = p.stats()
-        C = p.execute()
     ca, rb, work = stages.pair_workload(inp)
-    assert st["nnz_chat"] == int(work.sum())
+    if "chunks" in opts:     # north star C5: chunked expansion (row blocks in turn)
+        spg.trim_pool()      # (earlier full-size products left their workspaces cached)
+        C = spg.matmul_chunked(A, B, opts["chunks"])
+    else:
+        with spg.Plan(A, B, **opts) as p:
+            st = p.stats()
+            C = p.execute()
+        assert st["nnz_chat"] == int(work.sum())
     # (C3 / C5 hold ~9e9 entries: everything below stays on the GPU but the sampled rows)
     rowptr = C.rowptr.cpu().numpy()
     assert rowptr[-1] == C.nnz
