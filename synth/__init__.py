@@ -84,6 +84,29 @@ def rmat_edges(scale: int, edge_factor: int, a: float, b: float, c: float, seed:
     return _dedupe(src, dst, 1 << scale)
 
 
+def rmat_n_edges(n: int, nedges: int, a: float, b: float, c: float, seed: int):
+    """R-MAT over n nodes (any n): draws in the 2^ceil(log2 n) square, rejects endpoints >= n until
+    nedges edges are drawn, then drops duplicates (Table III, R-MAT [29])."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    scale = max(1, int(np.ceil(np.log2(n))))
+    ab, abc = a + b, a + b + c
+    got_s, got_d, have = [], [], 0
+    while have < nedges:
+        m = int((nedges - have) * 1.3) + 1024
+        src = np.zeros(m, dtype=np.int64)
+        dst = np.zeros(m, dtype=np.int64)
+        for _ in range(scale):
+            u = rng.random(m)
+            src = (src << 1) | (u >= ab)
+            dst = (dst << 1) | (((u >= a) & (u < ab)) | (u >= abc))
+        ok = (src < n) & (dst < n)
+        src, dst = src[ok][: nedges - have], dst[ok][: nedges - have]
+        got_s.append(src)
+        got_d.append(dst)
+        have += src.size
+    return _dedupe(np.concatenate(got_s), np.concatenate(got_d), n)
+
+
 def _powerlaw_weights(n: int, m: float, gamma: float, wmax: float) -> np.ndarray:
     p = 1.0 / (gamma - 1.0)
     i = np.arange(n, dtype=np.float64)
@@ -204,6 +227,23 @@ CONFIGS = {
                desc="soc-LiveJournal-shaped power-law (4.8M nodes, 69M edges) C=AxA"),
 }
 
+# PAPER.md Table III synthetic sets (L739-L779): S (scalability), P (skewness), SP (sparsity) for
+# C = A^2 and AB15-AB18 (distinct R-MAT operands A, B; scale 15-18, edge factor 16) for C = AB.
+_S = (0.45, 0.15, 0.15)
+_U = (0.25, 0.25, 0.25)
+for _q, (_n, _m) in enumerate([(250_000, 62_500), (500_000, 250_000), (750_000, 562_500), (1_000_000, 1_000_000)]):
+    CONFIGS[f"S{_q + 1}"] = dict(kind="rmat_n", n=_n, m=_m, a=_S[0], b=_S[1], c=_S[2],
+                                 desc=f"Table III s{_q + 1}: R-MAT {_n} nodes, {_m} elements, (0.45,0.15,0.15,0.25) C=AxA")
+for _q, _p in enumerate([(0.25, 0.25, 0.25), (0.45, 0.15, 0.15), (0.55, 0.15, 0.15), (0.57, 0.19, 0.19)]):
+    CONFIGS[f"P{_q + 1}"] = dict(kind="rmat_n", n=1_000_000, m=1_000_000, a=_p[0], b=_p[1], c=_p[2],
+                                 desc=f"Table III p{_q + 1}: R-MAT 1M nodes, 1M elements, {_p + (round(1 - sum(_p), 2),)} C=AxA")
+for _q, _m in enumerate([4_000_000, 3_000_000, 2_000_000, 1_000_000]):
+    CONFIGS[f"SP{_q + 1}"] = dict(kind="rmat_n", n=1_000_000, m=_m, a=_U[0], b=_U[1], c=_U[2],
+                                  desc=f"Table III sp{_q + 1}: R-MAT 1M nodes, {_m} elements, uniform C=AxA")
+for _sc in (15, 16, 17, 18):
+    CONFIGS[f"AB{_sc}"] = dict(kind="rmat_ab", scale=_sc, edge_factor=16, a=0.57, b=0.19, c=0.19,
+                               desc=f"Table III C=AB: distinct R-MAT A, B (scale {_sc}, edge factor 16)")
+
 
 def make_inputs(name: str, seed: int = 1, values: str = "real", **override) -> SparseInputs:
     """Build the seeded C = A x A inputs of config ``name`` (A = B, both layouts)."""
@@ -217,6 +257,15 @@ def make_inputs(name: str, seed: int = 1, values: str = "real", **override) -> S
         n = cfg["n"]
         src, dst = chung_lu_edges(n, cfg["m"], cfg["gamma_out"], cfg["gamma_in"], cfg["max_out"],
                                   cfg["max_in"], cfg["sigma"], seed, cfg.get("symmetric", False))
+    elif kind == "rmat_n":
+        n = cfg["n"]
+        src, dst = rmat_n_edges(n, cfg["m"], cfg["a"], cfg["b"], cfg["c"], seed)
+    elif kind == "rmat_ab":   # C = A B with two independent R-MAT operands
+        n = 1 << cfg["scale"]
+        ar, ac = rmat_edges(cfg["scale"], cfg["edge_factor"], cfg["a"], cfg["b"], cfg["c"], seed)
+        br, bc = rmat_edges(cfg["scale"], cfg["edge_factor"], cfg["a"], cfg["b"], cfg["c"], seed + 1000)
+        return _pack(name, n, n, n, ar.astype(np.int32), ac.astype(np.int32), edge_values(ar, ac, seed, values),
+                     br.astype(np.int32), bc.astype(np.int32), edge_values(br, bc, seed + 1000, values))
     elif kind == "er":
         n = cfg["n"]
         src, dst = er_edges(n, cfg["per_row"], seed)

@@ -324,6 +324,16 @@ def test_row_partition_and_row_blocks():
     assert_c_matches(C, inp)
 
 
+@pytest.mark.parametrize("name", ["S1", "S2", "S3", "P1", "P2", "P3", "P4", "SP1", "SP2", "SP3", "SP4",
+                                  "AB15", "AB16"])
+def test_table3_synthetic(name):
+    """PAPER.md Table III synthetic sets (S / P / SP for C = A^2, AB for C = AB) against the
+    oracle's whole C."""
+    inp = synth.make_inputs(name, seed=1)
+    A, B = spg.from_inputs(inp, "cuda")
+    assert_c_matches(spg.matmul(A, B), inp)
+
+
 @pytest.mark.parametrize("parts", [1, 3, 8])
 def test_chunked_execution(parts):
     """Chunked expansion (row blocks one after another on one GPU) gives the oracle's C."""
@@ -369,7 +379,7 @@ def test_validation_rejects_malformed():
 
 # ------------------------------------------------------------------ full sizes -------------
 @pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", FUSED), ("C3", {}), ("C4", {}), ("C5", {}),
-                                       ("C5", {"chunks": 4})])
+                                       ("C5", {"chunks": 4}), ("AB17", {}), ("AB18", {})])
 def test_full_size_sampled(name, opts):
     """BASELINE.json configs[1] at full size, in the bench's launch configuration: sampled rows
     compared with the oracle one by one, plus whole-matrix properties."""

@@ -34,3 +34,18 @@ def test_row_slice():
     a = synth.make_inputs("C1", seed=2)
     s = synth.row_slice_coo(a, 100, 300)
     assert s.m == 200 and s.nnz_a == int(((a.a_rowidx >= 100) & (a.a_rowidx < 300)).sum())
+
+
+def test_table3_shapes():
+    """PAPER.md Table III: node counts and element counts (duplicates dropped) of the S / P / SP sets,
+    distinct operands for the C = AB sets."""
+    import numpy as np
+    for name in ["S1", "S2", "S3", "S4", "P1", "P2", "P3", "P4", "SP1", "SP2", "SP3", "SP4"]:
+        cfg = synth.CONFIGS[name]
+        inp = synth.make_inputs(name, seed=1)
+        assert inp.m == inp.k == inp.n == cfg["n"]
+        assert 0.99 * cfg["m"] <= inp.nnz_a <= cfg["m"]
+        np.testing.assert_array_equal(np.diff(inp.a_colptr).sum(), inp.nnz_b)   # A = B
+    inp = synth.make_inputs("AB15", seed=1)
+    assert inp.m == inp.k == inp.n == 1 << 15
+    assert inp.nnz_a != inp.nnz_b or not np.array_equal(inp.a_rowidx, inp.b_colidx)
