@@ -42,24 +42,43 @@ __global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64
     }
 }
 
-// B' = B with every row padded to a multiple of 4 slots (col = INT32_MAX, val = 0); one thread
-// per row, 16-byte stores (measured: a warp per 32 rows is 2x slower -- rows are short)
+// B' = B with every row padded to a multiple of 4 slots (col = INT32_MAX, val = 0), 16-byte
+// stores.  Lane per row for rows of <= 64 entries; the warp's longer rows (hub rows of thousands
+// of entries) are then copied by the whole warp, one after another (a thread per row alone left
+// AB18's 100K-entry rows on one thread: 1.2 ms).
+__device__ __forceinline__ void pad_b_vec(const int32_t *__restrict__ b_colidx, const float *__restrict__ b_val,
+                                          int64_t b0, int64_t rb, int64_t d0, int64_t j, int32_t *__restrict__ bp_col,
+                                          float *__restrict__ bp_val) {
+    int32_t c[4];
+    float v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+        c[u] = j + u < rb ? b_colidx[b0 + j + u] : 0x7fffffff;
+        v[u] = j + u < rb ? b_val[b0 + j + u] : 0.f;
+    }
+    *reinterpret_cast<int4 *>(bp_col + d0 + j) = make_int4(c[0], c[1], c[2], c[3]);
+    *reinterpret_cast<float4 *>(bp_val + d0 + j) = make_float4(v[0], v[1], v[2], v[3]);
+}
+
 __global__ void k_pad_b(const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ b_colidx,
                         const float *__restrict__ b_val, int64_t K, int32_t *__restrict__ bp_col,
                         float *__restrict__ bp_val) {
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t b0 = b_rowptr[k], rb = b_rowptr[k + 1] - b0;
-        const int64_t d0 = bp_start(b0, k);
-        for (int64_t j = 0; j < rb; j += 4) {
-            int32_t c[4];
-            float v[4];
-#pragma unroll
-            for (int u = 0; u < 4; ++u) {
-                c[u] = j + u < rb ? b_colidx[b0 + j + u] : 0x7fffffff;
-                v[u] = j + u < rb ? b_val[b0 + j + u] : 0.f;
-            }
-            *reinterpret_cast<int4 *>(bp_col + d0 + j) = make_int4(c[0], c[1], c[2], c[3]);
-            *reinterpret_cast<float4 *>(bp_val + d0 + j) = make_float4(v[0], v[1], v[2], v[3]);
+    const int lane = threadIdx.x & 31;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t kb = (int64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31); kb < K; kb += stride) {
+        const int64_t k = kb + lane;
+        int64_t b0 = 0, rb = 0;
+        if (k < K) { b0 = b_rowptr[k]; rb = b_rowptr[k + 1] - b0; }
+        const bool lng = rb > 64;
+        if (!lng)
+            for (int64_t j = 0; j < rb; j += 4) pad_b_vec(b_colidx, b_val, b0, rb, bp_start(b0, k), j, bp_col, bp_val);
+        unsigned m = __ballot_sync(0xffffffffu, lng);
+        while (m) {
+            const int l = __ffs(m) - 1;
+            m &= m - 1;
+            const int64_t kl = kb + l;
+            const int64_t bl = __shfl_sync(0xffffffffu, b0, l), rl = __shfl_sync(0xffffffffu, rb, l);
+            for (int64_t j = 4 * lane; j < rl; j += 128) pad_b_vec(b_colidx, b_val, bl, rl, bp_start(bl, kl), j, bp_col, bp_val);
         }
     }
 }

@@ -1583,6 +1583,14 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         } else {
             bool done_coarse = false;
             if (cap <= g.coarse_cap) {
+                long long t_c = clock64();
+                auto sub = [&](int slot) {   // coarse-path sub-phase clocks (tuning, reserved[1] = 3)
+                    if (g.prof && threadIdx.x == 0) {
+                        const long long t = clock64();
+                        atomicAdd(g.prof + slot, (unsigned long long)(t - t_c));
+                        t_c = t;
+                    }
+                };
                 // sparse long row: coarse column partition through global scratch (two coalesced passes)
                 //  1. histogram over kCoarseBins column ranges; greedy groups of <= kLimCap entries
                 //  2. scatter the row into the block's scratch, grouped by column range
@@ -1647,6 +1655,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                             if (gstart[gi] == 0x7fffffff) gstart[gi] = gstart[gi + 1];
                 }
                 __syncthreads();
+                sub(10);   // min/max, histogram, grouping
                 if (!s_bad) {   // (a single column range holding > kLimCap products: window path)
                     const int ng = s_ngroups;
                     int32_t *sc_col = g.scratch_col + (int64_t)blockIdx.x * g.stage_cap;
@@ -1674,6 +1683,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                         }
                     }
                     __syncthreads();
+                    sub(11);   // scatter into scratch
                     for (int gi = 0; gi < ng; ++gi) {
                         const int g0 = gstart[gi], n = gstart[gi + 1] - g0;
                         if (n == 0) continue;
@@ -1689,6 +1699,8 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     }
                     if (threadIdx.x == 0) g.ccount[i] = nout;
                     __syncthreads();
+                    sub(12);   // group sorts
+                    if (g.prof && threadIdx.x == 0) atomicAdd(g.prof + 13, (unsigned long long)ng);
                     done_coarse = true;
                 }
                 __syncthreads();

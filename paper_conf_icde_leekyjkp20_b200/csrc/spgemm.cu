@@ -604,7 +604,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     TRY(palloc(p, &p->bp_col, p->nnz_b + 7 * K + 4, s));
     TRY(palloc(p, &p->bp_val, p->nnz_b + 7 * K + 4, s));
     if (K > 0)
-        LAUNCH("pad_b", s, k_pad_b<<<grid_for(K, 256), 256, 0, s>>>(p->b_rowptr, p->b_colidx, p->b_val, K, p->bp_col,
+        LAUNCH("pad_b", s, k_pad_b<<<grid_for(cdiv(K, 32) * 32, 256), 256, 0, s>>>(p->b_rowptr, p->b_colidx, p->b_val, K, p->bp_col,
                                                                     p->bp_val));
     // limited rows: index map, run lists, B-Limited scratch
     p->nlim = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketLim0];
