@@ -127,6 +127,8 @@ struct spgemm_plan_s {
     const float *b_val = nullptr;
     std::vector<void *> owned;
     int64_t bytes = 0;
+    unsigned char *arena_ptr = nullptr;   // bump arena (arena_alloc)
+    size_t arena_left = 0;
     // stage 1
     int64_t *work = nullptr, *rowwork = nullptr, *rowoff = nullptr, *base = nullptr;
     int32_t *deg = nullptr;
@@ -177,37 +179,52 @@ struct spgemm_plan_s {
     int state = 0;  // 1 planned, 2 expanded, 3 merged
 };
 
+// Plan workspaces come from a bump arena over a few large pool blocks (>= kArenaBlock bytes each,
+// freed together by spgemm_destroy): ~60 workspace and temporary arrays per plan would otherwise
+// cost ~130 stream-ordered malloc / free calls of host time on every product.
+constexpr size_t kArenaBlock = (size_t)64 << 20;
+constexpr size_t kArenaAlign = 256;
+
+static int arena_alloc(spgemm_plan_s *p, size_t bytes, void **out, cudaStream_t s) {
+    bytes = (bytes + kArenaAlign - 1) & ~(kArenaAlign - 1);
+    if (p->arena_left < bytes) {
+        const size_t blk = std::max(bytes, kArenaBlock);
+        void *v = nullptr;
+        cudaError_t e = p->pool ? cudaMallocFromPoolAsync(&v, blk, p->pool, s) : cudaMallocAsync(&v, blk, s);
+        if (e != cudaSuccess)
+            return fail(SPGEMM_ERR_OUT_OF_MEMORY, std::string("device allocation of ") + std::to_string(blk) +
+                                                      " bytes failed: " + cudaGetErrorString(e));
+        p->owned.push_back(v);
+        p->bytes += (int64_t)blk;
+        if (blk > bytes && blk - bytes > p->arena_left) {   // keep whichever block has more room
+            p->arena_ptr = (unsigned char *)v + bytes;
+            p->arena_left = blk - bytes;
+        }
+        *out = v;
+        return SPGEMM_OK;
+    }
+    *out = p->arena_ptr;
+    p->arena_ptr += bytes;
+    p->arena_left -= bytes;
+    return SPGEMM_OK;
+}
+
 template <typename T>
 static int palloc(spgemm_plan_s *p, T **ptr, int64_t count, cudaStream_t s) {
-    size_t bytes = (size_t)std::max<int64_t>(count, 1) * sizeof(T);
     void *v = nullptr;
-    cudaError_t e = p->pool ? cudaMallocFromPoolAsync(&v, bytes, p->pool, s) : cudaMallocAsync(&v, bytes, s);
-    if (e != cudaSuccess)
-        return fail(SPGEMM_ERR_OUT_OF_MEMORY, std::string("device allocation of ") + std::to_string(bytes) +
-                                                  " bytes failed: " + cudaGetErrorString(e));
-    p->owned.push_back(v);
-    p->bytes += (int64_t)bytes;
+    TRY(arena_alloc(p, (size_t)std::max<int64_t>(count, 1) * sizeof(T), &v, s));
     *ptr = (T *)v;
     return SPGEMM_OK;
 }
 
-// temporary allocation freed at the end of the caller's scope (stream-ordered)
+// temporary of a call's scope: also from the arena (released with the plan)
 struct Temp {
-    void *v = nullptr;
-    cudaStream_t s;
-    explicit Temp(cudaStream_t st) : s(st) {}
-    ~Temp() {
-        if (v) cudaFreeAsync(v, s);
-    }
+    explicit Temp(cudaStream_t) {}
 };
 
 template <typename T>
-static int talloc(spgemm_plan_s *p, Temp &t, T **ptr, int64_t count) {
-    size_t bytes = (size_t)std::max<int64_t>(count, 1) * sizeof(T);
-    cudaError_t e = p->pool ? cudaMallocFromPoolAsync(&t.v, bytes, p->pool, t.s) : cudaMallocAsync(&t.v, bytes, t.s);
-    if (e != cudaSuccess) return fail(SPGEMM_ERR_OUT_OF_MEMORY, "temporary device allocation failed");
-    *ptr = (T *)t.v;
-    return SPGEMM_OK;
+static int talloc(spgemm_plan_s *p, Temp &, T **ptr, int64_t count) {
+    return palloc(p, ptr, count, p->last_stream);
 }
 
 static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -953,6 +970,7 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
     if (!C->rowptr || (p->nnz_c > 0 && (!C->colidx || !C->val)))
         return fail(SPGEMM_ERR_INVALID_ARGUMENT, "C arrays are NULL");
     cudaStream_t s = (cudaStream_t)stream;
+    p->last_stream = s;
     CK(cudaSetDevice(p->dev));
     C->nrows = p->m;
     C->ncols = p->n;
@@ -1088,6 +1106,8 @@ int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_
     CK(cudaDeviceSynchronize());
     const void *src = nullptr;
     int64_t bytes = 0;
+    unsigned char *arena_ptr = nullptr;   // bump arena (arena_alloc)
+    size_t arena_left = 0;
     std::vector<int64_t> tmp;
     switch (what) {
         case SPGEMM_VIEW_WORK: src = p->work; bytes = p->k * 8; break;
