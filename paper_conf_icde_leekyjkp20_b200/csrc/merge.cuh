@@ -633,14 +633,16 @@ struct RowMeta {
     int64_t s;    // first slot of the row's Ĉ bucket
     int32_t L;    // padded length
     int32_t i;    // row id
+    int32_t Lv;   // products (valid slots)
+    int32_t pad;
 };
 
 __global__ void k_row_meta(const int32_t *__restrict__ order, int64_t n, const int64_t *__restrict__ rowoff,
-                           RowMeta *__restrict__ meta) {
+                           const int64_t *__restrict__ rowwork, RowMeta *__restrict__ meta) {
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
         const int i = order[q];
         const int64_t s = rowoff[i];
-        meta[q] = RowMeta{s, (int32_t)(rowoff[i + 1] - s), i};
+        meta[q] = RowMeta{s, (int32_t)(rowoff[i + 1] - s), i, (int32_t)rowwork[i], 0};
     }
 }
 
@@ -660,7 +662,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
     int *hist = (int *)(slice + S::kCap * 16);
     const int64_t stride = (int64_t)gridDim.x * GROUPS;
     int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid;
-    const RowMeta none{0, 0, -1};
+    const RowMeta none{0, 0, -1, 0, 0};
     RowMeta m0 = r < nrows ? meta[r] : none;
     RowMeta m1 = r + stride < nrows ? meta[r + stride] : none;
     int32_t key[EPT];
@@ -1208,6 +1210,167 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_wmp(const int32_t *_
             if (lane == 0 && !out_col_all) ccount[i] = ob;
         }
         g.sync();
+    }
+}
+
+// Software-pipelined warp merge-path bin (rows of <= 256 slots, one warp per row, in place):
+// a warp holds the next row's slots (2 vectors per lane) in registers and the row after that's
+// (offset, length, id) from the meta table while it merges the current row -- C4's 2M rows of
+// 8 runs x 8 were one dependent memory round trip chain per row.
+template <int GROUPS>
+__global__ void __launch_bounds__(32 * GROUPS) k_merge_wmp_pipe(const RowMeta *__restrict__ meta, int64_t nrows,
+                                                                int32_t *__restrict__ chat_col,
+                                                                float *__restrict__ chat_val,
+                                                                int64_t *__restrict__ ccount) {
+    constexpr int CAP = 256;
+    using S = WmpSmem<CAP>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    const int gid = threadIdx.x >> 5, lane = lane_id();
+    unsigned char *slice = smem_raw + (size_t)gid * S::kBytes;
+    uint64_t *bufA = (uint64_t *)slice;
+    uint64_t *bufB = bufA + CAP;
+    int *runsA = (int *)(bufB + CAP);
+    int *runsB = runsA + S::kRuns;
+    const unsigned lt = lanemask_lt();
+    const int64_t stride = (int64_t)gridDim.x * GROUPS;
+    int64_t r = (int64_t)blockIdx.x * GROUPS + gid;
+    const RowMeta none{0, 0, -1, 0, 0};
+    RowMeta m0 = r < nrows ? meta[r] : none;
+    RowMeta m1 = r + stride < nrows ? meta[r + stride] : none;
+    auto load = [&](const RowMeta &m, int4 (&c)[2], float4 (&f)[2]) {
+        const int nv = m.L >> 2;
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+            const int v = 32 * u + lane;
+            c[u] = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
+            f[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (v < nv) {
+                c[u] = __ldcs(reinterpret_cast<const int4 *>(chat_col + m.s) + v);
+                f[u] = __ldcs(reinterpret_cast<const float4 *>(chat_val + m.s) + v);
+            }
+        }
+    };
+    int4 c[2];
+    float4 f[2];
+    load(m0, c, f);
+    while (r < nrows) {
+        int4 cn[2];
+        float4 fn[2];
+        load(m1, cn, fn);
+        const RowMeta m2 = r + 2 * stride < nrows ? meta[r + 2 * stride] : none;
+        const int Lp = m0.L, Lv = m0.Lv, nv = Lp >> 2;
+        // 1. pack + run starts (a run starts where a vector's first key is below the previous key)
+        int R = 0;
+        {
+            int32_t carry = kKeyPad;
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+                const int v = 32 * u + lane;
+                int32_t prev = __shfl_up_sync(kFull, c[u].w, 1);
+                if (lane == 0) prev = carry;
+                carry = __shfl_sync(kFull, c[u].w, 31);
+                const bool start = v < nv && (v == 0 || c[u].x < prev);
+                const unsigned m = __ballot_sync(kFull, start);
+                if (start) runsA[R + __popc(m & lt)] = 4 * v;
+                R += __popc(m);
+                if (v < nv) {
+                    ulonglong2 *d = reinterpret_cast<ulonglong2 *>(bufA + 4 * v);
+                    d[0] = make_ulonglong2(pack_kv(c[u].x, f[u].x), pack_kv(c[u].y, f[u].y));
+                    d[1] = make_ulonglong2(pack_kv(c[u].z, f[u].z), pack_kv(c[u].w, f[u].w));
+                }
+            }
+            if (lane == 0) runsA[R] = Lp;
+            __syncwarp();
+        }
+        // 2. merge levels (merge path per lane over E consecutive outputs)
+        uint64_t *src = bufA, *dst = bufB;
+        int *rs = runsA, *rd = runsB;
+        const int E = (Lp + 31) / 32;
+        while (R > 1) {
+            const int npairs = (R + 1) >> 1;
+            int o = min(Lp, lane * E);
+            const int oend = min(Lp, o + E);
+            if (o < oend) {
+                int lo = 0, hi = npairs;
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (rs[2 * mid] <= o) lo = mid; else hi = mid;
+                }
+                int q = lo;
+                while (o < oend) {
+                    const int a0 = rs[2 * q], a1 = rs[min(2 * q + 1, R)], b1 = rs[min(2 * q + 2, R)];
+                    const int d = o - a0;
+                    int ilo = max(0, d - (b1 - a1)), ihi = min(d, a1 - a0);
+                    while (ilo < ihi) {
+                        const int mi = (ilo + ihi) >> 1;
+                        if (kv_key(src[a0 + mi]) <= kv_key(src[a1 + d - mi - 1])) ilo = mi + 1; else ihi = mi;
+                    }
+                    int ia = a0 + ilo, jb = a1 + d - ilo;
+                    uint64_t xa = ia < a1 ? src[ia] : kKvMax;
+                    uint64_t xb = jb < b1 ? src[jb] : kKvMax;
+                    const int pend = min(oend, b1);
+                    for (; o < pend; ++o) {
+                        const bool tA = kv_key(xa) <= kv_key(xb);
+                        dst[o] = tA ? xa : xb;
+                        const int nxt = tA ? ia + 1 : jb + 1;
+                        const uint64_t y = nxt < (tA ? a1 : b1) ? src[nxt] : kKvMax;
+                        ia = tA ? nxt : ia;
+                        jb = tA ? jb : nxt;
+                        xa = tA ? y : xa;
+                        xb = tA ? xb : y;
+                    }
+                    ++q;
+                }
+            }
+            for (int q = lane; q <= npairs; q += 32) rd[q] = q < npairs ? rs[2 * q] : Lp;
+            __syncwarp();
+            { uint64_t *t = src; src = dst; dst = t; }
+            { int *t = rs; rs = rd; rd = t; }
+            R = npairs;
+        }
+        // 3. fp64 reduction of the sorted products (sentinels last), in place at the row head
+        int ob = 0;
+        int32_t *__restrict__ out_col = chat_col + m0.s;
+        float *__restrict__ out_val = chat_val + m0.s;
+        for (int p0 = 0; p0 < Lv; p0 += 32) {
+            const int p = p0 + lane;
+            const bool in = p < Lv;
+            const uint64_t x = in ? src[p] : kKvMax;
+            const int32_t k = kv_key(x);
+            int32_t prev = __shfl_up_sync(kFull, k, 1);
+            if (lane == 0) prev = p0 > 0 ? kv_key(src[p0 - 1]) : ~k;
+            int32_t next = __shfl_down_sync(kFull, k, 1);
+            if (lane == 31) next = p + 1 < Lv ? kv_key(src[p + 1]) : kKeyPad;
+            const bool head = in && k != prev;
+            const unsigned hm = __ballot_sync(kFull, head);
+            const bool dup = in && next == k;
+            if (hm == kFull && !__any_sync(kFull, dup)) {
+                out_col[ob + lane] = k;
+                out_val[ob + lane] = kv_val(x);
+                ob += 32;
+                continue;
+            }
+            double acc = (double)kv_val(x);
+            if (head && dup)
+                for (int q = p + 1; q < Lv; ++q) {
+                    const uint64_t y = src[q];
+                    if (kv_key(y) != k) break;
+                    acc += (double)kv_val(y);
+                }
+            if (head) {
+                const int o = ob + __popc(hm & lt);
+                out_col[o] = k;
+                out_val[o] = (float)acc;
+            }
+            ob += __popc(hm);
+        }
+        if (lane == 0) ccount[m0.i] = ob;
+        __syncwarp();
+#pragma unroll
+        for (int u = 0; u < 2; ++u) { c[u] = cn[u]; f[u] = fn[u]; }
+        m0 = m1;
+        m1 = m2;
+        r += stride;
     }
 }
 

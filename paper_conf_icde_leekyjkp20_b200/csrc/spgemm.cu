@@ -730,7 +730,8 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     const int64_t M = p->m;
     if (M > 0 && p->opt.reserved[0] != 7) {
         if (!p->row_meta) TRY(palloc(p, &p->row_meta, M, s));
-        LAUNCH("merge_meta", s, k_row_meta<<<grid_for(M, 256), 256, 0, s>>>(p->row_order, M, p->rowoff, p->row_meta));
+        LAUNCH("merge_meta", s, k_row_meta<<<grid_for(M, 256), 256, 0, s>>>(p->row_order, M, p->rowoff, p->rowwork,
+                                                                             p->row_meta));
     }
     if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
     auto rows_of = [&](int b0, int b1, int64_t *cnt) {
@@ -772,7 +773,17 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     if (variant == 6) {
     } else if (variant == 1) TRY(launch_wcs_bin<4, 2>(p, s, rows, cnt, "merge_wcs256"));
     else if (variant == 2) TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
-    else TRY(launch_wmp_bin<1, 8, 256>(p, s, rows, cnt, "merge_wmp256"));
+    else if (variant == 7) TRY(launch_wmp_bin<1, 8, 256>(p, s, rows, cnt, "merge_wmp256"));
+    else if (cnt > 0) {   // software-pipelined warp merge path
+        constexpr int G = 8;
+        const int smem = WmpSmem<256>::kBytes * G;
+        int occ = 0;
+        TRY(kernel_occupancy((const void *)k_merge_wmp_pipe<G>, smem, 32 * G, &occ));
+        const int64_t q0 = p->row_starts[kRowBucketWarp64];
+        const int64_t grid = std::min<int64_t>(cdiv(cnt, G), (int64_t)p->num_sms * std::max(occ, 1));
+        LAUNCH("merge_wmp256", s, k_merge_wmp_pipe<G><<<(unsigned)grid, 32 * G, smem, s>>>(
+            p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount));
+    }
     if (variant == 1) {
         rows = rows_of(kRowBucketSort512, kRowBucketSort1K + 1, &cnt);
         TRY(launch_wcs_bin<1, 8>(p, s, rows, cnt, "merge_wcs1k"));
