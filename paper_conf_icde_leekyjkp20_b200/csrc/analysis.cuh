@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(256) k_row_work(const int64_t *__restrict__ a_
                                                   const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
                                                   const int64_t *__restrict__ b_rowptr,
                                                   unsigned long long *__restrict__ rowwork, int32_t *__restrict__ deg,
-                                                  unsigned long long *__restrict__ rowcap, int64_t *__restrict__ base) {
+                                                  unsigned long long *__restrict__ rowcap) {
     int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
     if (e0 >= nnz_a) return;
     int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
@@ -135,15 +135,12 @@ __global__ void __launch_bounds__(256) k_row_work(const int64_t *__restrict__ a_
             kend = __ldg(a_colptr + k + 1);
             rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
         }
-        int64_t rel = -1;
         if (rb > 0) {
             int32_t i = a_rowidx[e];
             atomicAdd(rowwork + i, (unsigned long long)rb);
             atomicAdd(deg + i, 1);
-            // the padded-bucket counter's old value is the run's offset inside row i's bucket
-            if (rowcap) rel = (int64_t)atomicAdd(rowcap + i, (unsigned long long)pad_run(rb));
+            if (rowcap) atomicAdd(rowcap + i, (unsigned long long)pad_run(rb));
         }
-        if (base) base[e] = rel;   // made absolute by k_entry_pass once the row offsets exist
     }
 }
 
@@ -171,6 +168,28 @@ __global__ void __launch_bounds__(256) k_row_reduce(const int64_t *__restrict__ 
         atomicAdd(&sc->m_nonempty, a);
         atomicMax(&sc->max_rowwork, b);
         atomicMax(&sc->max_deg, c);
+    }
+}
+
+// Run bases: the run of products of A entry e = (i, k) occupies Ĉ positions
+// [base[e], base[e] + nnz(b_k*)) inside row i's bucket (cursor starts at rowoff[i]), followed
+// by pad_run(nnz(b_k*)) - nnz(b_k*) sentinel slots.
+__global__ void __launch_bounds__(256) k_run_base(const int64_t *__restrict__ a_colptr,
+                                                  const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
+                                                  const int64_t *__restrict__ b_rowptr,
+                                                  unsigned long long *__restrict__ cursor, int64_t *__restrict__ base) {
+    int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
+    if (e0 >= nnz_a) return;
+    int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
+    int64_t kend = __ldg(a_colptr + k + 1);
+    int64_t rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
+    for (int64_t e = e0; e < e0 + 8 && e < nnz_a; ++e) {
+        while (e >= kend) {
+            ++k;
+            kend = __ldg(a_colptr + k + 1);
+            rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
+        }
+        base[e] = rb > 0 ? (int64_t)atomicAdd(cursor + a_rowidx[e], (unsigned long long)pad_run(rb)) : -1;
     }
 }
 
@@ -383,34 +402,24 @@ __global__ void k_lim_index(const int32_t *__restrict__ rows, int64_t nlim, cons
     }
 }
 
-// Per A entry, after the row offsets and the limited-row index exist: base[e] (relative run
-// offset from k_row_work) += rowoff[i]; entries of limited rows also append their run
-// (base, length) to the row's run list.
-__global__ void __launch_bounds__(256) k_entry_pass(const int64_t *__restrict__ a_colptr,
-                                                    const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
-                                                    const int64_t *__restrict__ b_rowptr,
-                                                    const int64_t *__restrict__ rowoff, int64_t *__restrict__ base,
-                                                    const int32_t *__restrict__ lim_index,
-                                                    const int64_t *__restrict__ run_start, int32_t *__restrict__ run_fill,
-                                                    int64_t *__restrict__ run_base, int32_t *__restrict__ run_len) {
+__global__ void __launch_bounds__(256) k_lim_runs(const int64_t *__restrict__ a_colptr,
+                                                  const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
+                                                  const int64_t *__restrict__ b_rowptr,
+                                                  const int64_t *__restrict__ base, const int32_t *__restrict__ lim_index,
+                                                  const int64_t *__restrict__ run_start, int32_t *__restrict__ run_fill,
+                                                  int64_t *__restrict__ run_base, int32_t *__restrict__ run_len) {
     int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
     if (e0 >= nnz_a) return;
-    int64_t k = lim_index ? upper_bound_idx(a_colptr, 0, K, e0) : 0;
-    int64_t kend = lim_index ? __ldg(a_colptr + k + 1) : 0;
+    int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
+    int64_t kend = __ldg(a_colptr + k + 1);
     for (int64_t e = e0; e < e0 + 8 && e < nnz_a; ++e) {
+        while (e >= kend) { ++k; kend = __ldg(a_colptr + k + 1); }
+        int32_t li = lim_index[a_rowidx[e]];
         int64_t b = base[e];
-        if (b < 0) continue;
-        const int32_t i = a_rowidx[e];
-        b += __ldg(rowoff + i);
-        base[e] = b;
-        if (lim_index) {
-            const int32_t li = lim_index[i];
-            if (li >= 0) {
-                while (e >= kend) { ++k; kend = __ldg(a_colptr + k + 1); }
-                const int slot = atomicAdd(run_fill + li, 1);
-                run_base[run_start[li] + slot] = b;
-                run_len[run_start[li] + slot] = (int32_t)(__ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k));
-            }
+        if (li >= 0 && b >= 0) {
+            int slot = atomicAdd(run_fill + li, 1);
+            run_base[run_start[li] + slot] = b;
+            run_len[run_start[li] + slot] = (int32_t)(__ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k));
         }
     }
 }

@@ -513,11 +513,19 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         if (p->nnz_a > 0)
             LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
                 p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg,
-                (unsigned long long *)rowcap, p->base));
+                (unsigned long long *)rowcap));
         TRY(scan_excl(p, rowcap, M, p->rowoff, s, "row_offsets"));   // padded bucket offsets
     }
     if (M > 0)
         LAUNCH("row_reduce", s, k_row_reduce<<<grid_for(M, 256, p->num_sms * 8), 256, 0, s>>>(p->rowwork, p->deg, M, p->scal));
+    if (p->nnz_a > 0) {
+        Temp tc(s);
+        unsigned long long *cursor;
+        TRY(talloc(p, tc, &cursor, M));
+        CK(cudaMemcpyAsync(cursor, p->rowoff, M * 8, cudaMemcpyDeviceToDevice, s));
+        LAUNCH("run_base", s, k_run_base<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, cursor, p->base));
+    }
     CK(cudaMemcpyAsync(&p->h_scal, p->scal, sizeof(PlanScalars), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&p->chat_cap, p->rowoff + M, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));  // sync 1: nnz(Ĉ) both ways, Ĉ capacity, #non-empty blocks
@@ -637,6 +645,9 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         p->lim_max_L = (int64_t)p->h_scal.lim_max_L;
         TRY(palloc(p, &p->run_base, p->lim_runs, s));
         TRY(palloc(p, &p->run_len, p->lim_runs, s));
+        LAUNCH("lim_runs", s, k_lim_runs<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->base, p->lim_index, p->run_start, p->run_fill,
+            p->run_base, p->run_len));
         p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
         p->stage_cap = p->lim_max_L;   // whole-row scratch (dense rows are regrouped by window)
         TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
@@ -646,11 +657,6 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
         TRY(palloc(p, &p->row_counter, 1, s));
     }
-    // absolute run bases (+ run lists of the limited rows)
-    if (p->nnz_a > 0)
-        LAUNCH("entry_pass", s, k_entry_pass<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
-            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->rowoff, p->base, p->nlim > 0 ? p->lim_index : nullptr,
-            p->run_start, p->run_fill, p->run_base, p->run_len));
     // merge state; Ĉ itself is allocated by spgemm_expand (or is the caller's C, spgemm_execute)
     const bool fused = p->opt.reserved[0] == kMergeFused;
     p->long_slots = fused ? (int64_t)p->h_scal.long_slots : 0;
@@ -1192,8 +1198,7 @@ int spgemm_row_partition(const spgemm_csc_t *A, const spgemm_csr_t *B, int32_t p
         }
         if (A->nnz > 0)
             LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(A->nnz, 8), 256), 256, 0, s>>>(
-                p->a_colptr, p->a_rowidx, K, A->nnz, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg, nullptr,
-                nullptr));
+                p->a_colptr, p->a_rowidx, K, A->nnz, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg, nullptr));
         TRY(scan_excl(p, p->rowwork, M, p->rowoff, s, "row_offsets"));
         LAUNCH("partition_bounds", s, k_partition_bounds<<<(unsigned)cdiv(parts + 1, 128), 128, 0, s>>>(p->rowoff, M, parts, bounds));
         CK(cudaMemcpyAsync(bounds_host, bounds, (parts + 1) * 8, cudaMemcpyDeviceToHost, s));
