@@ -363,6 +363,8 @@ def run_reference(args, ws, rank):
     """--impl reference: the oracle (this tier's reference arm) on the host cores."""
     if ws > 1 and rank != 0:
         return
+    if ws > 1:   # torchrun pins OMP_NUM_THREADS=1; rank 0 alone times the oracle on the host cores
+        os.environ["OMP_NUM_THREADS"] = str(os.cpu_count() or 1)
     import synth
     import oracle
     inp = synth.make_inputs(args.config, seed=args.seed)
