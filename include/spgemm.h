@@ -112,7 +112,17 @@ typedef struct {
     int32_t enable_gather;
     int32_t enable_limit;
     int32_t validate;         /* check input structure in spgemm_plan (default 1)               */
-    int32_t reserved[16];
+    int32_t reserved[16];     /* tuning / comparison knobs, 0 = default:
+                                 [0] merge variant: 1 register-staged counting sort, 2 bucket sort
+                                     everywhere, 3 merge path everywhere, 4 fused unit merge (C
+                                     placed by decoupled look-back, see spgemm_execute), 6 register
+                                     bitonic <= 256 slots, 7 no software pipelining, 8 pipelined
+                                     2K / 4K bins too;
+                                 [1] profiling: 1 unit merge without look-back (wrong C, timing
+                                     only), 2 unit-merge phase clocks, 3 B-Limited path clocks
+                                     (SPGEMM_VIEW_UNIT_PROFILE);
+                                 [2] 1 = per-row compaction kernels instead of the chunked one;
+                                 [3] 1 = row-product expansion (the paper's comparison order)   */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */
@@ -175,7 +185,10 @@ int spgemm_merge(spgemm_plan_t plan, void *stream, int64_t *nnz_c);
 int spgemm_output(spgemm_plan_t plan, spgemm_csr_out_t *C, void *stream);
 
 /* expand + merge + alloc(C arrays in `out_where`) + output.  C->rowptr/colidx/val are
- * set to the allocated buffers (owned by the caller).  Returns after `stream` holds C. */
+ * set to the allocated buffers (owned by the caller).  Returns after `stream` holds C.
+ * With the fused unit merge (options.reserved[0] = 4) and a device C, colidx / val are requested
+ * before the expansion with capacity nnz(Ĉ) (padded) >= nnz(C): they hold Ĉ during the merge and C
+ * in their first nnz(C) entries afterwards (C->nnz). */
 int spgemm_execute(spgemm_plan_t plan, spgemm_alloc_fn alloc, void *alloc_ctx, int32_t out_where,
                    spgemm_csr_out_t *C, void *stream);
 
