@@ -1124,8 +1124,6 @@ int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_
     CK(cudaDeviceSynchronize());
     const void *src = nullptr;
     int64_t bytes = 0;
-    unsigned char *arena_ptr = nullptr;   // bump arena (arena_alloc)
-    size_t arena_left = 0;
     std::vector<int64_t> tmp;
     switch (what) {
         case SPGEMM_VIEW_WORK: src = p->work; bytes = p->k * 8; break;
