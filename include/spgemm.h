@@ -117,7 +117,7 @@ typedef struct {
                                      everywhere, 3 merge path everywhere, 4 fused unit merge (C
                                      placed by decoupled look-back, see spgemm_execute), 6 register
                                      bitonic <= 256 slots, 7 no software pipelining, 8 pipelined
-                                     2K / 4K bins too;
+                                     2K / 4K bins too, 10 bucket-owner insertion sort;
                                  [1] profiling: 1 unit merge without look-back (wrong C, timing
                                      only), 2 unit-merge phase clocks, 3 B-Limited path clocks
                                      (SPGEMM_VIEW_UNIT_PROFILE);

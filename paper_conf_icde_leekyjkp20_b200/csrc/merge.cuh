@@ -443,6 +443,101 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
                                                        int *sc);
 
+// Bucket-owner variant: after the scatter, every thread owns the contiguous bucket range it
+// scanned, insertion-sorts its multi-key buckets in place and reduces them (equal keys never
+// leave a bucket) into the head of its slot range; a group scan of the per-thread counts places
+// them and each warp copies its lanes' ranges out coalesced.  No second (dk2, dv2) buffer and no
+// per-element ranking loop.  Returns -1 on a bucket of > kBucketMax keys.
+template <int NW, int GROUPS, int EPT>
+__device__ __forceinline__ int bucket_walk_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
+                                                       float (&val)[EPT], int L, int32_t *dk, float *dv, int *hist,
+                                                       int32_t *out_col, float *out_val, int *sc) {
+    constexpr int T = NW * 32;
+    int32_t mn = kKeyPad, mx = 0;
+#pragma unroll
+    for (int e = 0; e < EPT; ++e)
+        if (key[e] != kKeyPad) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
+    mn = g.reduce_min(mn, sc);
+    mx = g.reduce_max(mx, sc);
+    const uint32_t span = (uint32_t)(mx - mn);
+    const int lognb = nextpow2_log(L);
+    const int nb = 1 << lognb;
+    const int bits = span ? 32 - __clz(span) : 0;
+    const int sh = max(0, bits - lognb);
+    for (int b = g.gtid; b <= hidx(nb); b += T) hist[b] = 0;
+    g.sync();
+    int rk[EPT];
+#pragma unroll
+    for (int e = 0; e < EPT; ++e)
+        rk[e] = key[e] != kKeyPad ? atomicAdd(&hist[hidx((key[e] - mn) >> sh)], 1) : 0;
+    g.sync();
+    const int bpt = (nb + T - 1) / T;
+    const int b0 = min(nb, g.gtid * bpt), b1 = min(nb, b0 + bpt);
+    int cnt = 0, mxc = 0;
+    for (int b = b0; b < b1; ++b) {
+        const int c = hist[hidx(b)];
+        cnt += c;
+        mxc = max(mxc, c);
+    }
+    int tot;
+    int ex = g.excl_sum(cnt, sc, &tot);
+    if (g.reduce_max(mxc, sc) > kBucketMax) return -1;
+    const int S = ex, E = ex + cnt;
+    for (int b = b0; b < b1; ++b) {
+        const int c = hist[hidx(b)];
+        hist[hidx(b)] = ex;
+        ex += c;
+    }
+    if (g.gtid == 0) hist[hidx(nb)] = tot;
+    g.sync();
+#pragma unroll
+    for (int e = 0; e < EPT; ++e)
+        if (key[e] != kKeyPad) {
+            const int pos = hist[hidx((key[e] - mn) >> sh)] + rk[e];
+            dk[pos] = key[e];
+            dv[pos] = val[e];
+        }
+    g.sync();
+    // owner walk: sort each multi-key bucket (insertion), then reduce the range in place
+    {
+        int bs = S;
+        for (int b = b0; b < b1; ++b) {
+            const int be = b + 1 < b1 ? hist[hidx(b + 1)] : E;
+            for (int p = bs + 1; p < be; ++p) {
+                const int32_t kk = dk[p];
+                const float vv = dv[p];
+                int q = p - 1;
+                while (q >= bs && dk[q] > kk) { dk[q + 1] = dk[q]; dv[q + 1] = dv[q]; --q; }
+                dk[q + 1] = kk;
+                dv[q + 1] = vv;
+            }
+            bs = be;
+        }
+    }
+    int u = 0;
+    {
+        int32_t cur = -1;
+        double acc = 0.0;
+        for (int p = S; p < E; ++p) {
+            const int32_t k = dk[p];
+            const float v = dv[p];
+            if (k != cur) {
+                if (cur != -1) { dk[S + u] = cur; dv[S + u] = (float)acc; ++u; }
+                cur = k;
+                acc = (double)v;
+            } else {
+                acc += (double)v;
+            }
+        }
+        if (cur != -1) { dk[S + u] = cur; dv[S + u] = (float)acc; ++u; }
+    }
+    int U;
+    const int o = g.excl_sum(u, sc, &U);
+    const int64_t wbase = __shfl_sync(kFull, o, 0);
+    warp_copy_out(S, u, wbase, dk, dv, out_col, out_val);
+    return U;
+}
+
 // LS: buckets = 2^LS x (slots rounded up to a power of two); more buckets, fewer shared ones
 template <int NW, int GROUPS, int EPT, int LS = 0>
 __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
@@ -646,7 +741,7 @@ __global__ void k_row_meta(const int32_t *__restrict__ order, int64_t n, const i
     }
 }
 
-template <int NW, int GROUPS, int EPT, int LS = 0>
+template <int NW, int GROUPS, int EPT, int LS = 0, bool WALK = false>
 __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k_merge_bucket_pipe(
     const RowMeta *__restrict__ meta, int64_t nrows, int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
     int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows, unsigned *__restrict__ fb_count) {
@@ -674,9 +769,13 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
         bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, min(m1.L, S::kCap), kn, vn);
         const RowMeta m2 = r + 2 * stride < nrows ? meta[r + 2 * stride] : none;
         if (m0.L <= S::kCap) {
-            const int U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
-                                                                       chat_col + m0.s, chat_val + m0.s,
-                                                                       sc_all[g.gid]);
+            int U;
+            if constexpr (WALK)
+                U = bucket_walk_reduce_regs<NW, GROUPS, EPT>(g, key, val, m0.L, dk, dv, hist, chat_col + m0.s,
+                                                             chat_val + m0.s, sc_all[g.gid]);
+            else
+                U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
+                                                                 chat_col + m0.s, chat_val + m0.s, sc_all[g.gid]);
             if (g.gtid == 0) {
                 if (U >= 0) ccount[m0.i] = U;
                 else fb_rows[atomicAdd(fb_count, 1u)] = m0.i;

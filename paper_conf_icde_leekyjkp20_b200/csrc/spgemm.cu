@@ -293,16 +293,17 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
 }
 
 // software-pipelined in-place bucket bin over rows [b0, b1) of row_order (meta table in p->row_meta)
-template <int NW, int GROUPS, int EPT>
+template <int NW, int GROUPS, int EPT, bool WALK = false>
 static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int64_t cnt, const char *name,
                               int ctas_per_sm) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, 0>::kBytes * GROUPS;
+    auto kern = k_merge_bucket_pipe<NW, GROUPS, EPT, 0, WALK>;
     int occ = 0;
-    TRY(kernel_occupancy((const void *)k_merge_bucket_pipe<NW, GROUPS, EPT>, smem, NW * 32 * GROUPS, &occ));
+    TRY(kernel_occupancy((const void *)kern, smem, NW * 32 * GROUPS, &occ));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
     (void)ctas_per_sm;
-    LAUNCH(name, s, k_merge_bucket_pipe<NW, GROUPS, EPT><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
+    LAUNCH(name, s, kern<<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
         p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
     return SPGEMM_OK;
 }
@@ -802,6 +803,11 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         TRY(launch_bucket_bin<2, 4, 8>(p, s, rows, cnt, "merge_bucket512", 8));
         rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
         TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
+    } else if (variant == 10) {   // bucket-owner insertion sort + walk reduction
+        const int64_t q = p->row_starts[kRowBucketSort512];
+        TRY(launch_bucket_pipe<2, 4, 8, true>(p, s, q, p->row_starts[kRowBucketSort512 + 1] - q, "merge_bucket512", 8));
+        const int64_t q2 = p->row_starts[kRowBucketSort1K];
+        TRY(launch_bucket_pipe<4, 2, 8, true>(p, s, q2, p->row_starts[kRowBucketSort1K + 1] - q2, "merge_bucket1k", 8));
     } else {
         const int64_t q = p->row_starts[kRowBucketSort512];
         TRY(launch_bucket_pipe<2, 4, 8>(p, s, q, p->row_starts[kRowBucketSort512 + 1] - q, "merge_bucket512", 8));

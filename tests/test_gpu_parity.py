@@ -78,6 +78,7 @@ CASES = [
     ("C1", dict(reserved=(6,) + (0,) * 15)),   # merge variant: register bitonic for <= 256 slots
     ("C1", dict(reserved=(7,) + (0,) * 15)),   # merge variant: bucket bins without pipelining
     ("C1", dict(reserved=(8,) + (0,) * 15)),   # merge variant: all bucket bins pipelined
+    ("C1", dict(reserved=(10,) + (0,) * 15)),  # merge variant: bucket-owner insertion sort
     ("C1", dict(reserved=(0, 0, 0, 1) + (0,) * 12)),   # row-product expansion (comparison order)
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
@@ -226,6 +227,7 @@ def test_random_tiny(shape, dens, seed, skew, values):
     A, B = spg.from_inputs(inp, "cuda")
     for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(1,) + (0,) * 15),
                  dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15), FUSED, dict(reserved=(6,) + (0,) * 15),
+                 dict(reserved=(10,) + (0,) * 15),
                  dict(beta=1000.0, piece_work=64, split_ca_max=3, **FUSED)):
         C = spg.matmul(A, B, **opts)
         assert_c_matches(C, inp, signed=(values == "signed"))
