@@ -107,4 +107,49 @@ __device__ __forceinline__ int64_t upper_bound_idx(const int64_t *__restrict__ p
 __device__ __forceinline__ int ilog2_floor(uint64_t x) { return 63 - __clzll((long long)x); }
 __device__ __forceinline__ int ilog2_ceil(uint64_t x) { return x <= 1 ? 0 : 64 - __clzll((long long)(x - 1)); }
 
+// ---- decoupled look-back (single-pass scans, the fused unit merge): a status word per tile,
+// flag in the top 2 bits (1 aggregate, 2 inclusive prefix), value in the low 62.
+constexpr unsigned long long kLbAgg = 1ull << 62, kLbPre = 2ull << 62, kLbMask = (1ull << 62) - 1;
+
+__device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Decoupled look-back (one warp).  lb_publish: unit u's aggregate (unit 0: its inclusive
+// prefix) as soon as its merged count is known; lb_resolve (later): sums predecessors'
+// aggregates back to the nearest inclusive prefix, publishes u's inclusive prefix and returns the
+// exclusive one.
+__device__ __forceinline__ void lb_publish(unsigned long long *status, int64_t u, int64_t agg) {
+    __threadfence();
+    if (lane_id() == 0) st_release_u64(status + u, (u == 0 ? kLbPre : kLbAgg) | (unsigned long long)agg);
+}
+__device__ __forceinline__ int64_t lb_resolve(unsigned long long *status, int64_t u, int64_t agg) {
+    if (u == 0) return 0;
+    const int lane = lane_id();
+    int64_t excl = 0;
+    int64_t idx = u - 1 - lane;
+    while (true) {
+        unsigned long long s;
+        do {
+            s = idx >= 0 ? ld_acquire_u64(status + idx) : kLbPre;
+        } while (__any_sync(0xffffffffu, (s >> 62) == 0));
+        const unsigned pre = __ballot_sync(0xffffffffu, (s >> 62) == 2);
+        int64_t v = (int64_t)(s & kLbMask);
+        if (pre) {
+            if (lane > __ffs(pre) - 1) v = 0;
+            excl += warp_sum(v);
+            break;
+        }
+        excl += warp_sum(v);
+        idx -= 32;
+    }
+    if (lane == 0) st_release_u64(status + u, kLbPre | (unsigned long long)(excl + agg));
+    return excl;
+}
+
 }  // namespace spg

@@ -35,7 +35,6 @@ constexpr int kUnitCap = 4096;                       // slots of one unit (share
 constexpr int kUnitThreads = 256;                    // threads per unit CTA (also max rows per unit)
 constexpr int kUnitWindow = kUnitCap - kUnitRowMax;  // window of unit starts on the Ĉ offsets
 constexpr int kUnitNbMax = 2 * kUnitCap;             // sum over rows of nextpow2(L) <= 2 * slots
-constexpr unsigned long long kLbAgg = 1ull << 62, kLbPre = 2ull << 62, kLbMask = (1ull << 62) - 1;
 
 __host__ __device__ __forceinline__ bool unit_long_row(int64_t cap, int8_t cls) {
     return cap > kUnitRowMax || cls == RC_LIMITED;
@@ -66,47 +65,6 @@ __global__ void k_unit_rows(const int32_t *__restrict__ flag, const int64_t *__r
             *nunits = uoff[M];
         }
     }
-}
-
-__device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned long long v) {
-    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-
-// Decoupled look-back (one warp).  lb_publish: unit u's aggregate (unit 0: its inclusive
-// prefix) as soon as its merged count is known; lb_resolve (later): sums predecessors'
-// aggregates back to the nearest inclusive prefix, publishes u's inclusive prefix and returns the
-// exclusive one.
-__device__ __forceinline__ void lb_publish(unsigned long long *status, int64_t u, int64_t agg) {
-    __threadfence();
-    if (lane_id() == 0) st_release_u64(status + u, (u == 0 ? kLbPre : kLbAgg) | (unsigned long long)agg);
-}
-__device__ __forceinline__ int64_t lb_resolve(unsigned long long *status, int64_t u, int64_t agg) {
-    if (u == 0) return 0;
-    const int lane = lane_id();
-    int64_t excl = 0;
-    int64_t idx = u - 1 - lane;
-    while (true) {
-        unsigned long long s;
-        do {
-            s = idx >= 0 ? ld_acquire_u64(status + idx) : kLbPre;
-        } while (__any_sync(kFull, (s >> 62) == 0));
-        const unsigned pre = __ballot_sync(kFull, (s >> 62) == 2);
-        int64_t v = (int64_t)(s & kLbMask);
-        if (pre) {
-            if (lane > __ffs(pre) - 1) v = 0;
-            excl += warp_sum(v);
-            break;
-        }
-        excl += warp_sum(v);
-        idx -= 32;
-    }
-    if (lane == 0) st_release_u64(status + u, kLbPre | (unsigned long long)(excl + agg));
-    return excl;
 }
 
 struct UnitArgs {

@@ -8,62 +8,42 @@ constexpr int kScanThreads = 256;
 constexpr int kScanItems = 8;
 constexpr int kScanTile = kScanThreads * kScanItems;  // 2048
 
-// Pass 1: per-tile sums (striped, coalesced loads).
+// Single-pass exclusive scan (decoupled look-back): tiles claimed in order by a ticket, each
+// publishes its sum, resolves its prefix from its predecessors and writes out[]; out[n] = total.
+// status[] (ntiles words) and ticket must be zero.
 template <typename Tin>
-__global__ void __launch_bounds__(kScanThreads) k_scan_tile_sums(const Tin *__restrict__ in, int64_t n,
-                                                                 int64_t *__restrict__ tile_sums) {
+__global__ void __launch_bounds__(kScanThreads) k_scan_onepass(const Tin *__restrict__ in, int64_t n,
+                                                               int64_t *__restrict__ out,
+                                                               unsigned long long *__restrict__ status,
+                                                               unsigned long long *__restrict__ ticket) {
     __shared__ int64_t sm[kScanThreads / 32 + 1];
-    const int64_t base = (int64_t)blockIdx.x * kScanTile;
-    int64_t s = 0;
+    __shared__ int64_t s_tile, s_pre;
+    if (threadIdx.x == 0) s_tile = (int64_t)atomicAdd(ticket, 1ull);
+    __syncthreads();
+    const int64_t tile = s_tile;
+    const int64_t b0 = tile * kScanTile + (int64_t)threadIdx.x * kScanItems;
+    int64_t v[kScanItems];
+    int64_t local = 0;
 #pragma unroll
     for (int j = 0; j < kScanItems; ++j) {
-        int64_t idx = base + j * kScanThreads + threadIdx.x;
-        if (idx < n) s += (int64_t)in[idx];
+        v[j] = b0 + j < n ? (int64_t)in[b0 + j] : 0;
+        local += v[j];
     }
-    s = warp_sum(s);
-    if (lane_id() == 0) sm[warp_id()] = s;
+    int64_t tot;
+    const int64_t ex = block_excl_sum<kScanThreads>(local, sm, &tot);
+    if (warp_id() == 0) {
+        lb_publish(status, tile, tot);
+        const int64_t pre = lb_resolve(status, tile, tot);
+        if (lane_id() == 0) s_pre = pre;
+    }
     __syncthreads();
-    if (threadIdx.x == 0) {
-        int64_t t = 0;
-        for (int w = 0; w < kScanThreads / 32; ++w) t += sm[w];
-        tile_sums[blockIdx.x] = t;
-    }
-}
-
-// Pass 2: exclusive scan of the tile sums in place (one block, chunked with carry);
-// tile_sums[ntiles] receives the grand total.
-__global__ void __launch_bounds__(1024) k_scan_spine(int64_t *__restrict__ tile_sums, int64_t ntiles) {
-    __shared__ int64_t sm[1024 / 32 + 1];
-    int64_t carry = 0;
-    for (int64_t base = 0; base < ntiles; base += 1024) {
-        int64_t idx = base + threadIdx.x;
-        int64_t v = idx < ntiles ? tile_sums[idx] : 0;
-        int64_t tot;
-        int64_t ex = block_excl_sum<1024>(v, sm, &tot);
-        if (idx < ntiles) tile_sums[idx] = carry + ex;
-        carry += tot;
-    }
-    if (threadIdx.x == 0) tile_sums[ntiles] = carry;
-}
-
-// Pass 3: out[i] = tile_offset + exclusive prefix within the tile; out[n] = total.
-template <typename Tin>
-__global__ void __launch_bounds__(kScanThreads) k_scan_apply(const Tin *__restrict__ in, int64_t n,
-                                                             const int64_t *__restrict__ tile_off,
-                                                             int64_t *__restrict__ out, int64_t ntiles) {
-    __shared__ int64_t sm[kScanThreads / 32 + 1];
-    const int64_t base = (int64_t)blockIdx.x * kScanTile;
-    int64_t carry = tile_off[blockIdx.x];
-#pragma unroll 1
+    int64_t run = s_pre + ex;
+#pragma unroll
     for (int j = 0; j < kScanItems; ++j) {
-        int64_t idx = base + j * kScanThreads + threadIdx.x;
-        int64_t v = idx < n ? (int64_t)in[idx] : 0;
-        int64_t tot;
-        int64_t ex = block_excl_sum<kScanThreads>(v, sm, &tot);
-        if (idx < n) out[idx] = carry + ex;
-        carry += tot;
+        if (b0 + j < n) out[b0 + j] = run;
+        run += v[j];
     }
-    if (blockIdx.x == ntiles - 1 && threadIdx.x == 0) out[n] = tile_off[ntiles];
+    if (threadIdx.x == 0 && (tile + 1) * kScanTile >= n) out[n] = s_pre + tot;
 }
 
 // Stable partition by a per-item bucket id (< nb <= 255).  Tile = one 256-thread block.

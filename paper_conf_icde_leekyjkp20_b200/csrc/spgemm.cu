@@ -264,11 +264,10 @@ static int scan_excl(spgemm_plan_s *p, const Tin *in, int64_t n, int64_t *out, c
     }
     const int64_t ntiles = cdiv(n, kScanTile);
     Temp t(s);
-    int64_t *ts;
-    TRY(talloc(p, t, &ts, ntiles + 1));
-    LAUNCH(name, s, k_scan_tile_sums<Tin><<<(unsigned)ntiles, kScanThreads, 0, s>>>(in, n, ts));
-    LAUNCH(name, s, k_scan_spine<<<1, 1024, 0, s>>>(ts, ntiles));
-    LAUNCH(name, s, k_scan_apply<Tin><<<(unsigned)ntiles, kScanThreads, 0, s>>>(in, n, ts, out, ntiles));
+    unsigned long long *st;   // [ntiles] look-back words + ticket
+    TRY(talloc(p, t, &st, ntiles + 1));
+    CK(cudaMemsetAsync(st, 0, (ntiles + 1) * 8, s));
+    LAUNCH(name, s, k_scan_onepass<Tin><<<(unsigned)ntiles, kScanThreads, 0, s>>>(in, n, out, st, st + ntiles));
     return SPGEMM_OK;
 }
 
