@@ -344,6 +344,37 @@ def test_chunked_execution(parts):
     assert_c_matches(spg.matmul_chunked(A, B, parts), inp)
 
 
+def test_repeated_plans_and_concurrent_streams():
+    """Plans are single-use and independent: 20 products in a row keep the same workspace size, and
+    two host threads running products on two streams at once both match the oracle."""
+    import threading
+    inp = synth.make_inputs("C1", seed=6)
+    A, B = spg.from_inputs(inp, "cuda")
+    sizes = []
+    for _ in range(20):
+        with spg.Plan(A, B) as p:
+            C = p.execute()
+            sizes.append(p.stats()["bytes_workspace"])
+    assert len(set(sizes)) == 1
+    assert_c_matches(C, inp)
+    out = [None, None]
+
+    def run(q):
+        st = torch.cuda.Stream()
+        with torch.cuda.stream(st):
+            out[q] = spg.matmul(A, B, stream=st)
+        st.synchronize()
+
+    ts = [threading.Thread(target=run, args=(q,)) for q in range(2)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    for q in range(2):
+        assert_c_matches(out[q], inp)
+    spg.trim_pool()
+
+
 def test_empty_and_degenerate():
     for shape in [(5, 0, 7), (0, 4, 3), (3, 4, 0)]:
         m, k, n = shape
