@@ -437,7 +437,7 @@ __device__ __forceinline__ void bsr_load(const Group<NW, GROUPS> &g, const int32
     }
 }
 
-template <int NW, int GROUPS, int EPT, int LS = 0>
+template <int NW, int GROUPS, int EPT, int LS = 0, bool UNR2 = false>
 __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
                                                        float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
@@ -538,19 +538,22 @@ __device__ __forceinline__ int bucket_walk_reduce_regs(const Group<NW, GROUPS> &
     return U;
 }
 
-// LS: buckets = 2^LS x (slots rounded up to a power of two); more buckets, fewer shared ones
-template <int NW, int GROUPS, int EPT, int LS = 0>
+// LS: buckets = 2^LS x (slots rounded up to a power of two); more buckets, fewer shared ones.
+// UNR2: in-bucket ranking two keys per step (the B-Limited groups' wider buckets: C3 -5 %; the
+// regular bins' mostly 2-key buckets are faster without)
+template <int NW, int GROUPS, int EPT, int LS = 0, bool UNR2 = false>
 __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
                                                   int L, int32_t *dk, float *dv, int32_t *dk2, float *dv2,
                                                   int *hist, int32_t *out_col, float *out_val, int *sc) {
     int32_t key[EPT];
     float val[EPT];
     bsr_load<NW, GROUPS, EPT>(g, sk, sv, L, key, val);
-    return bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, L, dk, dv, dk2, dv2, hist, out_col, out_val, sc);
+    return bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, UNR2>(g, key, val, L, dk, dv, dk2, dv2, hist, out_col, out_val,
+                                                              sc);
 }
 
 // the row already in registers (bsr_load; software-pipelined callers load the next row early)
-template <int NW, int GROUPS, int EPT, int LS>
+template <int NW, int GROUPS, int EPT, int LS, bool UNR2>
 __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
                                                        float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
@@ -614,11 +617,19 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
             const int bs = hist[hidx(b)], be = hist[hidx(b + 1)];
             const int32_t kk = key[e];
             int rank = 0;
-            if (be - bs > 1)     // (a bucket of one key is already in place)
-                for (int q = bs; q < be; ++q) {
+            if (be - bs > 1) {   // (a bucket of one key is already in place)
+                int q = bs;
+                if constexpr (UNR2)
+                    for (; q + 1 < be; q += 2) {
+                        const int32_t k0 = dk[q], k1 = dk[q + 1];
+                        rank += ((k0 < kk) | ((k0 == kk) & (q < pos[e]))) +
+                                ((k1 < kk) | ((k1 == kk) & (q + 1 < pos[e])));
+                    }
+                for (; q < be; ++q) {
                     const int32_t kq = dk[q];
                     rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
                 }
+            }
             dk2[bs + rank] = kk;
             dv2[bs + rank] = val[e];
         }
@@ -1645,7 +1656,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
             int32_t *dk2 = (int32_t *)(smem_raw + kLimCap * 8);
             float *dv2 = (float *)(smem_raw + kLimCap * 12);
             int *hist = (int *)(smem_raw + kLimCap * 16);
-            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
+            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
                                                             dv2, hist, oc, ov, sc);
             if (U < 0)
                 U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
@@ -1949,7 +1960,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     for (int gi = 0; gi < ng; ++gi) {
                         const int g0 = gstart[gi], n = gstart[gi + 1] - g0;
                         if (n == 0) continue;
-                        int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(
+                        int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(
                             grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + kLimCap * 4),
                             (int32_t *)(smem_raw + kLimCap * 8), (float *)(smem_raw + kLimCap * 12),
                             (int *)(smem_raw + kLimCap * 16), oc + nout, ov + nout, sc);
@@ -2049,7 +2060,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 cp_async_wait_all();
                 __syncthreads();
-                int U = bucket_sort_reduce<kLimNW, 1, kLimEPT>(grp, k0, v0, total, k0, v0,
+                int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(grp, k0, v0, total, k0, v0,
                                                                 (int32_t *)(smem_raw + kLimCap * 8),
                                                                 (float *)(smem_raw + kLimCap * 12),
                                                                 (int *)(smem_raw + kLimCap * 16), st_col + nout,
