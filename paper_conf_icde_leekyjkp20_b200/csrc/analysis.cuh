@@ -123,23 +123,35 @@ __global__ void __launch_bounds__(256) k_row_work(const int64_t *__restrict__ a_
                                                   const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
                                                   const int64_t *__restrict__ b_rowptr,
                                                   unsigned long long *__restrict__ rowwork, int32_t *__restrict__ deg,
-                                                  unsigned long long *__restrict__ rowcap) {
+                                                  unsigned long long *__restrict__ rowcap,
+                                                  const int32_t *__restrict__ b_colidx = nullptr,
+                                                  int32_t *__restrict__ rowmn = nullptr,
+                                                  int32_t *__restrict__ rowmx = nullptr) {
+    // rowmn / rowmx (optional): the exact column range of row i of C -- min / max over the stored
+    // a_ik of b_k*'s first / last column (B's rows are ascending): every product of the row is in
+    // it and its ends are attained, so the merge's bucket mapping needs no range reduction.
     int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
     if (e0 >= nnz_a) return;
     int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
     int64_t kend = __ldg(a_colptr + k + 1);
-    int64_t rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
+    int64_t rb0 = __ldg(b_rowptr + k), rb1 = __ldg(b_rowptr + k + 1);
     for (int64_t e = e0; e < e0 + 8 && e < nnz_a; ++e) {
         while (e >= kend) {
             ++k;
             kend = __ldg(a_colptr + k + 1);
-            rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
+            rb0 = rb1;
+            rb1 = __ldg(b_rowptr + k + 1);
         }
+        const int64_t rb = rb1 - rb0;
         if (rb > 0) {
             int32_t i = a_rowidx[e];
             atomicAdd(rowwork + i, (unsigned long long)rb);
             atomicAdd(deg + i, 1);
             if (rowcap) atomicAdd(rowcap + i, (unsigned long long)pad_run(rb));
+            if (rowmn) {
+                atomicMin(rowmn + i, __ldg(b_colidx + rb0));
+                atomicMax(rowmx + i, __ldg(b_colidx + rb1 - 1));
+            }
         }
     }
 }

@@ -48,6 +48,20 @@ __device__ __forceinline__ T warp_max(T v) {
     return v;
 }
 
+// 32-bit integer reductions: one REDUX instruction instead of five shuffle rounds
+template <>
+__device__ __forceinline__ int warp_sum<int>(int v) { return __reduce_add_sync(0xffffffffu, v); }
+template <>
+__device__ __forceinline__ int warp_min<int>(int v) { return __reduce_min_sync(0xffffffffu, v); }
+template <>
+__device__ __forceinline__ int warp_max<int>(int v) { return __reduce_max_sync(0xffffffffu, v); }
+template <>
+__device__ __forceinline__ unsigned warp_sum<unsigned>(unsigned v) { return __reduce_add_sync(0xffffffffu, v); }
+template <>
+__device__ __forceinline__ unsigned warp_min<unsigned>(unsigned v) { return __reduce_min_sync(0xffffffffu, v); }
+template <>
+__device__ __forceinline__ unsigned warp_max<unsigned>(unsigned v) { return __reduce_max_sync(0xffffffffu, v); }
+
 // Block-wide exclusive sum over THREADS threads; returns exclusive prefix, *total = sum.
 // `smem` needs THREADS/32 + 1 slots.  Contains __syncthreads (all threads must call).
 template <int THREADS, typename T>

@@ -247,6 +247,49 @@ struct Group {
             return r;
         }
     }
+    // excl_sum with a single barrier: every thread combines the warp totals itself.  The caller
+    // guarantees a group barrier between these reads of sc[0, NW) and the next write to them.
+    __device__ __forceinline__ int excl_sum1(int v, int *sc, int *total) const {
+        const int inc = warp_incl_sum(v);
+        if constexpr (NW == 1) {
+            *total = __shfl_sync(kFull, inc, 31);
+            return inc - v;
+        } else {
+            const int w = gtid >> 5;
+            if (lane_id() == 31) sc[w] = inc;
+            sync();
+            int before = 0, tot = 0;
+            if constexpr (NW <= 8) {
+#pragma unroll
+                for (int q = 0; q < NW; ++q) {
+                    const int t = sc[q];
+                    before += q < w ? t : 0;
+                    tot += t;
+                }
+            } else {
+                const int t = lane_id() < NW ? sc[lane_id()] : 0;
+                const int ci = warp_incl_sum(t);
+                before = __shfl_sync(kFull, ci - t, w);
+                tot = __shfl_sync(kFull, ci, NW - 1);
+            }
+            *total = tot;
+            return before + inc - v;
+        }
+    }
+    // min and max in one shared-memory round; `sc` needs 2 * NW + 1 ints
+    __device__ __forceinline__ void reduce_minmax(int &mn, int &mx, int *sc) const {
+        mn = warp_min(mn);
+        mx = warp_max(mx);
+        if constexpr (NW > 1) {
+            if (lane_id() == 0) { sc[gtid >> 5] = mn; sc[NW + 1 + (gtid >> 5)] = mx; }
+            sync();
+            int a = sc[0], b = sc[NW + 1];
+            for (int q = 1; q < NW; ++q) { a = min(a, sc[q]); b = max(b, sc[NW + 1 + q]); }
+            sync();
+            mn = a;
+            mx = b;
+        }
+    }
     __device__ __forceinline__ int reduce_max(int v, int *sc) const {
         v = warp_max(v);
         if constexpr (NW == 1) return v;
@@ -441,7 +484,7 @@ template <int NW, int GROUPS, int EPT, int LS = 0, bool UNR2 = false>
 __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
                                                        float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
-                                                       int *sc);
+                                                       int *sc, int32_t pmn = 1, int32_t pmx = 0);
 
 // Bucket-owner variant: after the scatter, every thread owns the contiguous bucket range it
 // scanned, insertion-sorts its multi-key buckets in place and reduces them (equal keys never
@@ -544,12 +587,13 @@ __device__ __forceinline__ int bucket_walk_reduce_regs(const Group<NW, GROUPS> &
 template <int NW, int GROUPS, int EPT, int LS = 0, bool UNR2 = false>
 __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv,
                                                   int L, int32_t *dk, float *dv, int32_t *dk2, float *dv2,
-                                                  int *hist, int32_t *out_col, float *out_val, int *sc) {
+                                                  int *hist, int32_t *out_col, float *out_val, int *sc,
+                                                  int32_t pmn = 1, int32_t pmx = 0) {
     int32_t key[EPT];
     float val[EPT];
     bsr_load<NW, GROUPS, EPT>(g, sk, sv, L, key, val);
     return bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, UNR2>(g, key, val, L, dk, dv, dk2, dv2, hist, out_col, out_val,
-                                                              sc);
+                                                              sc, pmn, pmx);
 }
 
 // the row already in registers (bsr_load; software-pipelined callers load the next row early)
@@ -557,14 +601,17 @@ template <int NW, int GROUPS, int EPT, int LS, bool UNR2>
 __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
                                                        float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
-                                                       int *sc) {
+                                                       int *sc, int32_t pmn, int32_t pmx) {
     constexpr int T = NW * 32;
-    int32_t mn = kKeyPad, mx = 0;
+    int32_t mn = pmn, mx = pmx;
+    if (pmn > pmx) {   // no exact column range from the plan (rowmn / rowmx): reduce it here
+        mn = kKeyPad;
+        mx = 0;
 #pragma unroll
-    for (int e = 0; e < EPT; ++e)
-        if (key[e] != kKeyPad) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
-    mn = g.reduce_min(mn, sc);
-    mx = g.reduce_max(mx, sc);
+        for (int e = 0; e < EPT; ++e)
+            if (key[e] != kKeyPad) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
+        g.reduce_minmax(mn, mx, sc);
+    }
     const uint32_t span = (uint32_t)(mx - mn);
     const int lognb = nextpow2_log(L) + LS;
     const int nb = 1 << lognb;
@@ -587,9 +634,9 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
         cnt += c;
         mxc = max(mxc, c);
     }
-    int tot;
-    int ex = g.excl_sum(cnt, sc, &tot);
-    if (g.reduce_max(mxc, sc) > kBucketMax) return -1;
+    int tot;   // (an over-full bucket adds 2^24 to the total: the overflow test rides on the scan)
+    int ex = g.excl_sum(cnt + (mxc > kBucketMax ? (1 << 24) : 0), sc, &tot);
+    if (tot >= (1 << 24)) return -1;
     for (int b = b0; b < b1; ++b) {
         const int c = hist[hidx(b)];
         hist[hidx(b)] = ex;
@@ -650,7 +697,7 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
         }
     }
     int U;
-    int o = g.excl_sum(nh, sc, &U);
+    int o = g.excl_sum1(nh, sc, &U);
     {   // a segment continuing from the previous slice is summed by that slice's thread
         int32_t prevk = before, cur = -1;
         double acc = 0.0;
@@ -701,10 +748,12 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
                                                                   unsigned *__restrict__ fb_count, int64_t cap_skip,
                                                                   const int64_t *__restrict__ crowptr,
                                                                   int32_t *__restrict__ out_col,
-                                                                  float *__restrict__ out_val) {
+                                                                  float *__restrict__ out_val,
+                                                                  const int32_t *__restrict__ rowmn,
+                                                                  const int32_t *__restrict__ rowmx) {
     using S = BucketSmem<NW, EPT, LS>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ int sc_all[GROUPS][NW + 1];
+    __shared__ int sc_all[GROUPS][2 * NW + 2];
     const Group<NW, GROUPS> g;
     unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
     int32_t *dk = (int32_t *)slice;
@@ -720,7 +769,8 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
         const int64_t o = out_col ? crowptr[i] : s;
         const int U = bucket_sort_reduce<NW, GROUPS, EPT, LS>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
                                                           (out_col ? out_col : chat_col) + o,
-                                                          (out_col ? out_val : chat_val) + o, sc_all[g.gid]);
+                                                          (out_col ? out_val : chat_val) + o, sc_all[g.gid],
+                                                          rowmn ? rowmn[i] : 1, rowmn ? rowmx[i] : 0);
         if (g.gtid == 0) {
             if (U >= 0) ccount[i] = U;
             else if (fb_rows) fb_rows[atomicAdd(fb_count, 1u)] = i;
@@ -744,21 +794,27 @@ struct RowMeta {
 };
 
 __global__ void k_row_meta(const int32_t *__restrict__ order, int64_t n, const int64_t *__restrict__ rowoff,
-                           const int64_t *__restrict__ rowwork, RowMeta *__restrict__ meta) {
+                           const int64_t *__restrict__ rowwork, const int32_t *__restrict__ rowmn,
+                           const int32_t *__restrict__ rowmx, RowMeta *__restrict__ meta,
+                           int2 *__restrict__ rng) {
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
         const int i = order[q];
         const int64_t s = rowoff[i];
         meta[q] = RowMeta{s, (int32_t)(rowoff[i + 1] - s), i, (int32_t)rowwork[i], 0};
+        // exact column range of the row (mn > mx: unknown), apart from the meta table: loaded
+        // per row at the top of the pipelined loop instead of held three rows ahead in registers
+        if (rng) rng[q] = rowmn ? make_int2(rowmn[i], rowmx[i]) : make_int2(1, 0);
     }
 }
 
 template <int NW, int GROUPS, int EPT, int LS = 0, bool WALK = false>
 __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k_merge_bucket_pipe(
     const RowMeta *__restrict__ meta, int64_t nrows, int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
-    int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows, unsigned *__restrict__ fb_count) {
+    int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows, unsigned *__restrict__ fb_count,
+    const int2 *__restrict__ rng) {
     using S = BucketSmem<NW, EPT, LS>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ int sc_all[GROUPS][NW + 1];
+    __shared__ int sc_all[GROUPS][2 * NW + 2];
     const Group<NW, GROUPS> g;
     unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
     int32_t *dk = (int32_t *)slice;
@@ -775,6 +831,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
     float val[EPT];
     bsr_load<NW, GROUPS, EPT>(g, chat_col + m0.s, chat_val + m0.s, min(m0.L, S::kCap), key, val);
     while (r < nrows) {
+        const int2 rg = rng ? rng[r] : make_int2(1, 0);
         int32_t kn[EPT];
         float vn[EPT];
         bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, min(m1.L, S::kCap), kn, vn);
@@ -786,7 +843,8 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
                                                              chat_val + m0.s, sc_all[g.gid]);
             else
                 U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
-                                                                 chat_col + m0.s, chat_val + m0.s, sc_all[g.gid]);
+                                                                 chat_col + m0.s, chat_val + m0.s, sc_all[g.gid],
+                                                                 rg.x, rg.y);
             if (g.gtid == 0) {
                 if (U >= 0) ccount[m0.i] = U;
                 else fb_rows[atomicAdd(fb_count, 1u)] = m0.i;
@@ -1620,7 +1678,7 @@ __device__ __forceinline__ int count_below(const int32_t *__restrict__ col, int6
 
 __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ int sc[kLimNW + 1];
+    __shared__ int sc[2 * kLimNW + 2];
     __shared__ int64_t row_sm;
     const Group<kLimNW, 1> grp;
     const int lane = lane_id(), w = warp_id();

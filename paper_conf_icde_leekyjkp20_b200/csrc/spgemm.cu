@@ -166,6 +166,8 @@ struct spgemm_plan_s {
     int32_t *fb_rows = nullptr;
     unsigned *fb_count = nullptr;
     RowMeta *row_meta = nullptr;   // (offset, length, id) in row_order (pipelined merge bins)
+    int32_t *rowmn = nullptr, *rowmx = nullptr;   // exact column range per row of C (bucket mapping)
+    int64_t *row_rng = nullptr;    // (rowmn, rowmx) as int2 in row_order (pipelined bucket bins)
     bool chat_external = false;
     bool c_in_chat = false;        // C compact at the head of the Ĉ arrays (fused merge)    // Ĉ lives in the caller's C buffers (spgemm_execute, device C)
     // merge units (merge_units.cuh): long rows merged into the side buffer, then one unit kernel
@@ -303,7 +305,8 @@ static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int6
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
     (void)ctas_per_sm;
     LAUNCH(name, s, kern<<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
-        p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count));
+        p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count,
+        p->row_rng ? (const int2 *)p->row_rng + q0 : nullptr));
     return SPGEMM_OK;
 }
 
@@ -317,7 +320,7 @@ static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *ro
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
     LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT, LS><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
         rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0,
-        side ? p->side_off : nullptr, side ? p->side_col : nullptr, side ? p->side_val : nullptr));
+        side ? p->side_off : nullptr, side ? p->side_col : nullptr, side ? p->side_val : nullptr, p->rowmn, p->rowmx));
     return SPGEMM_OK;
 }
 
@@ -499,9 +502,18 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     TRY(palloc(p, &p->rowoff, M + 1, s));
     TRY(palloc(p, &p->deg, M, s));
     TRY(palloc(p, &p->base, p->nnz_a, s));
+    const bool col_range = p->opt.reserved[4] != 1;
+    if (col_range) {
+        TRY(palloc(p, &p->rowmn, M, s));
+        TRY(palloc(p, &p->rowmx, M, s));
+    }
     if (M > 0) {
         CK(cudaMemsetAsync(p->rowwork, 0, M * 8, s));
         CK(cudaMemsetAsync(p->deg, 0, M * 4, s));
+        if (col_range) {   // empty rows keep mn > mx ("unknown")
+            CK(cudaMemsetAsync(p->rowmn, 0x7f, M * 4, s));
+            CK(cudaMemsetAsync(p->rowmx, 0, M * 4, s));
+        }
     }
     if (K > 0)
         LAUNCH("pair_work", s, k_pair_work<<<grid_for(K, 256, p->num_sms * 8), 256, 0, s>>>(p->a_colptr, p->b_rowptr, K,
@@ -514,7 +526,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         if (p->nnz_a > 0)
             LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
                 p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg,
-                (unsigned long long *)rowcap));
+                (unsigned long long *)rowcap, p->b_colidx, p->rowmn, p->rowmx));
         TRY(scan_excl(p, rowcap, M, p->rowoff, s, "row_offsets"));   // padded bucket offsets
     }
     if (M > 0)
@@ -737,8 +749,10 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     const int64_t M = p->m;
     if (M > 0 && p->opt.reserved[0] != 7) {
         if (!p->row_meta) TRY(palloc(p, &p->row_meta, M, s));
+        if (p->rowmn && !p->row_rng) TRY(palloc(p, &p->row_rng, M, s));
         LAUNCH("merge_meta", s, k_row_meta<<<grid_for(M, 256), 256, 0, s>>>(p->row_order, M, p->rowoff, p->rowwork,
-                                                                             p->row_meta));
+                                                                             p->rowmn, p->rowmx, p->row_meta,
+                                                                             (int2 *)p->row_rng));
     }
     if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
     auto rows_of = [&](int b0, int b1, int64_t *cnt) {
