@@ -122,7 +122,9 @@ typedef struct {
                                      only), 2 unit-merge phase clocks, 3 B-Limited path clocks
                                      (SPGEMM_VIEW_UNIT_PROFILE);
                                  [2] 1 = per-row compaction kernels instead of the chunked one;
-                                 [3] 1 = row-product expansion (the paper's comparison order)   */
+                                 [3] 1 = row-product expansion (the paper's comparison order);
+                                 [4] 1 = no per-row column range from the plan (the merge
+                                     reduces each row's min / max column itself)              */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */
@@ -154,7 +156,11 @@ typedef enum {
     SPGEMM_VIEW_CHAT_COL = 7,    /* int32[nnz_chat] after spgemm_expand (before merge)       */
     SPGEMM_VIEW_CHAT_VAL = 8,    /* fp32[nnz_chat]                                            */
     SPGEMM_VIEW_CROWPTR = 9,     /* int64[m+1] C row pointers after spgemm_merge             */
-    SPGEMM_VIEW_UNIT_PROFILE = 10 /* uint64[16] merge-unit phase clocks (options.reserved[1]=2) */
+    SPGEMM_VIEW_UNIT_PROFILE = 10,/* uint64[16] merge-unit phase clocks (options.reserved[1]=2) */
+    SPGEMM_VIEW_ROW_COLMIN = 11, /* int32[m]   first column of row i of C (the merge's bucket
+                                    range; computed in spgemm_plan; empty rows 0x7f7f7f7f;
+                                    size 0 with options.reserved[4] = 1)                       */
+    SPGEMM_VIEW_ROW_COLMAX = 12  /* int32[m]   last column of row i of C (empty rows 0)       */
 } spgemm_view;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;

@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(_HERE, "libspgemm.so")
 
 SPGEMM_DEVICE, SPGEMM_HOST = 0, 1
 VIEW_WORK, VIEW_ROWWORK, VIEW_ROWOFF, VIEW_PAIR_CLASS, VIEW_PIECES, VIEW_GATHER, VIEW_ROW_CLASS, \
-    VIEW_CHAT_COL, VIEW_CHAT_VAL, VIEW_CROWPTR, VIEW_UNIT_PROFILE = range(11)
+    VIEW_CHAT_COL, VIEW_CHAT_VAL, VIEW_CROWPTR, VIEW_UNIT_PROFILE, VIEW_ROW_COLMIN, VIEW_ROW_COLMAX = range(13)
 
 EXPORTED = ["spgemm_abi_version", "spgemm_last_error", "spgemm_default_options", "spgemm_plan",
             "spgemm_expand", "spgemm_merge", "spgemm_output", "spgemm_execute", "spgemm_get_stats",

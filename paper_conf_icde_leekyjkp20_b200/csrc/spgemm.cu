@@ -1150,6 +1150,8 @@ int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_
         case SPGEMM_VIEW_ROWOFF: src = p->rowoff; bytes = (p->m + 1) * 8; break;
         case SPGEMM_VIEW_PAIR_CLASS: src = p->pair_cls; bytes = p->k; break;
         case SPGEMM_VIEW_ROW_CLASS: src = p->row_cls; bytes = p->m; break;
+        case SPGEMM_VIEW_ROW_COLMIN: src = p->rowmn; bytes = p->rowmn ? p->m * 4 : 0; break;
+        case SPGEMM_VIEW_ROW_COLMAX: src = p->rowmx; bytes = p->rowmx ? p->m * 4 : 0; break;
         case SPGEMM_VIEW_CHAT_COL:
             if (p->state != 2) return fail(SPGEMM_ERR_STATE, "Ĉ is only inspectable between expand and merge");
             src = p->chat_col; bytes = p->chat_cap * 4; break;

@@ -111,6 +111,22 @@ def test_stage1_workload(seed):
     p.destroy()
 
 
+@pytest.mark.parametrize("name", ["C1", "tiny"])
+def test_stage1_row_column_range(name):
+    """The plan's per-row column range (the merge's bucket mapping, R12) is exactly the
+    first / last column of each row of the oracle's C; empty rows keep min > max."""
+    inp = _inp("C1") if name == "C1" else synth.random_tiny(300, 700, 500, 0.03, 0.05, 9, skew=True)
+    p, keep = _plan(inp)
+    mn = p.inspect(spg.VIEW_ROW_COLMIN, np.int32)
+    mx = p.inspect(spg.VIEW_ROW_COLMAX, np.int32)
+    rowptr, col, _ = oracle.gustavson(inp)
+    ne = np.diff(rowptr) > 0
+    np.testing.assert_array_equal(mn[ne], col[rowptr[:-1][ne]])
+    np.testing.assert_array_equal(mx[ne], col[rowptr[1:][ne] - 1])
+    assert np.all(mn[~ne] > mx[~ne])
+    p.destroy()
+
+
 # ------------------------------------------------------------------ stage (2) -------------
 @pytest.mark.parametrize("name,opts", CASES)
 def test_stage2_reorganizer(name, opts):
