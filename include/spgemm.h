@@ -111,7 +111,11 @@ typedef struct {
                                  the non-limited kernels' capacity take the long-row kernels     */
     int32_t enable_gather;
     int32_t enable_limit;
-    int32_t validate;         /* check input structure in spgemm_plan (default 1)               */
+    int32_t validate;         /* check input structure in spgemm_plan (default 1).  With 0 the
+                                 caller guarantees the contracts above: the merge relies on B's
+                                 ascending rows (each run is sorted; the per-row column range is
+                                 read from the first / last entry of b_k*) -- unsorted rows are
+                                 then undefined behaviour, not an error                          */
     int32_t reserved[16];     /* tuning / comparison knobs, 0 = default:
                                  [0] merge variant: 1 register-staged counting sort, 2 bucket sort
                                      everywhere, 3 merge path everywhere, 4 fused unit merge (C
