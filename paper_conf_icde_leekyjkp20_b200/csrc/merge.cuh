@@ -1957,7 +1957,11 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     int tot;
                     int ex = grp.excl_sum(cnt, sc, &tot);
                     mxb = grp.reduce_max(mxb, sc);
-                    constexpr int T = kLimCap * 3 / 4;   // groups < T + max bin <= kLimCap (7/8: same speed)
+                    // groups < T + max bin <= kLimCap: 3/4 of the sorter when no bin exceeds 1/4 of it
+                    // (fewer, fuller sorts: C3 182 -> 159 ms; 7/8: same speed), else 1/2, so rows
+                    // with one heavy column range still take this path (C5: 3/4 alone sent them to
+                    // the window path, limited merge 86 -> 115 ms)
+                    const int T = mxb <= kLimCap / 4 ? kLimCap * 3 / 4 : kLimCap / 2;
 #pragma unroll
                     for (int u = 0; u < BPT; ++u) {
                         fh[threadIdx.x * BPT + u] = ex / T;     // group id of the bin
