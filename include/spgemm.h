@@ -162,9 +162,10 @@ typedef enum {
     SPGEMM_VIEW_CROWPTR = 9,     /* int64[m+1] C row pointers after spgemm_merge             */
     SPGEMM_VIEW_UNIT_PROFILE = 10,/* uint64[16] merge-unit phase clocks (options.reserved[1]=2) */
     SPGEMM_VIEW_ROW_COLMIN = 11, /* int32[m]   first column of row i of C (the merge's bucket
-                                    range; computed in spgemm_plan; empty rows 0x7f7f7f7f;
+                                    range; computed in spgemm_plan for rows whose padded Ĉ
+                                    bucket exceeds 256 slots; other rows 0x7f7f7f7f = unknown;
                                     size 0 with options.reserved[4] = 1)                       */
-    SPGEMM_VIEW_ROW_COLMAX = 12  /* int32[m]   last column of row i of C (empty rows 0)       */
+    SPGEMM_VIEW_ROW_COLMAX = 12  /* int32[m]   last column of row i of C (unknown rows 0)     */
 } spgemm_view;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;

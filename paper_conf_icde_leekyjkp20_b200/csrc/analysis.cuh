@@ -123,35 +123,23 @@ __global__ void __launch_bounds__(256) k_row_work(const int64_t *__restrict__ a_
                                                   const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
                                                   const int64_t *__restrict__ b_rowptr,
                                                   unsigned long long *__restrict__ rowwork, int32_t *__restrict__ deg,
-                                                  unsigned long long *__restrict__ rowcap,
-                                                  const int32_t *__restrict__ b_colidx = nullptr,
-                                                  int32_t *__restrict__ rowmn = nullptr,
-                                                  int32_t *__restrict__ rowmx = nullptr) {
-    // rowmn / rowmx (optional): the exact column range of row i of C -- min / max over the stored
-    // a_ik of b_k*'s first / last column (B's rows are ascending): every product of the row is in
-    // it and its ends are attained, so the merge's bucket mapping needs no range reduction.
+                                                  unsigned long long *__restrict__ rowcap) {
     int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
     if (e0 >= nnz_a) return;
     int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
     int64_t kend = __ldg(a_colptr + k + 1);
-    int64_t rb0 = __ldg(b_rowptr + k), rb1 = __ldg(b_rowptr + k + 1);
+    int64_t rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
     for (int64_t e = e0; e < e0 + 8 && e < nnz_a; ++e) {
         while (e >= kend) {
             ++k;
             kend = __ldg(a_colptr + k + 1);
-            rb0 = rb1;
-            rb1 = __ldg(b_rowptr + k + 1);
+            rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
         }
-        const int64_t rb = rb1 - rb0;
         if (rb > 0) {
             int32_t i = a_rowidx[e];
             atomicAdd(rowwork + i, (unsigned long long)rb);
             atomicAdd(deg + i, 1);
             if (rowcap) atomicAdd(rowcap + i, (unsigned long long)pad_run(rb));
-            if (rowmn) {
-                atomicMin(rowmn + i, __ldg(b_colidx + rb0));
-                atomicMax(rowmx + i, __ldg(b_colidx + rb1 - 1));
-            }
         }
     }
 }
@@ -186,22 +174,44 @@ __global__ void __launch_bounds__(256) k_row_reduce(const int64_t *__restrict__ 
 // Run bases: the run of products of A entry e = (i, k) occupies Ĉ positions
 // [base[e], base[e] + nnz(b_k*)) inside row i's bucket (cursor starts at rowoff[i]), followed
 // by pad_run(nnz(b_k*)) - nnz(b_k*) sentinel slots.
+// rows whose padded Ĉ bucket is longer than this get the plan's column range (bucket-sort bins)
+constexpr int64_t kRangeMinSlots = 256;
+
 __global__ void __launch_bounds__(256) k_run_base(const int64_t *__restrict__ a_colptr,
                                                   const int32_t *__restrict__ a_rowidx, int64_t K, int64_t nnz_a,
                                                   const int64_t *__restrict__ b_rowptr,
-                                                  unsigned long long *__restrict__ cursor, int64_t *__restrict__ base) {
+                                                  unsigned long long *__restrict__ cursor, int64_t *__restrict__ base,
+                                                  const int64_t *__restrict__ rowoff = nullptr,
+                                                  const int32_t *__restrict__ b_colidx = nullptr,
+                                                  int32_t *__restrict__ rowmn = nullptr,
+                                                  int32_t *__restrict__ rowmx = nullptr) {
+    // rowmn / rowmx (optional): the exact column range of row i of C -- min / max over the stored
+    // a_ik of b_k*'s first / last column (B's rows are ascending): every product of the row is in
+    // it and its ends are attained, so the bucket-sort bins need no range reduction.  Only rows
+    // whose padded bucket exceeds kRangeMinSlots (the bucket-sorted ones) pay the two atomics.
     int64_t e0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
     if (e0 >= nnz_a) return;
     int64_t k = upper_bound_idx(a_colptr, 0, K, e0);
     int64_t kend = __ldg(a_colptr + k + 1);
-    int64_t rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
+    int64_t rb0 = __ldg(b_rowptr + k), rb1 = __ldg(b_rowptr + k + 1);
     for (int64_t e = e0; e < e0 + 8 && e < nnz_a; ++e) {
         while (e >= kend) {
             ++k;
             kend = __ldg(a_colptr + k + 1);
-            rb = __ldg(b_rowptr + k + 1) - __ldg(b_rowptr + k);
+            rb0 = rb1;
+            rb1 = __ldg(b_rowptr + k + 1);
         }
-        base[e] = rb > 0 ? (int64_t)atomicAdd(cursor + a_rowidx[e], (unsigned long long)pad_run(rb)) : -1;
+        const int64_t rb = rb1 - rb0;
+        if (rb > 0) {
+            const int32_t i = a_rowidx[e];
+            base[e] = (int64_t)atomicAdd(cursor + i, (unsigned long long)pad_run(rb));
+            if (rowmn && __ldg(rowoff + i + 1) - __ldg(rowoff + i) > kRangeMinSlots) {
+                atomicMin(rowmn + i, __ldg(b_colidx + rb0));
+                atomicMax(rowmx + i, __ldg(b_colidx + rb1 - 1));
+            }
+        } else {
+            base[e] = -1;
+        }
     }
 }
 

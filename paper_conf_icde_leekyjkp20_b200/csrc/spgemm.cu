@@ -526,7 +526,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         if (p->nnz_a > 0)
             LAUNCH("row_work", s, k_row_work<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
                 p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, (unsigned long long *)p->rowwork, p->deg,
-                (unsigned long long *)rowcap, p->b_colidx, p->rowmn, p->rowmx));
+                (unsigned long long *)rowcap));
         TRY(scan_excl(p, rowcap, M, p->rowoff, s, "row_offsets"));   // padded bucket offsets
     }
     if (M > 0)
@@ -537,7 +537,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         TRY(talloc(p, tc, &cursor, M));
         CK(cudaMemcpyAsync(cursor, p->rowoff, M * 8, cudaMemcpyDeviceToDevice, s));
         LAUNCH("run_base", s, k_run_base<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
-            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, cursor, p->base));
+            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, cursor, p->base, p->rowoff, p->b_colidx, p->rowmn,
+            p->rowmx));
     }
     CK(cudaMemcpyAsync(&p->h_scal, p->scal, sizeof(PlanScalars), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(&p->chat_cap, p->rowoff + M, 8, cudaMemcpyDeviceToHost, s));
