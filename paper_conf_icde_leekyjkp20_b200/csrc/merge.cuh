@@ -776,7 +776,9 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
             else if (fb_rows) fb_rows[atomicAdd(fb_count, 1u)] = i;
             else ccount[i] = -1;   // limited list: k_merge_limited takes the row (merge-path fallback)
         }
-        g.sync();
+        // (no barrier: the next row first writes hist, whose last reads -- the ranking -- and
+        // those of sc are behind the reduction phase's barriers; dk / dv, read by the copy-out,
+        // are next written after two more barriers)
     }
     (void)cap_skip;
 }
@@ -850,7 +852,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
                 else fb_rows[atomicAdd(fb_count, 1u)] = m0.i;
             }
         }
-        g.sync();
+        if constexpr (WALK) g.sync();   // (bucket sort: no barrier needed between rows, see k_merge_bucket)
 #pragma unroll
         for (int e = 0; e < EPT; ++e) { key[e] = kn[e]; val[e] = vn[e]; }
         m0 = m1;
