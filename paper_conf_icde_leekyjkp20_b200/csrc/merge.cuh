@@ -480,7 +480,7 @@ __device__ __forceinline__ void bsr_load(const Group<NW, GROUPS> &g, const int32
     }
 }
 
-template <int NW, int GROUPS, int EPT, int LS = 0, bool UNR2 = false>
+template <int NW, int GROUPS, int EPT, int LS = 0, bool UNR2 = false, int PRECLEAR = 0>
 __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
                                                        float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
@@ -597,7 +597,7 @@ __device__ __forceinline__ int bucket_sort_reduce(const Group<NW, GROUPS> &g, co
 }
 
 // the row already in registers (bsr_load; software-pipelined callers load the next row early)
-template <int NW, int GROUPS, int EPT, int LS, bool UNR2>
+template <int NW, int GROUPS, int EPT, int LS, bool UNR2, int PRECLEAR>
 __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
                                                        float (&val)[EPT], int L, int32_t *dk, float *dv, int32_t *dk2,
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
@@ -617,8 +617,12 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
     const int nb = 1 << lognb;
     const int bits = span ? 32 - __clz(span) : 0;
     const int sh = max(0, bits - lognb);
-    for (int b = g.gtid; b <= hidx(nb); b += T) hist[b] = 0;
-    g.sync();
+    // PRECLEAR > 0: the caller zeroed hist[0, PRECLEAR] (and the previous row cleared it after its
+    // ranking), so the row starts with its atomics -- one barrier less per row
+    if constexpr (PRECLEAR == 0) {
+        for (int b = g.gtid; b <= hidx(nb); b += T) hist[b] = 0;
+        g.sync();
+    }
     // one shared atomic per element (spread-address ATOMS cost ~2 cycles per lane): its return
     // value is the element's rank inside its bucket, reused by the scatter below
     int rk[EPT];
@@ -636,7 +640,13 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
     }
     int tot;   // (an over-full bucket adds 2^24 to the total: the overflow test rides on the scan)
     int ex = g.excl_sum(cnt + (mxc > kBucketMax ? (1 << 24) : 0), sc, &tot);
-    if (tot >= (1 << 24)) return -1;
+    if (tot >= (1 << 24)) {
+        if constexpr (PRECLEAR > 0) {   // (the cnt reads above are behind the scan's barriers)
+            for (int b = g.gtid; b <= PRECLEAR; b += T) hist[b] = 0;
+            g.sync();
+        }
+        return -1;
+    }
     for (int b = b0; b < b1; ++b) {
         const int c = hist[hidx(b)];
         hist[hidx(b)] = ex;
@@ -682,6 +692,8 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
         }
     }
     g.sync();
+    if constexpr (PRECLEAR > 0)   // hist's last reads (the ranking) are done: clear it for the next row
+        for (int b = g.gtid; b <= PRECLEAR; b += T) hist[b] = 0;
     // 3. segmented reduction over contiguous slices (fp64), compacted into (dk, dv)
     L = tot;   // valid (non-sentinel) entries
     const int E = ((L + T - 1) / T) | 1;     // odd stride between thread slices: no bank conflicts
@@ -832,6 +844,10 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
     int32_t key[EPT];
     float val[EPT];
     bsr_load<NW, GROUPS, EPT>(g, chat_col + m0.s, chat_val + m0.s, min(m0.L, S::kCap), key, val);
+    if constexpr (!WALK) {   // PRECLEAR: hist starts zeroed, every row leaves it zeroed
+        for (int b = g.gtid; b <= hidx(S::kNb); b += NW * 32) hist[b] = 0;
+        g.sync();
+    }
     while (r < nrows) {
         const int2 rg = rng ? rng[r] : make_int2(1, 0);
         int32_t kn[EPT];
@@ -844,7 +860,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
                 U = bucket_walk_reduce_regs<NW, GROUPS, EPT>(g, key, val, m0.L, dk, dv, hist, chat_col + m0.s,
                                                              chat_val + m0.s, sc_all[g.gid]);
             else
-                U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
+                U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, false, hidx(S::kNb)>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
                                                                  chat_col + m0.s, chat_val + m0.s, sc_all[g.gid],
                                                                  rg.x, rg.y);
             if (g.gtid == 0) {
