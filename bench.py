@@ -7,9 +7,14 @@ compaction) + spgemm_destroy, through the C-ABI.  Inputs are resident in HBM whe
 region starts.  Metric (BASELINE.json): GFLOPS = 2 x intermediate products / s; the HBM
 roofline fraction of the dominant kernel and of the whole step are reported beside it.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
-Multi-GPU: launched with torch.distributed.run, one rank per GPU, rows of C partitioned into
-balanced row blocks (strong scaling of one product); value = all products / max-over-ranks time.
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
+Default workload: C5 (BASELINE.json configs[4], the metric's 1/2/4/8-GPU config; it fits one B200).
+Multi-GPU: one rank per GPU over NCCL (torch.distributed.run; `--gpus N` without WORLD_SIZE in the
+environment re-launches itself that way).  Rank 0 generates the input, computes the balanced
+row-block partition of C on its GPU, broadcasts B and sends every rank its row slice of A (NCCL,
+dist.py); each rank runs the whole path on its block (strong scaling of one product).  value = all
+products / max-over-ranks device time; the C row-block gather to rank 0 is timed on its own
+(`c_gather`), outside the step.
 """
 from __future__ import annotations
 
@@ -36,7 +41,7 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C2")
+    ap.add_argument("--config", default="C5")
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
@@ -165,49 +170,99 @@ def dist_env():
     return ws, rank, local
 
 
+def relaunch(args) -> int:
+    """`bench.py --gpus N` outside torch.distributed: run N ranks (one per GPU) under
+    torch.distributed.run on 127.0.0.1 with the same arguments; rank 0 prints the line."""
+    import socket
+    sck = socket.socket()
+    sck.bind(("127.0.0.1", 0))
+    port = sck.getsockname()[1]
+    sck.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 def flush_l2(buf):
     buf.add_(1)  # write 512 MiB (> 126 MB L2) between timed steps
 
 
 def main():
     args = parse()
-    ws, rank, local = dist_env()
-    import torch
     if args.impl == "reference":
+        ws, rank, _ = dist_env()
         return run_reference(args, ws, rank)
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        sys.exit(relaunch(args))
+    ws, rank, local = dist_env()
+    if "WORLD_SIZE" in os.environ and ws != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws} (launch one rank per GPU)")
+    import torch
     import synth
     import paper_conf_icde_leekyjkp20_b200 as spg
+    from paper_conf_icde_leekyjkp20_b200 import dist as pdist
     from paper_conf_icde_leekyjkp20_b200.build import build_library
     if rank == 0:
         build_library()
-    if os.environ.get("SPGEMM_BENCH_SHARE_GPU"):   # test mode: N ranks share the visible GPUs (gloo)
+    share = bool(os.environ.get("SPGEMM_BENCH_SHARE_GPU"))   # test mode: N ranks share the visible GPUs (gloo)
+    if share:
         local = local % torch.cuda.device_count()
-    if ws > 1:
-        import torch.distributed as dist
-        torch.cuda.set_device(local)
-        if os.environ.get("SPGEMM_BENCH_SHARE_GPU"):
-            dist.init_process_group("gloo")
-        else:
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        dist.barrier()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    inp_full = synth.make_inputs(args.config, seed=args.seed)
-    A_full, B_full = spg.from_inputs(inp_full, dev)
-    nparts, part = (ws, rank)
-    if args.slice:
-        nparts, part = (int(x) for x in args.slice.split(":"))
-    if nparts > 1:
-        from paper_conf_icde_leekyjkp20_b200 import dist as pdist
-        bounds = spg.row_partition(A_full, B_full, nparts)
-        rank_ = part
-        A = pdist.csc_row_slice(A_full, int(bounds[rank_]), int(bounds[rank_ + 1]))
-        B = B_full
-        inp = synth.SparseInputs(f"{args.config}[{bounds[rank_]}:{bounds[rank_ + 1]}]", A.nrows, A.ncols, B.ncols,
+    dist = None
+    if ws > 1:
+        import torch.distributed as dist
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
+        if rank == 0:
+            build_library()
+        dist.barrier()
+    comm_dev = torch.device("cpu") if share else dev
+    inp_full = None
+    if rank == 0 or ws == 1:
+        inp_full = synth.make_inputs(args.config, seed=args.seed)
+    if ws > 1:
+        # rank 0: input, partition; NCCL: B broadcast, A row-slice scatter (input movement, untimed)
+        t_dist = time.perf_counter()
+        if rank == 0:
+            A_full, B_full = spg.from_inputs(inp_full, dev)
+            bounds = torch.from_numpy(spg.row_partition(A_full, B_full, ws)).to(comm_dev)
+            A_src = spg.CSC(A_full.nrows, A_full.ncols, A_full.colptr.to(comm_dev), A_full.rowidx.to(comm_dev),
+                            A_full.val.to(comm_dev))
+            B_src = spg.CSR(B_full.nrows, B_full.ncols, B_full.rowptr.to(comm_dev), B_full.colidx.to(comm_dev),
+                            B_full.val.to(comm_dev))
+        else:
+            bounds = torch.zeros(ws + 1, dtype=torch.int64, device=comm_dev)
+            A_src = B_src = None
+        dist.broadcast(bounds, src=0)
+        B = pdist.broadcast_csr(B_src, src=0, device=comm_dev)
+        A = pdist.scatter_row_slices(A_src, bounds.tolist(), src=0, device=comm_dev)
+        A = spg.CSC(A.nrows, A.ncols, A.colptr.to(dev), A.rowidx.to(dev), A.val.to(dev))
+        B = spg.CSR(B.nrows, B.ncols, B.rowptr.to(dev), B.colidx.to(dev), B.val.to(dev))
+        if rank == 0:
+            del A_full, B_full, A_src, B_src
+        torch.cuda.synchronize()
+        dist.barrier()
+        dist_s = time.perf_counter() - t_dist
+        bounds = bounds.tolist()
+        inp = synth.SparseInputs(f"{args.config}[{bounds[rank]}:{bounds[rank + 1]}]", A.nrows, A.ncols, B.ncols,
                                  A.colptr.cpu().numpy(), A.rowidx.cpu().numpy(), A.val.cpu().numpy(),
-                                 inp_full.b_rowptr, inp_full.b_colidx, inp_full.b_val)
+                                 B.rowptr.cpu().numpy(), B.colidx.cpu().numpy(), B.val.cpu().numpy())
     else:
-        inp, A, B = inp_full, A_full, B_full
+        dist_s, bounds = 0.0, None
+        A_full, B_full = spg.from_inputs(inp_full, dev)
+        if args.slice:   # scaling study: rank r's row block of an N-way partition, alone on this GPU
+            nparts, part = (int(x) for x in args.slice.split(":"))
+            bounds = spg.row_partition(A_full, B_full, nparts)
+            A = pdist.csc_row_slice(A_full, int(bounds[part]), int(bounds[part + 1]))
+            B = B_full
+            inp = synth.SparseInputs(f"{args.config}[{bounds[part]}:{bounds[part + 1]}]", A.nrows, A.ncols, B.ncols,
+                                     A.colptr.cpu().numpy(), A.rowidx.cpu().numpy(), A.val.cpu().numpy(),
+                                     inp_full.b_rowptr, inp_full.b_colidx, inp_full.b_val)
+        else:
+            inp, A, B = inp_full, A_full, B_full
     stream = torch.cuda.current_stream(dev)
     opts = dict(validate=0)
     for kv in args.opt:
@@ -284,8 +339,10 @@ def main():
     total_ms = float(sum(step_ms))
     products = st["nnz_chat"]
     # max over ranks of the device time; total products over ranks
+    rank_ms = [round(total_ms / args.steps, 4)]
     if ws > 1:
-        t = torch.tensor([total_ms, float(products), float(nnz_c), float(launches)], dtype=torch.float64, device=dev)
+        t = torch.tensor([total_ms, float(products), float(nnz_c), float(launches), float(inp.nnz_a)],
+                         dtype=torch.float64, device=comm_dev)
         tmax = t.clone()
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
         tsum = t.clone()
@@ -294,8 +351,14 @@ def main():
         products_all = int(tsum[1])
         nnz_c_all = int(tsum[2])
         launches_all = int(tsum[3])
+        nnz_a_all = int(tsum[4])
+        every = [torch.zeros(1, dtype=torch.float64, device=comm_dev) for _ in range(ws)]
+        dist.all_gather(every, t[:1].clone())
+        rank_ms = [round(float(x) / args.steps, 4) for x in every]
+        m_all = int(bounds[-1])
     else:
         total_ms_all, products_all, nnz_c_all, launches_all = total_ms, products, nnz_c, launches
+        nnz_a_all, m_all = inp.nnz_a, inp.m
     ms_per_step = total_ms_all / args.steps
     value = 2.0 * products_all / (ms_per_step / 1e3) / 1e9
 
@@ -314,7 +377,7 @@ def main():
     groups = {
         "expand": ("expand_", 8 * products + 12 * nnz_a + 8 * nnz_b),
         "merge": ("merge_", 8 * products + 8 * nnz_c + 16 * inp.m),
-        "compact": ("compact", 16 * nnz_c + 8 * inp.m),
+        "compact": ("compact", 16 * nnz_c + 8 * inp.m),   # (legacy bin merge only)
     }
     gms = {g: sum(v for n, v in k_ms.items() if n.startswith(pre)) for g, (pre, _) in groups.items()}
     top = max(gms, key=lambda g: gms[g])
@@ -323,8 +386,8 @@ def main():
     # DRAM bytes of the same kernel group per step, from the committed ncu --set full capture
     # (scripts/ncu_traffic.py); null when no capture of this config exists
     traffic, traffic_src = None, None
-    tpath = os.path.join(ROOT, "profiles", f"r1_traffic_{args.config}.json")
-    if os.path.exists(tpath) and ws == 1:
+    tpath = os.path.join(ROOT, "profiles", f"r2_traffic_{args.config}.json")
+    if os.path.exists(tpath) and ws == 1 and not args.slice and not args.opt:
         try:
             tj = json.load(open(tpath))
             traffic = tj["groups"][top]["dram_bytes"]
@@ -342,8 +405,8 @@ def main():
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32 (fp64 merge accumulation)",
         "data": "synthetic (seeded generator, synth/)",
-        "config": {"workload": f"{args.config}: " + synth.CONFIGS[args.config]["desc"], "m": inp_full.m,
-                   "nnz_a": inp_full.nnz_a, "products": products_all, "nnz_c": nnz_c_all,
+        "config": {"workload": f"{args.config}: " + synth.CONFIGS[args.config]["desc"], "m": m_all,
+                   "nnz_a": nnz_a_all, "products": products_all, "nnz_c": nnz_c_all,
                    "parallelism": f"row-partition x{ws}" if ws > 1 else "single GPU",
                    "l2": "flushed between steps (512 MiB write); Ĉ >> L2", "seed": args.seed,
                    "step": "plan+execute+destroy via C-ABI, device-resident inputs",
@@ -354,10 +417,31 @@ def main():
                           "def": "A + B + 2*Ĉ(8 B/product) + C, per step"},
         "kernel_ms": breakdown,
         "gpu_launches": launches_all,
-        "merge_units": {"units": st.get("n_units"), "fallback": st.get("n_units_fallback")},
+        "rank_ms_per_step": rank_ms,
         "clocks": clocks,
         "wall_s": round(wall, 3),
     }
+    if ws > 1:
+        # C row-block gather to rank 0 (NCCL point-to-point into one CSR, no concatenation copy):
+        # output movement, timed on its own
+        p = spg.Plan(A, B, stream=stream, **opts)
+        C = p.execute()
+        p.destroy()
+        Cc = C if not share else spg.CSR(C.nrows, C.ncols, C.rowptr.cpu(), C.colidx.cpu(), C.val.cpu())
+        torch.cuda.synchronize()
+        dist.barrier()
+        g0 = time.perf_counter()
+        G = pdist.gather_row_blocks(Cc, dst=0)
+        torch.cuda.synchronize()
+        g_s = time.perf_counter() - g0
+        gb = torch.tensor([g_s], dtype=torch.float64, device=comm_dev)
+        dist.all_reduce(gb, op=dist.ReduceOp.MAX)
+        out["c_gather"] = {"ms": round(float(gb[0]) * 1e3, 3), "bytes": int(nnz_c_all * 8 + (m_all + 1) * 8),
+                           "to": "rank 0", "how": "NCCL send/recv into one CSR; synchronised wall time, max over ranks",
+                           "input_distribution_s": round(dist_s, 3)}
+        if rank == 0:
+            assert G.nnz == nnz_c_all and G.nrows == m_all
+        del C, Cc, G
     # e2e through the C-ABI with host buffers (H2D of A, B and D2H of C inside the timed region)
     if not args.no_e2e:
         Ah, Bh = spg.from_inputs(inp, "cpu")
@@ -378,7 +462,7 @@ def main():
                 es.append(dt)
         e2e_t = sum(es) / len(es)
         if ws > 1:
-            tt = torch.tensor([e2e_t], dtype=torch.float64, device=dev)
+            tt = torch.tensor([e2e_t], dtype=torch.float64, device=comm_dev)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             e2e_t = float(tt[0])
         out["e2e"] = {"value": round(2.0 * products_all / e2e_t / 1e9, 3), "unit": UNIT,

@@ -18,8 +18,11 @@
  *   spgemm_expand   (3) expansion: every product (i, j, a_ik*b_kj) written into the
  *                       row-bucketed intermediate matrix Ĉ (L321-L323 L).
  *   spgemm_merge    (4) merge: per Ĉ row, sort by column + segmented reduce (fp64
- *                       accumulation, one rounding to fp32); long rows B-Limited.
- *   spgemm_output       CSR compaction of the merged rows into caller buffers.
+ *                       accumulation, one rounding to fp32); long rows B-Limited.  Default
+ *                       (merge tiles): C is placed by a decoupled look-back at the head of
+ *                       the Ĉ arrays, in place -- no separate compaction pass.
+ *   spgemm_output       copy of C (head of the Ĉ arrays) into caller buffers; nothing to copy
+ *                       when the caller's arrays are the Ĉ arrays (spgemm_execute, device C).
  *   spgemm_execute  = expand + merge + allocate C (callback) + output.
  *
  * Conventions for every call:
@@ -128,7 +131,10 @@ typedef struct {
                                  [2] 1 = per-row compaction kernels instead of the chunked one;
                                  [3] 1 = row-product expansion (the paper's comparison order);
                                  [4] 1 = no per-row column range from the plan (the merge
-                                     reduces each row's min / max column itself)              */
+                                     reduces each row's min / max column itself);
+                                 [5] 1 = legacy per-bin merge + CSR compaction (merge.cuh; also
+                                     selected by any bin variant in [0]); 0 with [0] = 0: the
+                                     merge-tile kernel (merge_tiles.cuh), C placed in place     */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */
@@ -197,9 +203,10 @@ int spgemm_output(spgemm_plan_t plan, spgemm_csr_out_t *C, void *stream);
 
 /* expand + merge + alloc(C arrays in `out_where`) + output.  C->rowptr/colidx/val are
  * set to the allocated buffers (owned by the caller).  Returns after `stream` holds C.
- * With the fused unit merge (options.reserved[0] = 4) and a device C, colidx / val are requested
- * before the expansion with capacity nnz(Ĉ) (padded) >= nnz(C): they hold Ĉ during the merge and C
- * in their first nnz(C) entries afterwards (C->nnz). */
+ * With a device C and the default merge (or the fused unit merge, options.reserved[0] = 4),
+ * colidx / val are requested BEFORE the expansion with capacity nnz(Ĉ) (padded slots) >= nnz(C):
+ * they hold Ĉ during the merge and C in their first C->nnz entries afterwards (one buffer for
+ * both: no second nnz(Ĉ)-sized allocation, no copy). */
 int spgemm_execute(spgemm_plan_t plan, spgemm_alloc_fn alloc, void *alloc_ctx, int32_t out_where,
                    spgemm_csr_out_t *C, void *stream);
 
@@ -210,7 +217,8 @@ int spgemm_get_stats(spgemm_plan_t plan, spgemm_stats_t *stats);
 int spgemm_inspect(spgemm_plan_t plan, int32_t what, void *host_dst, int64_t capacity_bytes,
                    int64_t *size_bytes);
 
-/* Frees every workspace of the plan (stream-ordered on the plan's last stream). */
+/* Frees every workspace of the plan (stream-ordered on the plan's last stream).  Workspaces
+ * include the temporaries of every call (e.g. host-output staging): they live until here. */
 int spgemm_destroy(spgemm_plan_t plan);
 
 /* Multi-GPU / chunked execution: balanced row-block partition of C = A x B (R8).

@@ -227,16 +227,3 @@ def balanced_row_partition(rowwork, parts: int):
     b.append(rowwork.size)
     return np.array(b, dtype=np.int64)
 
-
-def chunk_rows(rowwork, budget: int):
-    """Greedy consecutive row chunks whose Ĉ fits ``budget`` products (a row larger than
-    the budget forms a chunk of its own)."""
-    bounds = [0]
-    acc = 0
-    for i, w in enumerate(rowwork.tolist()):
-        if acc > 0 and acc + w > budget:
-            bounds.append(i)
-            acc = 0
-        acc += w
-    bounds.append(rowwork.size)
-    return np.array(bounds, dtype=np.int64)

@@ -264,7 +264,7 @@ class HostBufferPool:
     def get(self, slot: int, nbytes: int) -> torch.Tensor:
         b = self.bufs.get(slot)
         if b is None or b.numel() < nbytes:
-            b = torch.empty(int(nbytes * 1.25) + 64, dtype=torch.uint8, pin_memory=True)
+            b = torch.empty(int(nbytes) + 4096, dtype=torch.uint8, pin_memory=True)
             self.bufs[slot] = b
         return b[:nbytes]
 

@@ -56,6 +56,7 @@ struct PlanScalars {
     unsigned long long lim_max_deg;  // max runs of a limited row
     unsigned long long lim_max_L;    // max products of a limited row
     unsigned long long long_slots;   // padded Ĉ slots of the long rows (side buffer of the merge)
+    unsigned long long lim_slots;    // padded Ĉ slots of the limited rows (column-group scratch)
     int invalid;                     // validation failure bits
     int pad;
 };
@@ -361,8 +362,8 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
                                                       const int32_t *__restrict__ deg, int64_t M, int64_t t_lim,
                                                       int64_t cap_max, int8_t *__restrict__ rcls,
                                                       uint8_t *__restrict__ bucket, PlanScalars *sc) {
-    __shared__ unsigned long long sm[4][8];
-    unsigned long long runs = 0, mdeg = 0, mlen = 0, lslots = 0;
+    __shared__ unsigned long long sm[5][8];
+    unsigned long long runs = 0, mdeg = 0, mlen = 0, lslots = 0, limslots = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (int64_t)gridDim.x * blockDim.x) {
         // L = products of the row (paper class); cap = its padded bucket length (kernel capacity)
         const int64_t L = rowwork[i];
@@ -377,6 +378,7 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
             runs += (unsigned long long)deg[i];
             mdeg = max(mdeg, (unsigned long long)deg[i]);
             mlen = max(mlen, (unsigned long long)cap);
+            limslots += (unsigned long long)cap;
         }
         else if (cap <= kWarpRowMax) { c = RC_WARP; b = kRowBucketWarp; }
         else if (cap <= 64) { c = RC_WARP_SORT; b = kRowBucketWarp64; }
@@ -394,14 +396,19 @@ __global__ void __launch_bounds__(256) k_row_classify(const int64_t *__restrict_
     mdeg = warp_max(mdeg);
     mlen = warp_max(mlen);
     lslots = warp_sum(lslots);
+    limslots = warp_sum(limslots);
     if (lane_id() == 0) {
         sm[0][warp_id()] = runs; sm[1][warp_id()] = mdeg; sm[2][warp_id()] = mlen; sm[3][warp_id()] = lslots;
+        sm[4][warp_id()] = limslots;
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned long long a = 0, b = 0, c = 0, d = 0;
-        for (int w = 0; w < 8; ++w) { a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); d += sm[3][w]; }
+        unsigned long long a = 0, b = 0, c = 0, d = 0, e = 0;
+        for (int w = 0; w < 8; ++w) {
+            a += sm[0][w]; b = max(b, sm[1][w]); c = max(c, sm[2][w]); d += sm[3][w]; e += sm[4][w];
+        }
         if (d) atomicAdd(&sc->long_slots, d);
+        if (e) atomicAdd(&sc->lim_slots, e);
         if (a) atomicAdd(&sc->lim_runs, a);
         if (b) atomicMax(&sc->lim_max_deg, b);
         if (c) atomicMax(&sc->lim_max_L, c);

@@ -638,9 +638,13 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
         cnt += c;
         mxc = max(mxc, c);
     }
-    int tot;   // (an over-full bucket adds 2^24 to the total: the overflow test rides on the scan)
-    int ex = g.excl_sum(cnt + (mxc > kBucketMax ? (1 << 24) : 0), sc, &tot);
-    if (tot >= (1 << 24)) {
+    // (an over-full bucket adds 2^16 to the total: the overflow test rides on the scan.  A row holds
+    // at most 9216 < 2^16 slots and a group at most 1024 threads, so the flagged total stays below
+    // 2^26 + 2^16 and cannot wrap, and any flag lifts it above every real count)
+    static_assert(NW * 32 <= 1024, "overflow flag sized for <= 1024 threads");
+    int tot;
+    int ex = g.excl_sum(cnt + (mxc > kBucketMax ? (1 << 16) : 0), sc, &tot);
+    if (tot >= (1 << 16)) {
         if constexpr (PRECLEAR > 0) {   // (the cnt reads above are behind the scan's barriers)
             for (int b = g.gtid; b <= PRECLEAR; b += T) hist[b] = 0;
             g.sync();

@@ -17,6 +17,8 @@
 #include "expand.cuh"
 #include "merge.cuh"
 #include "merge_units.cuh"
+#include "merge_tiles.cuh"
+#include "merge_long.cuh"
 #include "scan.cuh"
 
 using namespace spg;
@@ -95,8 +97,15 @@ struct TimedLaunch {
     } while (0)
 
 // ------------------------------------------------------------------ memory ---------------
+// One stream-ordered pool per device, created on first use under a lock (plans may be created
+// from several host threads).  Its release threshold is unbounded: freed plan workspaces stay
+// cached for the next plan (no driver allocation per product); spgemm_trim_pool returns them.
 static cudaMemPool_t pool_for_device(int dev) {
-    static cudaMemPool_t pools[64] = {};
+    constexpr int kMaxDevices = 64;
+    static cudaMemPool_t pools[kMaxDevices] = {};
+    static std::mutex mu;
+    if (dev < 0 || dev >= kMaxDevices) return nullptr;   // callers fall back to cudaMallocAsync
+    std::lock_guard<std::mutex> lk(mu);
     if (!pools[dev]) {
         cudaMemPoolProps props = {};
         props.allocType = cudaMemAllocationTypePinned;
@@ -178,6 +187,19 @@ struct spgemm_plan_s {
     int32_t *unit_row = nullptr;
     int64_t *nunits = nullptr;
     unsigned long long *unit_status = nullptr, *unit_ticket = nullptr;
+    // merge tiles (merge_tiles.cuh): tile table, look-back words
+    TileDesc *tiles = nullptr;
+    // long rows by column groups (merge_long.cuh)
+    bool long_groups = false;
+    int64_t lg_groups = 0, lg_slots = 0;
+    int64_t *lg_xoff = nullptr, *lg_yoff = nullptr, *lg_goff = nullptr, *lg_dense = nullptr;
+    int32_t *lg_scol = nullptr, *lg_gcnt = nullptr, *lg_glo = nullptr, *lg_gnum = nullptr;
+    float *lg_sval = nullptr;
+    int8_t *lg_gkind = nullptr;
+    unsigned long long *lg_ctr = nullptr;   // [0] row ticket, [1] dense-group count
+    int64_t *tile_cnt = nullptr, *tile_base = nullptr;
+    unsigned long long *tile_status = nullptr;
+    int64_t tiles_max = 0;
     int64_t nnz_c = -1;
     int state = 0;  // 1 planned, 2 expanded, 3 merged
 };
@@ -234,6 +256,12 @@ static inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 static inline unsigned grid_for(int64_t n, int threads, int64_t cap = 148 * 64) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(n, threads), cap));
 }
+
+// merge selection: the tile merge (merge_tiles.cuh, default) places C at the head of the Ĉ arrays;
+// options.reserved[5] = 1 or a legacy bin variant in reserved[0] selects the per-bin merge +
+// compaction (merge.cuh), reserved[0] = 4 the fused unit merge (merge_units.cuh)
+static inline bool use_tile_merge(const spgemm_options_t &o) { return o.reserved[0] == 0 && o.reserved[5] == 0; }
+static inline bool c_in_place(const spgemm_options_t &o) { return use_tile_merge(o) || o.reserved[0] == kMergeFused; }
 
 // Large-smem kernels: opt-in shared memory size and resident blocks per SM, queried once per
 // (kernel, device, smem, threads) -- these runtime calls cost host microseconds on every step.
@@ -494,6 +522,11 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         if (p->nnz_b > 0)
             LAUNCH("validate", s, k_validate_idx<<<grid_for(cdiv(p->nnz_b, 8), 256, 1 << 30), 256, 0, s>>>(
                 p->b_rowptr, p->b_colidx, K, p->nnz_b, p->n, flag, 8));
+        // the workload kernels below index rowwork / deg / cursors by a_rowidx: reject bad indices
+        // before any of them runs (an out-of-range row would write outside the plan's arrays)
+        CK(cudaMemcpyAsync(&hs, p->scal, sizeof(hs), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hs.invalid) return fail(SPGEMM_ERR_INVALID_INPUT, "malformed indices (range / order) in A or B");
     }
 
     // ---- stage (1): workload analysis -------------------------------------------------
@@ -658,22 +691,54 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
                                                                                   nruns));
             TRY(scan_excl(p, nruns, p->nlim, p->run_start, s, "lim_scan"));
         }
+        // default merge: long rows by column groups (merge_long.cuh) when the plan has their column
+        // ranges and every row fits the partition kernel's tables; else the legacy long-row kernels
+        p->long_groups = use_tile_merge(o) && col_range && p->n <= (1ll << 27) &&
+                         (int64_t)p->h_scal.lim_max_L <= kLongMaxL && p->opt.reserved[6] != 1;
+        if (p->long_groups) {
+            TRY(palloc(p, &p->lg_xoff, p->nlim + 1, s));
+            TRY(palloc(p, &p->lg_yoff, p->nlim + 1, s));
+            {
+                Temp tx(s), ty(s);
+                int64_t *xs, *ys;
+                TRY(talloc(p, tx, &xs, p->nlim));
+                TRY(talloc(p, ty, &ys, p->nlim));
+                LAUNCH("long_sizes", s, k_long_sizes<<<grid_for(p->nlim, 256), 256, 0, s>>>(lrows, p->nlim, p->rowwork,
+                                                                                           xs, ys));
+                TRY(scan_excl(p, xs, p->nlim, p->lg_xoff, s, "long_sizes"));
+                TRY(scan_excl(p, ys, p->nlim, p->lg_yoff, s, "long_sizes"));
+            }
+            // host bounds (no sync): sum pad(Lv) <= limited slots; sum of group bounds <= 4 slots / cap + 8 rows
+            p->lg_slots = (int64_t)p->h_scal.lim_slots + 16;
+            p->lg_groups = 4 * ((int64_t)p->h_scal.lim_slots / kGroupCap + 1) + 8 * p->nlim + 8;
+            TRY(palloc(p, &p->lg_scol, p->lg_slots, s));
+            TRY(palloc(p, &p->lg_sval, p->lg_slots, s));
+            TRY(palloc(p, &p->lg_goff, p->lg_groups, s));
+            TRY(palloc(p, &p->lg_gcnt, p->lg_groups, s));
+            TRY(palloc(p, &p->lg_glo, p->lg_groups, s));
+            TRY(palloc(p, &p->lg_gkind, p->lg_groups, s));
+            TRY(palloc(p, &p->lg_dense, p->lg_groups, s));
+            TRY(palloc(p, &p->lg_gnum, p->nlim, s));
+            TRY(palloc(p, &p->lg_ctr, 2, s));
+        }
         p->lim_runs = (int64_t)p->h_scal.lim_runs;
         p->lim_max_deg = (int64_t)p->h_scal.lim_max_deg;
         p->lim_max_L = (int64_t)p->h_scal.lim_max_L;
-        TRY(palloc(p, &p->run_base, p->lim_runs, s));
-        TRY(palloc(p, &p->run_len, p->lim_runs, s));
-        LAUNCH("lim_runs", s, k_lim_runs<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
-            p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->base, p->lim_index, p->run_start, p->run_fill,
-            p->run_base, p->run_len));
         p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
-        p->stage_cap = p->lim_max_L;   // whole-row scratch (dense rows are regrouped by window)
-        TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
-        TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
-        p->lim_max_deg += 1;   // per-block stride of the cursor / cnt scratch (cnt holds R+1 offsets)
-        TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
-        TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
-        TRY(palloc(p, &p->row_counter, 1, s));
+        if (!p->long_groups) {   // legacy long-row kernels: run lists + per-CTA whole-row scratch
+            TRY(palloc(p, &p->run_base, p->lim_runs, s));
+            TRY(palloc(p, &p->run_len, p->lim_runs, s));
+            LAUNCH("lim_runs", s, k_lim_runs<<<(unsigned)cdiv(cdiv(p->nnz_a, 8), 256), 256, 0, s>>>(
+                p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->base, p->lim_index, p->run_start, p->run_fill,
+                p->run_base, p->run_len));
+            p->stage_cap = p->lim_max_L;   // whole-row scratch (dense rows are regrouped by window)
+            TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
+            TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
+            p->lim_max_deg += 1;   // per-block stride of the cursor / cnt scratch (cnt holds R+1 offsets)
+            TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
+            TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
+            TRY(palloc(p, &p->row_counter, 1, s));
+        }
     }
     // merge state; Ĉ itself is allocated by spgemm_expand (or is the caller's C, spgemm_execute)
     const bool fused = p->opt.reserved[0] == kMergeFused;
@@ -892,6 +957,134 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     return SPGEMM_OK;
 }
 
+// B-Limited rows (merge.cuh): merged in place at the head of their Ĉ bucket, ccount[i] = length
+static int merge_limited_in_place(spgemm_plan_s *p, cudaStream_t s) {
+    if (p->nlim == 0) return SPGEMM_OK;
+    CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
+    LimitedArgs g;
+    g.rows = p->row_order + p->row_starts[kRowBucketLim0];
+    g.nrows = p->nlim;
+    g.rowoff = p->rowoff;
+    g.rowwork = p->rowwork;
+    g.run_start = p->run_start;
+    g.run_base = p->run_base;
+    g.run_len = p->run_len;
+    g.chat_col = p->chat_col;
+    g.chat_val = p->chat_val;
+    g.ccount = p->ccount;
+    g.scratch_cursor = p->scr_cursor;
+    g.scratch_cnt = p->scr_cnt;
+    g.scratch_col = p->scr_col;
+    g.scratch_val = p->scr_val;
+    g.max_deg = p->lim_max_deg;
+    g.stage_cap = p->stage_cap;
+    g.row_counter = p->row_counter;
+    g.out_col = nullptr;   // merged in place
+    g.out_val = nullptr;
+    g.out_off = nullptr;
+    g.skip_small = 1;
+    g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
+    if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
+    g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
+    // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
+    // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
+    TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
+    TRY(kernel_occupancy((const void *)k_merge_limited, kLimSmem, 0, nullptr));
+    LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
+    return SPGEMM_OK;
+}
+
+// Default merge (merge_tiles.cuh): B-Limited rows in place, then one persistent kernel over the tiles
+// (short-row groups and long-row chunks) in row order, C placed by look-back at the head of Ĉ.
+static int merge_tiles_path(spgemm_plan_s *p, cudaStream_t s) {
+    const int64_t M = p->m;
+    if (M == 0) {
+        CK(cudaMemsetAsync(p->crowptr, 0, 8, s));
+        return SPGEMM_OK;
+    }
+    CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
+    LongTables lt{};
+    if (p->nlim > 0 && p->long_groups) {
+        // B-Limited rows: column-group partition (limit_ctas_per_sm partition CTAs per SM, longest
+        // rows first), then the dense groups merged in place in the scratch
+        CK(cudaMemsetAsync(p->lg_ctr, 0, 16, s));
+        LongArgs la;
+        la.rows = p->row_order + p->row_starts[kRowBucketLim0];
+        la.nrows = p->nlim;
+        la.rowoff = p->rowoff;
+        la.rowwork = p->rowwork;
+        la.rowmn = p->rowmn;
+        la.rowmx = p->rowmx;
+        la.col = p->chat_col;
+        la.val = p->chat_val;
+        la.xoff = p->lg_xoff;
+        la.yoff = p->lg_yoff;
+        la.scol = p->lg_scol;
+        la.sval = p->lg_sval;
+        la.g_off = p->lg_goff;
+        la.g_cnt = p->lg_gcnt;
+        la.g_lo = p->lg_glo;
+        la.g_kind = p->lg_gkind;
+        la.g_num = p->lg_gnum;
+        la.dense_list = p->lg_dense;
+        la.dense_count = p->lg_ctr + 1;
+        la.counter = p->lg_ctr;
+        int occ = 0;
+        TRY(kernel_occupancy((const void *)k_long_partition, kPartSmem, kPartT, &occ));
+        const int64_t grid = std::min<int64_t>((int64_t)p->num_sms * std::min(std::max(occ, 1), p->opt.limit_ctas_per_sm),
+                                               p->nlim);
+        LAUNCH("merge_long_partition", s, k_long_partition<<<(unsigned)grid, kPartT, kPartSmem, s>>>(la));
+        TRY(kernel_occupancy((const void *)k_long_dense, kDenseSmem, kDenseT, nullptr));
+        LAUNCH("merge_long_dense", s, k_long_dense<<<(unsigned)p->num_sms, kDenseT, kDenseSmem, s>>>(
+            p->lg_dense, p->lg_ctr + 1, p->lg_goff, p->lg_gcnt, p->lg_glo, p->lg_gkind, p->lg_scol, p->lg_sval));
+        lt.lim_index = p->lim_index;
+        lt.yoff = p->lg_yoff;
+        lt.g_num = p->lg_gnum;
+        lt.g_off = p->lg_goff;
+        lt.g_cnt = p->lg_gcnt;
+        lt.g_kind = p->lg_gkind;
+    } else {
+        TRY(merge_limited_in_place(p, s));
+    }
+    const int64_t nch = cdiv(M, kTileRowChunk);
+    if (!p->tiles) {
+        // short tiles <= M; long-row tiles <= groups + merged chunks (<= groups + slots / chunk), or
+        // in-place chunks <= nlim + nnz(Ĉ) / kCopyChunk
+        p->tiles_max = M + p->nlim + p->chat_cap / kCopyChunk + 2 * p->lg_groups + 1;
+        TRY(palloc(p, &p->tiles, p->tiles_max, s));
+        TRY(palloc(p, &p->tile_cnt, nch, s));
+        TRY(palloc(p, &p->tile_base, nch + 1, s));
+        TRY(palloc(p, &p->tile_status, p->tiles_max + 2, s));
+    }
+    LAUNCH("merge_tiles_table", s, k_tile_table<false><<<(unsigned)cdiv(nch * 32, 128), 128, 0, s>>>(
+        p->rowoff, p->row_cls, p->ccount, lt, M, p->tile_cnt, nullptr, nullptr));
+    TRY(scan_excl(p, p->tile_cnt, nch, p->tile_base, s, "merge_tiles_table"));
+    LAUNCH("merge_tiles_table", s, k_tile_table<true><<<(unsigned)cdiv(nch * 32, 128), 128, 0, s>>>(
+        p->rowoff, p->row_cls, p->ccount, lt, M, nullptr, p->tile_base, p->tiles));
+    CK(cudaMemsetAsync(p->tile_status, 0, (p->tiles_max + 2) * 8, s));
+    TileArgs ta;
+    ta.tiles = p->tiles;
+    ta.ntiles = p->tile_base + nch;
+    ta.rowoff = p->rowoff;
+    ta.rowwork = p->rowwork;
+    ta.ccount = p->ccount;
+    ta.col = p->chat_col;
+    ta.val = p->chat_val;
+    ta.crowptr = p->crowptr;
+    ta.M = M;
+    ta.status = p->tile_status;
+    ta.ticket = p->tile_status + p->tiles_max + 1;
+    ta.lt = lt;
+    ta.scol = p->lg_scol;
+    ta.sval = p->lg_sval;
+    using TS = TileSmem<kTileThreads, kTileEPT>;
+    auto kern = k_merge_tiles<kTileThreads, kTileEPT>;
+    int occ = 0;
+    TRY(kernel_occupancy((const void *)kern, TS::kBytes, kTileThreads, &occ));
+    LAUNCH("merge_tiles", s, kern<<<(unsigned)(p->num_sms * std::max(occ, 1)), kTileThreads, TS::kBytes, s>>>(ta));
+    return SPGEMM_OK;
+}
+
 static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
     const int64_t M = p->m;
     if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
@@ -993,8 +1186,10 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     p->last_stream = s;
     CK(cudaSetDevice(p->dev));
     const int64_t M = p->m;
-    p->c_in_chat = p->opt.reserved[0] == kMergeFused;
-    TRY(p->c_in_chat ? merge_fused(p, s) : merge_bins(p, s));
+    p->c_in_chat = c_in_place(p->opt);
+    if (use_tile_merge(p->opt)) TRY(merge_tiles_path(p, s));
+    else if (p->opt.reserved[0] == kMergeFused) TRY(merge_fused(p, s));
+    else TRY(merge_bins(p, s));
     CK(cudaMemcpyAsync(&p->nnz_c, p->crowptr + M, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     p->state = 3;
@@ -1015,7 +1210,7 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
     C->nnz = p->nnz_c;
     const int64_t nnz = p->nnz_c;
     if (p->c_in_chat) {
-        // fused merge: C is compact at the head of the Ĉ arrays (merge_units.cuh)
+        // tile / fused merge: C is compact at the head of the Ĉ arrays (merge_tiles.cuh, merge_units.cuh)
         const cudaMemcpyKind kind = C->where == SPGEMM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
         CK(cudaMemcpyAsync(C->rowptr, p->crowptr, (p->m + 1) * 8, kind, s));
         if (nnz > 0 && C->colidx != p->chat_col) {
@@ -1075,7 +1270,7 @@ int spgemm_execute(spgemm_plan_t p, spgemm_alloc_fn alloc, void *ctx, int32_t ou
         return fail(SPGEMM_ERR_INVALID_ARGUMENT, "bad out_where");
     if (p->state != 1) return fail(SPGEMM_ERR_STATE, "spgemm_execute needs a fresh plan");
     C->where = out_where;
-    if (out_where == SPGEMM_DEVICE && p->opt.reserved[0] == kMergeFused) {
+    if (out_where == SPGEMM_DEVICE && c_in_place(p->opt)) {
         // device C: its column / value arrays (capacity nnz(Ĉ) slots) hold Ĉ during the merge and
         // C at their head afterwards -- no copy, no second nnz(Ĉ)-sized buffer
         C->rowptr = (int64_t *)alloc((size_t)(p->m + 1) * 8, out_where, ctx);

@@ -98,28 +98,40 @@ def concat_row_blocks(blocks: List[CSR]) -> CSR:
 
 
 def gather_row_blocks(C: CSR, dst: int = 0) -> CSR | None:
-    """Gather every rank's row block of C to rank ``dst`` (None on the other ranks)."""
+    """Gather every rank's row block of C to rank ``dst`` (None on the other ranks).  Rank ``dst``
+    allocates C once and receives every block straight into its slice (no concatenation copy);
+    the received row pointers are shifted by the preceding blocks' nnz afterwards."""
     rank, world = dist.get_rank(), dist.get_world_size()
     dev = C.rowptr.device
     meta = torch.tensor([C.nrows, C.nnz], dtype=torch.int64, device=dev)
     metas = [torch.empty_like(meta) for _ in range(world)]
     dist.all_gather(metas, meta)
     if rank != dst:
-        for t in (C.rowptr, C.colidx, C.val):
+        for t in (C.rowptr, C.colidx[:C.nnz], C.val[:C.nnz]):
             if t.numel():
                 dist.send(t.contiguous(), dst=dst)
         return None
-    blocks = []
-    for r in range(world):
-        nrows, nnz = (int(x) for x in metas[r].tolist())
+    sizes = [tuple(int(x) for x in m.tolist()) for m in metas]
+    M = sum(s[0] for s in sizes)
+    NNZ = sum(s[1] for s in sizes)
+    rowptr = torch.empty(M + 1, dtype=torch.int64, device=dev)
+    colidx = torch.empty(NNZ, dtype=torch.int32, device=dev)
+    val = torch.empty(NNZ, dtype=torch.float32, device=dev)
+    r0 = e0 = 0
+    for r, (nrows, nnz) in enumerate(sizes):
+        rp = rowptr[r0:r0 + nrows + 1]
+        ci, vv = colidx[e0:e0 + nnz], val[e0:e0 + nnz]
         if r == rank:
-            blocks.append(C)
-            continue
-        rowptr = torch.empty(nrows + 1, dtype=torch.int64, device=dev)
-        colidx = torch.empty(nnz, dtype=torch.int32, device=dev)
-        val = torch.empty(nnz, dtype=torch.float32, device=dev)
-        for t in (rowptr, colidx, val):
-            if t.numel():
-                dist.recv(t, src=r)
-        blocks.append(CSR(nrows, C.ncols, rowptr, colidx, val))
-    return concat_row_blocks(blocks)
+            rp.copy_(C.rowptr)
+            if nnz:
+                ci.copy_(C.colidx[:nnz])
+                vv.copy_(C.val[:nnz])
+        else:
+            for t in (rp, ci, vv):
+                if t.numel():
+                    buf = t if t.is_contiguous() else torch.empty_like(t)
+                    dist.recv(buf, src=r)
+        rp.add_(e0)   # block-local row pointers -> global (the next block overwrites rp[-1] with the same value)
+        r0 += nrows
+        e0 += nnz
+    return CSR(M, C.ncols, rowptr, colidx, val)

@@ -21,7 +21,8 @@ Workload recipes (stated in DESIGN.md §3, "input recipe"):
 
 Values are a counter-based hash of (row, col, seed) so any entry can be
 recomputed independently; ``kind='real'`` gives values in [0.5, 1.5) on a
-2**-23 grid (exactly representable in fp32), ``kind='int'`` gives {1,2,3,4}.
+2**-23 grid (exactly representable in fp32), ``kind='int'`` gives {1,2,3,4},
+``kind='pm1'`` gives +-1 (exact sums, many of them exactly zero).
 """
 from __future__ import annotations
 
@@ -56,6 +57,8 @@ def edge_values(rows: np.ndarray, cols: np.ndarray, seed: int, kind: str = "real
         return (0.5 + (h >> np.uint64(41)).astype(np.float64) * 2.0 ** -23).astype(np.float32)
     if kind == "int":
         return (1 + (h >> np.uint64(62))).astype(np.float32)
+    if kind == "pm1":   # +-1: exact integer sums with frequent exact cancellation (computed zeros)
+        return np.where((h >> np.uint64(63)) == 1, -1.0, 1.0).astype(np.float32)
     if kind == "signed":
         v = (0.5 + (h >> np.uint64(41)).astype(np.float64) * 2.0 ** -23)
         sign = np.where((h & np.uint64(1)) == 1, -1.0, 1.0)
@@ -113,6 +116,8 @@ def _powerlaw_weights(n: int, m: float, gamma: float, wmax: float) -> np.ndarray
     lo, hi = 1e-6, 1e12
     for _ in range(200):
         mid = np.sqrt(lo * hi)
+        if mid <= lo or mid >= hi:   # converged to adjacent doubles: later steps change nothing
+            break
         w = (i + mid) ** (-p)
         w *= m / w.sum()
         if w[0] > wmax:
@@ -121,6 +126,15 @@ def _powerlaw_weights(n: int, m: float, gamma: float, wmax: float) -> np.ndarray
             hi = mid
     w = (i + hi) ** (-p)
     return w * (m / w.sum())
+
+
+def _inverse_cdf(cdf: np.ndarray, u: np.ndarray) -> np.ndarray:
+    """np.searchsorted(cdf, u, side='right'), element for element; the draws are searched in sorted
+    order (a cache-friendly sweep of the table) and put back in draw order."""
+    order = np.argsort(u, kind="stable")
+    out = np.empty(u.size, dtype=np.int64)
+    out[order] = np.searchsorted(cdf, u[order], side="right")
+    return out
 
 
 def chung_lu_edges(n: int, m: int, gamma_out: float, gamma_in: float, max_out: float,
@@ -140,8 +154,8 @@ def chung_lu_edges(n: int, m: int, gamma_out: float, gamma_in: float, max_out: f
     m_draw = m // 2 if symmetric else m
     cdf_o = np.cumsum(w_out)
     cdf_i = np.cumsum(w_in)
-    src = np.searchsorted(cdf_o, rng.random(m_draw) * cdf_o[-1], side="right")
-    dst = np.searchsorted(cdf_i, rng.random(m_draw) * cdf_i[-1], side="right")
+    src = _inverse_cdf(cdf_o, rng.random(m_draw) * cdf_o[-1])
+    dst = _inverse_cdf(cdf_i, rng.random(m_draw) * cdf_i[-1])
     np.minimum(src, n - 1, out=src)
     np.minimum(dst, n - 1, out=dst)
     perm = rng.permutation(n)

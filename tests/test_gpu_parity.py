@@ -262,7 +262,7 @@ def test_integer_values_exact():
     np.testing.assert_array_equal(C.val.cpu().numpy().astype(np.float64), val)   # exact
 
 
-def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False):
+def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False, kind="real"):
     rng = np.random.default_rng(seed)
     ar, ac = np.nonzero(rng.random((m, k)) < a_density)
     br = np.repeat(np.arange(k), run_len)
@@ -275,8 +275,8 @@ def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False)
     bc = np.concatenate(cols)
     if narrow:
         bc[:run_len] = np.arange(run_len) * 3
-    return synth.from_coo("wide", m, k, n, (ar, ac, synth.edge_values(ar, ac, seed)),
-                          (br, bc, synth.edge_values(br, bc, seed + 1)))
+    return synth.from_coo("wide", m, k, n, (ar, ac, synth.edge_values(ar, ac, seed, kind)),
+                          (br, bc, synth.edge_values(br, bc, seed + 1, kind)))
 
 
 @pytest.mark.parametrize("m,k,n,dens,run_len,hub,narrow", [
@@ -430,57 +430,69 @@ def test_validation_rejects_malformed():
         spg.Plan(A, B)
 
 
-# ------------------------------------------------------------------ full sizes -------------
-@pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", FUSED), ("C3", {}), ("C4", {}), ("C5", {}),
-                                       ("C5", {"chunks": 4}), ("AB17", {}), ("AB18", {})])
-def test_full_size_sampled(name, opts):
-    """BASELINE.json configs[1] at full size, in the bench's launch configuration: sampled rows
-    compared with the oracle one by one, plus whole-matrix properties."""
-    inp = synth.make_inputs(name, seed=1)
+# ------------------------------------------------------------------ computed zeros ----------
+def _assert_exact(C, inp):
+    rowptr, col, val = oracle.gustavson(inp)
+    np.testing.assert_array_equal(C.rowptr.cpu().numpy(), rowptr)
+    np.testing.assert_array_equal(C.colidx.cpu().numpy(), col)
+    np.testing.assert_array_equal(C.val.cpu().numpy().astype(np.float64), val)   # +-1 sums: exact
+    return val
+
+
+def test_computed_zeros_hand():
+    """c_0j = (+1)(b_0j) + (-1)(b_1j) with b_0* = b_1*: every entry of row 0 cancels exactly and is
+    still stored (R7: "merged into unique elements", PAPER.md L453-L455 L)."""
+    cols = np.array([3, 17, 40, 41], dtype=np.int32)
+    br = np.repeat(np.array([0, 1], dtype=np.int32), cols.size)
+    bc = np.tile(cols, 2)
+    bv = np.tile(np.array([0.5, 1.25, 2.0, 3.0], dtype=np.float32), 2)
+    inp = synth.from_coo("cancel", 2, 2, 64, (np.array([0, 0, 1]), np.array([0, 1, 1]),
+                                              np.array([1.0, -1.0, 2.0], dtype=np.float32)), (br, bc, bv))
     A, B = spg.from_inputs(inp, "cuda")
-    torch.cuda.empty_cache()
-    ca, rb, work = stages.pair_workload(inp)
-    if "chunks" in opts:     # north star C5: chunked expansion (row blocks in turn)
-        spg.trim_pool()      # (earlier full-size products left their workspaces cached)
-        C = spg.matmul_chunked(A, B, opts["chunks"])
-    else:
+    for opts in ({}, dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)):
+        C = spg.matmul(A, B, **opts)
+        val = _assert_exact(C, inp)
+        assert C.rowptr.cpu().tolist() == [0, 4, 8]
+        assert np.all(val[:4] == 0) and np.all(C.val[:4].cpu().numpy() == 0)
+
+
+@pytest.mark.parametrize("opts", [{}, dict(beta=10.0), dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)])
+def test_computed_zeros_pm1(opts):
+    """+-1 values (synth kind 'pm1'): thousands of entries cancel exactly; the structure keeps them and
+    the values are exact (short rows, the paper's β-Limiting rows, and the legacy bins)."""
+    inp = synth.make_inputs("C1", seed=2, values="pm1")
+    A, B = spg.from_inputs(inp, "cuda")
+    val = _assert_exact(spg.matmul(A, B, **opts), inp)
+    assert (val == 0).sum() > 1000
+
+
+def test_computed_zeros_long_rows():
+    """Exact cancellation inside B-Limited rows (padded bucket > 4096 slots)."""
+    inp = _wide_inputs(40, 120, 70000, 0.25, 300, 3, narrow=True, kind="pm1")
+    A, B = spg.from_inputs(inp, "cuda")
+    with spg.Plan(A, B) as p:
+        assert p.stats()["n_rows_bin"][5] > 0
+        C = p.execute()
+    val = _assert_exact(C, inp)
+    assert (val == 0).sum() > 0
+
+
+# ------------------------------------------------------------------ overflow regression -----
+def test_limited_bucket_overflow_many_heavy_buckets():
+    """one limited row of <= 9216 slots in which >= 128 buckets overflow (69 runs of
+    the same 130 columns spread over ~130K columns: 130 buckets of 69 equal keys).  The overflow flag
+    of the bucket scan must not wrap; the row takes the fallback and matches the oracle."""
+    k, run = 69, 130
+    cols = np.sort(np.random.default_rng(4).choice(130_000, run, replace=False)).astype(np.int32)
+    br = np.repeat(np.arange(k, dtype=np.int32), run)
+    bc = np.tile(cols, k)
+    ar = np.zeros(k, dtype=np.int32)
+    ac = np.arange(k, dtype=np.int32)
+    inp = synth.from_coo("heavy", 1, k, 130_000, (ar, ac, synth.edge_values(ar, ac, 1)),
+                         (br, bc, synth.edge_values(br, bc, 2)))
+    A, B = spg.from_inputs(inp, "cuda")
+    for opts in ({}, dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)):
         with spg.Plan(A, B, **opts) as p:
-            st = p.stats()
+            assert p.stats()["n_rows_bin"][5] == 1   # the row is B-Limited (9108 padded slots)
             C = p.execute()
-        assert st["nnz_chat"] == int(work.sum())
-    # (C3 / C5 hold ~9e9 entries: everything below stays on the GPU but the sampled rows)
-    rowptr = C.rowptr.cpu().numpy()
-    assert rowptr[-1] == C.nnz
-    rng = np.random.default_rng(0)
-    rowwork = stages.row_workload(inp)
-    heavy = np.argsort(rowwork)[-200:]
-    rows = np.unique(np.concatenate([rng.integers(0, inp.m, 3000), heavy])).astype(np.int32)
-    orp, ocol, oval = oracle.gustavson(inp, rows=rows)
-    for t, i in enumerate(rows):
-        gc = C.colidx[rowptr[i]:rowptr[i + 1]].cpu().numpy()
-        np.testing.assert_array_equal(gc, ocol[orp[t]:orp[t + 1]])
-        ov = oval[orp[t]:orp[t + 1]]
-        gv = C.val[rowptr[i]:rowptr[i + 1]].cpu().numpy().astype(np.float64)
-        assert np.all(np.abs(gv - ov) <= RTOL * np.abs(ov))
-    # canonical CSR (columns strictly ascending in every row) and C 1 = A (B 1), in chunks
-    rp = C.rowptr
-    lhs = torch.zeros(inp.m, dtype=torch.float64, device="cuda")
-    chunk = 1 << 27
-    for q0 in range(0, C.nnz, chunk):
-        q1 = min(C.nnz, q0 + chunk)
-        pos = torch.arange(q0, q1, device="cuda")
-        row = torch.searchsorted(rp, pos, right=True) - 1
-        lhs.index_add_(0, row, C.val[q0:q1].double())
-        if q1 - q0 > 1:
-            same_row = row[1:] == row[:-1]
-            asc = C.colidx[q0 + 1:q1] > C.colidx[q0:q1 - 1]
-            assert bool(torch.all(asc | ~same_row))
-        if q0 > 0 and row[0] == torch.searchsorted(rp, torch.tensor([q0 - 1], device="cuda"), right=True)[0] - 1:
-            assert int(C.colidx[q0]) > int(C.colidx[q0 - 1])
-        del pos, row
-    ones_b = np.bincount(np.repeat(np.arange(inp.k), np.diff(inp.b_rowptr)), weights=inp.b_val.astype(np.float64),
-                         minlength=inp.k)
-    a_cols = np.repeat(np.arange(inp.k), ca)
-    rhs = np.bincount(inp.a_rowidx, weights=inp.a_val.astype(np.float64) * ones_b[a_cols], minlength=inp.m)
-    lhs = lhs.cpu().numpy()
-    np.testing.assert_allclose(lhs, rhs, rtol=1e-5)
+        assert_c_matches(C, inp)

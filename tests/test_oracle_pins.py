@@ -299,3 +299,27 @@ def test_thresholds_formulas():
     assert stages.limiting_threshold(100000, 100, 10.0, 4096) == 100
     assert stages.limiting_threshold(10 ** 9, 100, 10.0, 4096) == 4096
     assert stages.limiting_threshold(10 ** 9, 100, 0.0, 4096) == 4096
+
+
+def test_chat_row_offsets_hand_example():
+    """Ĉ row offsets = exclusive scan of the row-wise nnz (L289-L291 R), pinned by the hand example's
+    rowwork 4 2 3 0 -> offsets 0 4 6 9 9 (tests/golden/hand_example_4x4.txt)."""
+    inp, sec, sc = _inputs_from_golden("hand_example_4x4.txt")
+    np.testing.assert_array_equal(stages.chat_row_offsets(stages.row_workload(inp)), sc["rowoff"])
+    np.testing.assert_array_equal(stages.chat_row_offsets(np.zeros(0, np.int64)), [0])
+
+
+def test_gather_order_hand_list():
+    """R5 packing order of the B-Gathering lists against a hand-derived list
+    (tests/golden/r5_gather_order.txt): bins by 2^(n-1) < t <= 2^n, inside a bin by
+    floor(log2 nnz(a_*k)) then k -- a plain k order or a swapped key fails it."""
+    kv = {r[0]: [int(x) for x in r[1:]] for r in read_kv("r5_gather_order.txt")}
+    ca = np.array(kv["ca"], dtype=np.int64)
+    rb = np.array(kv["rb"], dtype=np.int64)
+    work = ca * rb
+    cls = stages.classify_pairs(ca, rb, work, t_dom=10 ** 9, split_ca_max=10 ** 9)
+    assert list(np.nonzero(cls == stages.LOW)[0]) == [0, 1, 2, 3, 4, 6, 8, 9, 10]
+    assert cls[5] == stages.NORMAL and cls[7] == stages.EMPTY
+    lists = stages.gather_lists(ca, rb, cls)
+    for b in range(6):
+        np.testing.assert_array_equal(lists[b], kv[f"bin{b}"])
