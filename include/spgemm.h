@@ -18,11 +18,12 @@
  *   spgemm_expand   (3) expansion: every product (i, j, a_ik*b_kj) written into the
  *                       row-bucketed intermediate matrix Ĉ (L321-L323 L).
  *   spgemm_merge    (4) merge: per Ĉ row, sort by column + segmented reduce (fp64
- *                       accumulation, one rounding to fp32); long rows B-Limited.  Default
- *                       (merge tiles): C is placed by a decoupled look-back at the head of
- *                       the Ĉ arrays, in place -- no separate compaction pass.
- *   spgemm_output       copy of C (head of the Ĉ arrays) into caller buffers; nothing to copy
- *                       when the caller's arrays are the Ĉ arrays (spgemm_execute, device C).
+ *                       accumulation, one rounding to fp32); long rows B-Limited.  Rows are
+ *                       merged in place in their Ĉ buckets (default), or -- tile merge,
+ *                       options.reserved[5] = 2 -- placed by a decoupled look-back at the head
+ *                       of the Ĉ arrays (C in place, no compaction pass).
+ *   spgemm_output       CSR compaction of the merged rows into caller buffers (tile merge: a copy
+ *                       of C's head, nothing when the caller's arrays are the Ĉ arrays).
  *   spgemm_execute  = expand + merge + allocate C (callback) + output.
  *
  * Conventions for every call:
@@ -132,9 +133,14 @@ typedef struct {
                                  [3] 1 = row-product expansion (the paper's comparison order);
                                  [4] 1 = no per-row column range from the plan (the merge
                                      reduces each row's min / max column itself);
-                                 [5] 1 = legacy per-bin merge + CSR compaction (merge.cuh; also
-                                     selected by any bin variant in [0]); 0 with [0] = 0: the
-                                     merge-tile kernel (merge_tiles.cuh), C placed in place     */
+                                 [5] 2 = tile merge (merge_tiles.cuh, merge_long.cuh): tiles of
+                                     short rows and column groups of the long rows in row order,
+                                     C placed by look-back in place, no compaction ([0] = 0);
+                                 [6] 1 = with [5] = 2: long rows by the per-bin long-row kernels
+                                     (merged in place, then moved) instead of column groups;
+                                 [7] > 0: fixed B-Splitting factor for every Dominator (the
+                                     Fig. 11 sweep; capped at the column's power of two);
+                                 [8] 1 = record per-SM busy times for the LBI (SPGEMM_VIEW_LBI) */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */
@@ -171,7 +177,12 @@ typedef enum {
                                     range; computed in spgemm_plan for rows whose padded Ĉ
                                     bucket exceeds 256 slots; other rows 0x7f7f7f7f = unknown;
                                     size 0 with options.reserved[4] = 1)                       */
-    SPGEMM_VIEW_ROW_COLMAX = 12  /* int32[m]   last column of row i of C (unknown rows 0)     */
+    SPGEMM_VIEW_ROW_COLMAX = 12, /* int32[m]   last column of row i of C (unknown rows 0)     */
+    SPGEMM_VIEW_LBI = 13         /* uint64[2][257] with options.reserved[8] = 1, after the kernels ran:
+                                    per kernel (0 expansion, 1 B-Limited merge) [0] = first CTA start,
+                                    [1 + smid] = last CTA end on that SM (%globaltimer ns); the
+                                    load balancing index of PAPER.md Eq. (3) (L564-L577 R) is
+                                    mean_i(T_i) / max_i(T_i), T_i = [1 + i] - [0] over the SMs     */
 } spgemm_view;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;
@@ -203,7 +214,8 @@ int spgemm_output(spgemm_plan_t plan, spgemm_csr_out_t *C, void *stream);
 
 /* expand + merge + alloc(C arrays in `out_where`) + output.  C->rowptr/colidx/val are
  * set to the allocated buffers (owned by the caller).  Returns after `stream` holds C.
- * With a device C and the default merge (or the fused unit merge, options.reserved[0] = 4),
+ * With a device C and the tile merge (options.reserved[5] = 2) or the fused unit merge
+ * (options.reserved[0] = 4),
  * colidx / val are requested BEFORE the expansion with capacity nnz(Ĉ) (padded slots) >= nnz(C):
  * they hold Ĉ during the merge and C in their first C->nnz entries afterwards (one buffer for
  * both: no second nnz(Ĉ)-sized allocation, no copy). */

@@ -78,11 +78,17 @@ def classify_pairs(ca, rb, work, t_dom: int, split_ca_max: int):
 
 # --- (3) B-Splitting (L320-L415, Fig. 5) ----------------------------------------------------
 
-def splitting_factor(ca: int, blen: int, piece_work: int, split_ca_max: int) -> int:
+def splitting_factor(ca: int, blen: int, piece_work: int, split_ca_max: int, fixed_f: int = 0) -> int:
     """Smallest power of two f (L410-L413 L: "splitting factor (2^n)") such that each
     greedy piece of the column, ceil(ca/f) entries, stays within piece_work products
     and split_ca_max computations per thread; f never exceeds the column length's
-    next power of two (one entry per piece)."""
+    next power of two (one entry per piece).  fixed_f > 0 (Fig. 11's sweep over the
+    splitting factor, L640-L687 L) imposes the factor, with the same cap."""
+    if fixed_f > 0:
+        f = 1
+        while f < fixed_f and f < ca:
+            f *= 2
+        return f
     f = 1
     while f < ca:
         chunk = -(-ca // f)
@@ -92,7 +98,7 @@ def splitting_factor(ca: int, blen: int, piece_work: int, split_ca_max: int) -> 
     return f
 
 
-def split_pieces(inp, cls, piece_work: int, b_tile: int, split_ca_max: int):
+def split_pieces(inp, cls, piece_work: int, b_tile: int, split_ca_max: int, fixed_f: int = 0):
     """Pieces (k, a_lo, a_hi, b_lo, b_hi) (absolute entry ranges into A's rowidx and
     B's colidx) for every dominator, in order of ascending k, then B tile, then A piece.
     The A column is split greedily: piece p takes entries [p*chunk, (p+1)*chunk)
@@ -108,7 +114,7 @@ def split_pieces(inp, cls, piece_work: int, b_tile: int, split_ca_max: int):
         b0, b1 = int(inp.b_rowptr[k]), int(inp.b_rowptr[k + 1])
         ca, rb = a1 - a0, b1 - b0
         blen = min(rb, b_tile)
-        f = splitting_factor(ca, blen, piece_work, split_ca_max)
+        f = splitting_factor(ca, blen, piece_work, split_ca_max, fixed_f)
         chunk = -(-ca // f)
         for bs in range(b0, b1, b_tile):
             be = min(b1, bs + b_tile)

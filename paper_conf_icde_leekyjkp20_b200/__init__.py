@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(_HERE, "libspgemm.so")
 
 SPGEMM_DEVICE, SPGEMM_HOST = 0, 1
 VIEW_WORK, VIEW_ROWWORK, VIEW_ROWOFF, VIEW_PAIR_CLASS, VIEW_PIECES, VIEW_GATHER, VIEW_ROW_CLASS, \
-    VIEW_CHAT_COL, VIEW_CHAT_VAL, VIEW_CROWPTR, VIEW_UNIT_PROFILE, VIEW_ROW_COLMIN, VIEW_ROW_COLMAX = range(13)
+    VIEW_CHAT_COL, VIEW_CHAT_VAL, VIEW_CROWPTR, VIEW_UNIT_PROFILE, VIEW_ROW_COLMIN, VIEW_ROW_COLMAX, VIEW_LBI = range(14)
 
 EXPORTED = ["spgemm_abi_version", "spgemm_last_error", "spgemm_default_options", "spgemm_plan",
             "spgemm_expand", "spgemm_merge", "spgemm_output", "spgemm_execute", "spgemm_get_stats",
@@ -236,6 +236,25 @@ class Plan:
         buf = np.empty(max(size.value, 1), dtype=np.uint8)
         _check(lib().spgemm_inspect(self.h, view, buf.ctypes.data_as(ctypes.c_void_p), buf.size, ctypes.byref(size)))
         return buf[: size.value].view(dtype)
+
+    def lbi(self) -> dict:
+        """Load balancing index (Eq. (3), L564-L577 R) of the expansion and of the B-Limited
+        merge kernel of this plan (plan created with reserved[8] = 1, after merge): mean over the
+        SMs of the SM's busy time T_i normalised by the longest, T_i = last CTA end on SM i - the
+        kernel's first CTA start (SMs that ran nothing count as 0)."""
+        import numpy as np
+        raw = self.inspect(VIEW_LBI, np.uint64).reshape(2, -1).astype(np.int64)
+        nsm = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+        out = {}
+        for name, row in zip(("expand", "merge_limited"), raw):
+            t0, ends = int(row[0]), row[1:1 + nsm]
+            if t0 <= 0 or ends.max() <= 0:   # (0xff.. = never started: -1 as int64)
+                out[name] = None
+                continue
+            busy = np.where(ends > 0, ends - t0, 0).astype(np.float64)
+            out[name] = {"lbi": float(busy.mean() / busy.max()), "max_ms": float(busy.max() / 1e6),
+                         "mean_ms": float(busy.mean() / 1e6)}
+        return out
 
     def destroy(self):
         if getattr(self, "h", None):

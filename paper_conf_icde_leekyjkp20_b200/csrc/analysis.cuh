@@ -238,12 +238,19 @@ struct SplitParams {
     int64_t piece_work;
     int32_t b_tile;
     int32_t split_ca_max;
+    int32_t fixed_f;      // > 0: every Dominator split by this factor (Fig. 11 sweep; capped at ca's)
 };
 
 // Splitting factor f = 2^n (L410-L413 L): smallest power of two whose greedy chunk of
 // ceil(ca/f) column entries keeps a piece within piece_work products and split_ca_max
-// computations per thread.
+// computations per thread.  A fixed factor (options.reserved[7], the Fig. 11 sweep) is used as
+// given, but never beyond the smallest power of two >= ca (one entry per piece).
 __device__ __forceinline__ int64_t splitting_factor(int64_t ca, int64_t blen, const SplitParams &p) {
+    if (p.fixed_f > 0) {
+        int64_t f = 1;
+        while (f < p.fixed_f && f < ca) f <<= 1;
+        return f;
+    }
     int64_t f = 1;
     while (f < ca) {
         int64_t chunk = (ca + f - 1) / f;

@@ -149,9 +149,11 @@ __device__ __forceinline__ int64_t lb_resolve(unsigned long long *status, int64_
     int64_t idx = u - 1 - lane;
     while (true) {
         unsigned long long s;
-        do {
+        while (true) {
             s = idx >= 0 ? ld_acquire_u64(status + idx) : kLbPre;
-        } while (__any_sync(0xffffffffu, (s >> 62) == 0));
+            if (!__any_sync(0xffffffffu, (s >> 62) == 0)) break;
+            __nanosleep(64);   // (a spinning warp takes issue slots from the SM's other warps)
+        }
         const unsigned pre = __ballot_sync(0xffffffffu, (s >> 62) == 2);
         int64_t v = (int64_t)(s & kLbMask);
         if (pre) {
@@ -164,6 +166,31 @@ __device__ __forceinline__ int64_t lb_resolve(unsigned long long *status, int64_
     }
     if (lane == 0) st_release_u64(status + u, kLbPre | (unsigned long long)(excl + agg));
     return excl;
+}
+
+// ---- load balancing index (Eq. (3), L564-L577 R): LBI = (1/N) sum_i cycles(SM_i) /
+// max cycles(SM), N = #SMs.  Opt-in recording (options.reserved[8] = 1): lbi[0] = the kernel's first
+// CTA start, lbi[1 + smid] = the last CTA end on that SM (%globaltimer, ns); the host takes
+// cycles(SM_i) = lbi[1 + i] - lbi[0].
+constexpr int kLbiSlots = 1 + 256;
+__device__ __forceinline__ unsigned long long gtimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ unsigned sm_id() {
+    unsigned s;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+    return s;
+}
+__device__ __forceinline__ void lbi_start(unsigned long long *lbi) {
+    if (lbi && threadIdx.x == 0) atomicMin(lbi, gtimer_ns());
+}
+__device__ __forceinline__ void lbi_end(unsigned long long *lbi) {   // (uniform: lbi is a kernel argument)
+    if (lbi) {
+        __syncthreads();
+        if (threadIdx.x == 0) atomicMax(lbi + 1 + (sm_id() & 255), gtimer_ns());
+    }
 }
 
 }  // namespace spg

@@ -120,7 +120,8 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     const Piece *__restrict__ pieces, const int64_t *__restrict__ uoff, int64_t npieces,
     const int64_t *__restrict__ tile_p0, const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ bp_col,
     const float *__restrict__ bp_val, const float *__restrict__ a_val, const int64_t *__restrict__ base,
-    int32_t *__restrict__ chat_col, float *__restrict__ chat_val) {
+    int32_t *__restrict__ chat_col, float *__restrict__ chat_val, unsigned long long *lbi) {
+    lbi_start(lbi);
     __shared__ int64_t s_uoff[kExpPieceCache + 1];
     __shared__ int64_t s_alo[kExpPieceCache];
     __shared__ int64_t s_bsrc[kExpPieceCache];
@@ -200,6 +201,7 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
                 }
         }
     }
+    lbi_end(lbi);
 }
 
 // ------------------------------------------------ row-product expansion (comparison) ---

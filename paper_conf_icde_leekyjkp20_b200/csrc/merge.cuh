@@ -1674,6 +1674,7 @@ struct LimitedArgs {
     int skip_small;
     unsigned long long *prof;     // NULL, or per-path clock totals [0..10) (tuning)
     int64_t coarse_cap;           // rows up to this many slots take the coarse-partition path
+    unsigned long long *lbi;      // NULL, or per-SM busy times (LBI, Eq. (3))
 };
 
 __device__ __forceinline__ void smem_add_f64(double *addr, double v) {
@@ -1699,6 +1700,7 @@ __device__ __forceinline__ int count_below(const int32_t *__restrict__ col, int6
 }
 
 __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g) {
+    lbi_start(g.lbi);
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ int sc[2 * kLimNW + 2];
     __shared__ int64_t row_sm;
@@ -2173,6 +2175,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         __syncthreads();
         rec(dense ? 2 : 3);
     }
+    lbi_end(g.lbi);
 }
 
 // Single-run rows: already sorted and duplicate-free; merged length = bucket length.

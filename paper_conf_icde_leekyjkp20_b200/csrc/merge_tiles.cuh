@@ -36,7 +36,7 @@ namespace spg {
 constexpr int kTileThreads = 512;
 constexpr int kTileEPT = 8;
 constexpr int kTileCap = kTileThreads * kTileEPT;   // 4096 slots (= kLimitCapacity: longer rows are B-Limited)
-constexpr int kTileMaxRows = 256;                   // rows of one tile (one thread per row in the row phases)
+constexpr int kTileMaxRows = kTileThreads;          // rows of one tile (every row owns >= 1 thread)
 constexpr int kTileRowChunk = 1024;                 // rows per warp of the tile-table builder
 constexpr int kCopyChunk = kTileThreads * 8;        // merged entries per long-row chunk tile
 static_assert(kTileCap >= kLimitCapacity, "every non-limited row must fit one tile");
@@ -94,11 +94,12 @@ __global__ void __launch_bounds__(128) k_tile_table(const int64_t *__restrict__ 
         const int nin = i1 - w0 < 32 ? (int)(i1 - w0) : 32;
         while (done < nin) {
             // rows [done, j) join the open tile; lane j is a B-Limited row or does not fit
-            const int64_t cc = (lane >= done && lane < nin) ? cap : 0;
+            // a short row owns ceil(cap / EPT) threads of the tile (>= its slots / EPT); a tile has T
+            const int64_t cc = (lane >= done && lane < nin) ? (cap + kTileEPT - 1) / kTileEPT : 0;
             const int64_t pre = warp_incl_sum(cc);
             const int64_t first = open >= 0 ? open : w0 + done;   // first row of the tile being grown
             const bool ev = lane >= done && lane < nin &&
-                            (lim || acc + pre > kTileCap || (w0 + lane) - first >= kTileMaxRows);
+                            (lim || acc + pre > kTileThreads || (w0 + lane) - first >= kTileMaxRows);
             const unsigned m = __ballot_sync(kFull, ev);
             const int j = m ? __ffs(m) - 1 : nin;
             if (j > done) {
@@ -149,7 +150,7 @@ __global__ void __launch_bounds__(128) k_tile_table(const int64_t *__restrict__ 
                 done = j + 1;
             } else {
                 open = w0 + j;   // row j starts the next tile
-                acc = __shfl_sync(kFull, cap, j);
+                acc = (__shfl_sync(kFull, cap, j) + kTileEPT - 1) / kTileEPT;
                 done = j + 1;
             }
         }
@@ -211,57 +212,96 @@ struct TileArgs {
     LongTables lt;                 // long-row groups (merge_long.cuh)
     int32_t *scol;                 // their scratch
     float *sval;
+    int debug;                     // options.reserved[1] (tuning only): 1 = no look-back (every tile
+                                   // writes at its own input position: wrong C, timing only), 2 =
+                                   // per-phase clock64 totals of thread 0 into prof[0..16)
+    unsigned long long *prof;
 };
+#define TILE_PH(k)                                                   \
+    do {                                                             \
+        if (prof_on) {                                               \
+            const long long _t = clock64();                          \
+            ph[k] += (unsigned long long)(_t - t_last);              \
+            t_last = _t;                                             \
+        }                                                            \
+    } while (0)
 
 template <int T, int EPT>
 struct TileSmem {
     static constexpr int kCap = T * EPT;
-    static constexpr int kNb = 2 * kCap;                  // sum over rows of 2^ceil(log2 Lv) <= 2 * slots
-    static constexpr int kHistWords = hidx(kNb) + 4;      // (+ the end-of-tile entry)
-    static constexpr int kRowWords = 8 * (kTileMaxRows + 1);
-    // layout: keys | vals (bulk copy target, then the sorted tile) | hist (bucket counts / starts; then
-    // merged values + slice carries) | binfo (bucket of every scattered slot; then merged keys) | rows
-    static constexpr int kBytes = kCap * 8 + kHistWords * 4 + kCap * 4 + kRowWords * 4;
-    static_assert(kHistWords * 4 >= kCap * 4 + T * 12, "merged values + carries alias the histogram");
+    static constexpr int kNb = 2 * kCap;   // row r's buckets live at [2 ro[r], 2 ro[r] + 2^ceil(log2 Lv)) < 2 ro[r+1]
+    static constexpr int kRowWords = 7 * (kTileMaxRows + 1);
+    // layout: keys | vals (bulk copy target, scatter target, then the merged tile) | hist (bucket counts /
+    // starts, then the sorted tile) | binfo (bucket of every scattered slot, then slice carries) | rows
+    static constexpr int kBytes = kCap * 8 + (kNb + 8) * 4 + kCap * 4 + kRowWords * 4;
+    static_assert(kNb >= 2 * kCap && kCap >= 3 * T, "sorted tile aliases the histogram, carries binfo");
 };
+
+// exclusive sum over the CTA with one barrier: `sc` holds NW + 1 ints and must not be written again
+// before a later barrier (callers alternate two buffers)
+template <int NW>
+__device__ __forceinline__ int cta_excl_sum(int v, int *sc, int *total) {
+    const int inc = warp_incl_sum(v);
+    const int w = warp_id();
+    if (lane_id() == 31) sc[w] = inc;
+    __syncthreads();
+    const int t = lane_id() < NW ? sc[lane_id()] : 0;
+    const int ci = warp_incl_sum(t);
+    *total = __shfl_sync(kFull, ci, NW - 1);
+    return __shfl_sync(kFull, ci - t, w) + inc - v;
+}
+
+// bucket parameters of a row: as many buckets as fit its region of the histogram (2 cap slots, cap =
+// the row's padded slots >= its products), i.e. 2^floor(log2(2 cap)), over its column span [mn, mx]
+__device__ __forceinline__ int row_shift(int cap, int mn, int mx) {
+    const uint32_t span = (uint32_t)(mx - mn);
+    const int bits = span ? 32 - __clz(span) : 0;
+    return max(0, bits - (32 - __clz(2 * cap) - 1));
+}
 
 template <int T, int EPT>
 __global__ void __launch_bounds__(T, 2) k_merge_tiles(TileArgs a) {
     using S = TileSmem<T, EPT>;
     constexpr int NW = T / 32;
     constexpr int RW = kTileMaxRows + 1;
-    static_assert(EPT % 4 == 0, "vector loads");
+    constexpr int BPT = S::kNb / T;                    // buckets per thread in the scan
+    static_assert(EPT % 4 == 0 && BPT % 4 == 0, "vector accesses");
     constexpr int E2M = (S::kCap + T - 1) / T + 1;    // max slice length of the reduction (odd stride)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     int32_t *sk = (int32_t *)smem_raw;                      // tile keys (bulk copy target, then sorted)
     float *sv = (float *)(smem_raw + S::kCap * 4);
-    int *hist = (int *)(smem_raw + S::kCap * 8);            // bucket counts / starts
-    int *binfo = hist + S::kHistWords;                      // (bucket start << 16) | keys to rank against
+    int *hist = (int *)(smem_raw + S::kCap * 8);            // bucket counts / starts [kNb + 1]
+    int *binfo = hist + S::kNb + 8;                         // (bucket start << 16) | keys to rank against
     int *ro = binfo + S::kCap;        // row slot offsets in the tile [nr + 1]
     int *rv = ro + RW;                // products per row
     int *rmn = rv + RW;               // column min / max per row
     int *rmx = rmn + RW;
-    int *rbb = rmx + RW;              // first bucket of the row [nr + 1]
-    int *rsh = rbb + RW;              // bucket shift
-    int *rss = rsh + RW;              // first sorted position of the row [nr + 1]
+    int *rss = rmx + RW;              // first sorted position of the row [nr + 1]
     int *rout = rss + RW;             // first merged position of the row
-    int32_t *ok = binfo;              // merged tile (after the ranking): keys
-    float *ov = (float *)hist;        //   values
-    double *lead = (double *)(hist + S::kCap);             // slice carries: sum before the first head
+    int *rth = rout + RW;             // first thread of the row [nr + 1] (a row owns ceil(cap / EPT))
+    int32_t *tk = (int32_t *)hist;                          // sorted tile (the ranking's output): keys
+    float *tv = (float *)(hist + S::kCap);                  //   values
+    int32_t *ok = sk;                                       // merged tile (staging of the copy-out)
+    float *ov = sv;
+    double *lead = (double *)binfo;                         // slice carries: sum before the first head
     int *hhead = (int *)(lead + T);                         //   and whether the slice has a head
     __shared__ uint64_t mbar;
     __shared__ int64_t s_t, s_P;
-    __shared__ int sc[NW + 1];
+    __shared__ int sc0[NW + 1], sc1[NW + 1];
     const int tid = threadIdx.x;
-    const Group<NW, 1> g;
-    if (tid == 0) mbar_init(&mbar, 1);
+    const bool prof_on = a.debug == 2 && tid == 0;
+    __shared__ unsigned long long ph[16];
+    long long t_last = clock64();
+    if (tid < 16) ph[tid] = 0;
+    if (tid == 0) {
+        mbar_init(&mbar, 1);
+        s_t = (int64_t)atomicAdd(a.ticket, 1ull);
+    }
     __syncthreads();
     const int64_t NT = *a.ntiles;
     uint32_t phase = 0;
     while (true) {
-        if (tid == 0) s_t = (int64_t)atomicAdd(a.ticket, 1ull);
-        __syncthreads();
-        const int64_t t = s_t;
+        const int64_t t = s_t;   // (claimed before the previous barrier)
         if (t >= NT) break;
         const TileDesc d = a.tiles[t];
         if (d.kind == TK_COPY || d.kind == TK_INPLACE) {
@@ -296,9 +336,12 @@ __global__ void __launch_bounds__(T, 2) k_merge_tiles(TileArgs a) {
             }
             __syncthreads();   // the whole chunk is in registers before its count is published
             if (warp_id() == 0) {
-                lb_publish(a.status, t, U);
-                const int64_t P = lb_resolve(a.status, t, U);
-                if (lane_id() == 0) s_P = P;
+                if (a.debug != 1) lb_publish(a.status, t, U);
+                const int64_t P = a.debug == 1 ? src : lb_resolve(a.status, t, U);
+                if (lane_id() == 0) {
+                    s_P = P;
+                    s_t = (int64_t)atomicAdd(a.ticket, 1ull);   // next tile
+                }
             }
             __syncthreads();
             const int64_t P = s_P;
@@ -311,9 +354,14 @@ __global__ void __launch_bounds__(T, 2) k_merge_tiles(TileArgs a) {
                 const int q = j * T + tid;
                 if (q < U) { a.col[P + q] = ck[j]; a.val[P + q] = cv[j]; }
             }
+            __syncthreads();   // (s_P is read before the next tile rewrites it)
+            if (prof_on) ph[12]++;
+            TILE_PH(10);
             continue;
         }
         // ---- rows [r0, r1) of Ĉ, or one column group of a long row (one row, scratch input) ------
+        // Row r owns the threads [rth[r], rth[r+1]), ceil(cap_r / EPT) of them: thread t takes the
+        // slots ro[r] + EPT (t - rth[r]) + [0, EPT) of its row only (no row tracking per slot).
         const bool grp = d.kind == TK_GROUP;
         int r0, nr, n, lo_in = 0, cnt = 0;
         int64_t S0;
@@ -337,305 +385,297 @@ __global__ void __launch_bounds__(T, 2) k_merge_tiles(TileArgs a) {
             src_col = a.scol;
             src_val = a.sval;
         }
+        {   // row table + thread allotment (one exclusive sum over the rows)
+            int nth = 0;
+            if (tid < nr) {
+                int o0, o1, lv;
+                if (!grp) {
+                    o0 = (int)(a.rowoff[r0 + tid] - S0);
+                    o1 = (int)(a.rowoff[r0 + tid + 1] - S0);
+                    lv = (int)a.rowwork[r0 + tid];
+                } else {
+                    o0 = 0;
+                    o1 = n;
+                    lv = cnt;
+                }
+                ro[tid] = o0;
+                rv[tid] = lv;
+                nth = (o1 - o0 + EPT - 1) / EPT;
+            }
+            int tot;
+            const int th = cta_excl_sum<NW>(nth, sc1, &tot);   // (also the barrier after the previous
+            if (tid < nr) rth[tid] = th;                       //  tile's copy-out of sk / sv, rout)
+            if (tid == 0) { ro[nr] = n; rth[nr] = tot; }
+        }
         if (tid == 0 && n > 0) {
-            fence_proxy_async_smem();   // previous tile's reads / writes of sk, sv come first
+            fence_proxy_async_smem();   // the generic-proxy accesses of sk, sv come first
             mbar_expect_tx(&mbar, (uint32_t)n * 8u);
             bulk_g2s(sk, src_col + S0, (uint32_t)n * 4u, &mbar);
             bulk_g2s(sv, src_val + S0, (uint32_t)n * 4u, &mbar);
         }
-        if (!grp) {
-            for (int r = tid; r < nr; r += T) {
-                ro[r] = (int)(a.rowoff[r0 + r] - S0);
-                rv[r] = (int)a.rowwork[r0 + r];
-                rmn[r] = kKeyPad;
-                rmx[r] = -1;
-                rout[r] = -1;
-            }
-        } else if (tid == 0) {
-            ro[0] = 0;
-            rv[0] = cnt;
-            rmn[0] = kKeyPad;
-            rmx[0] = -1;
-            rout[0] = -1;
-        }
-        if (tid == 0) ro[nr] = n;
-        {   // zero the histogram (it held the previous tile's merged values, read before the claim)
+        {
             int4 *h4 = reinterpret_cast<int4 *>(hist);
-            for (int q = tid; q < S::kHistWords / 4; q += T) h4[q] = make_int4(0, 0, 0, 0);
+            for (int q = tid; q < (2 * EPT * T) / 4 + 2; q += T) h4[q] = make_int4(0, 0, 0, 0);
+            for (int r = tid; r < nr; r += T) { rmn[r] = kKeyPad; rmx[r] = -1; rout[r] = -1; }
         }
-        __syncthreads();
+        __syncthreads();   // (B1) row table, rth
+        TILE_PH(0);
+        const int NTH = rth[nr];
+        // my row: last r with rth[r] <= tid (rows without slots share the next row's first thread)
+        int row = 0;
+        if (tid < NTH && nr > 1) {
+            int lo = 0, hi = nr;
+            while (hi - lo > 1) {
+                const int mid = (lo + hi) >> 1;
+                if (rth[mid] <= tid) lo = mid; else hi = mid;
+            }
+            row = lo;
+        }
+        const bool act = tid < NTH;
+        const int k_in_row = tid - rth[row];
+        const int ps = ro[row] + EPT * k_in_row;                              // my first slot
+        const int rlo = grp ? lo_in : ro[row], rhi = grp ? lo_in + cnt : ro[row + 1];   // my row's slots
+        auto load_keys = [&](int32_t (&kk)[EPT]) {
+#pragma unroll
+            for (int v = 0; v < EPT / 4; ++v) {
+                int4 c = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
+                if (act && ps + 4 * v < n) c = *reinterpret_cast<const int4 *>(sk + ps + 4 * v);
+                kk[4 * v] = c.x; kk[4 * v + 1] = c.y; kk[4 * v + 2] = c.z; kk[4 * v + 3] = c.w;
+            }
+#pragma unroll
+            for (int e = 0; e < EPT; ++e)
+                if (ps + e < rlo || ps + e >= rhi) kk[e] = kKeyPad;
+        };
         if (n > 0) {
             mbar_wait(&mbar, phase);
             phase ^= 1;
         }
-        // ---- registers: slots [p0, p0 + EPT) of the tile; the row of p0 ---------------------
-        const int p0 = tid * EPT;
-        int32_t key[EPT];
-        float val[EPT];
-#pragma unroll
-        for (int v = 0; v < EPT / 4; ++v) {
-            const int p = p0 + 4 * v;
-            int4 c = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
-            float4 f = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (p < n) {
-                c = *reinterpret_cast<const int4 *>(sk + p);
-                f = *reinterpret_cast<const float4 *>(sv + p);
-            }
-            key[4 * v] = c.x; key[4 * v + 1] = c.y; key[4 * v + 2] = c.z; key[4 * v + 3] = c.w;
-            val[4 * v] = f.x; val[4 * v + 1] = f.y; val[4 * v + 2] = f.z; val[4 * v + 3] = f.w;
-        }
-        if (grp) {   // slots of the neighbouring groups inside the aligned window are not ours
+        TILE_PH(1);
+        {   // per-row column min / max (one pair of shared atomics per thread)
+            int32_t key[EPT];
+            load_keys(key);
+            int lmn = kKeyPad, lmx = -1;
 #pragma unroll
             for (int e = 0; e < EPT; ++e)
-                if (p0 + e < lo_in || p0 + e >= lo_in + cnt) key[e] = kKeyPad;
+                if (key[e] != kKeyPad) { lmn = min(lmn, key[e]); lmx = max(lmx, key[e]); }
+            if (lmx >= 0) { atomicMin(&rmn[row], lmn); atomicMax(&rmx[row], lmx); }
         }
-        int row0 = 0;
-        if (p0 < n && nr > 1) {
-            int lo = 0, hi = nr;
-            while (hi - lo > 1) {
-                const int mid = (lo + hi) >> 1;
-                if (ro[mid] <= p0) lo = mid; else hi = mid;
-            }
-            row0 = lo;
-        }
-        {   // per-row column min / max (one pair of shared atomics per row segment of the thread)
-            int row = row0, nxt = ro[row0 + 1];
-            int cur = -1, lmn = 0, lmx = 0;
+        __syncthreads();   // (B2)
+        TILE_PH(2);
+        // ---- histogram: row r's buckets live at [2 EPT rth[r], 2 EPT rth[r+1]) -- 2^floor(log2) of
+        //      that many over its column span; the atomic's return value is the key's rank in its
+        //      bucket.  bk = bucket | rank << 13 | exact << 26 ------------------------------------------
+        int bk[EPT];
+        {
+            int32_t key[EPT];
+            load_keys(key);
+            const int base = 2 * EPT * rth[row];
+            const int mn = rmn[row];
+            const int sh = row_shift(EPT * (rth[row + 1] - rth[row]), mn, rmx[row]);
 #pragma unroll
             for (int e = 0; e < EPT; ++e) {
-                const int p = p0 + e;
-                if (key[e] != kKeyPad) {
-                    while (p >= nxt) { ++row; nxt = ro[row + 1]; }
-                    if (row != cur) {
-                        if (cur >= 0) { atomicMin(&rmn[cur], lmn); atomicMax(&rmx[cur], lmx); }
-                        cur = row;
-                        lmn = lmx = key[e];
-                    } else {
-                        lmn = min(lmn, key[e]);
-                        lmx = max(lmx, key[e]);
-                    }
-                }
-            }
-            if (cur >= 0) { atomicMin(&rmn[cur], lmn); atomicMax(&rmx[cur], lmx); }
-        }
-        __syncthreads();
-        // ---- per-row bucket parameters; row-major bucket bases -------------------------------
-        {
-            int nbr = 0;
-            if (tid < nr) {
-                const int Lv = rv[tid];
-                if (Lv > 0) {
-                    const uint32_t span = (uint32_t)(rmx[tid] - rmn[tid]);
-                    const int lognb = nextpow2_log(Lv);
-                    const int bits = span ? 32 - __clz(span) : 0;
-                    const int sh = max(0, bits - lognb);
-                    rsh[tid] = sh;
-                    nbr = (int)(span >> sh) + 1;
-                }
-            }
-            int NB;
-            const int bb = g.excl_sum1(nbr, sc, &NB);
-            if (tid < nr) rbb[tid] = bb;
-            if (tid == 0) rbb[nr] = NB;
-        }
-        __syncthreads();
-        // ---- histogram: the returned count is the key's rank inside its bucket ---------------
-        int bk[EPT], rk[EPT];   // bucket (bit 30: exact bucket, all keys equal; -1: no key), rank
-        {
-            int row = row0, nxt = ro[row0 + 1];
-            int base = rbb[row], mn = rmn[row], sh = rsh[row];
-#pragma unroll
-            for (int e = 0; e < EPT; ++e) {
-                const int p = p0 + e;
                 bk[e] = -1;
-                rk[e] = 0;
                 if (key[e] != kKeyPad) {
-                    if (p >= nxt) {
-                        do { ++row; nxt = ro[row + 1]; } while (p >= nxt);
-                        base = rbb[row];
-                        mn = rmn[row];
-                        sh = rsh[row];
-                    }
                     const int b = base + ((key[e] - mn) >> sh);
-                    rk[e] = atomicAdd(&hist[hidx(b)], 1);
-                    bk[e] = b | (sh == 0 ? (1 << 30) : 0);
+                    const int rk = atomicAdd(&hist[b], 1);
+                    bk[e] = b | (rk << 13) | ((sh == 0) << 26);
                 }
             }
         }
-        __syncthreads();
-        // ---- bucket starts: exclusive scan (each thread a contiguous range of buckets) -------
+        __syncthreads();   // (B3)
+        TILE_PH(3);
+        // ---- bucket starts: exclusive scan, BPT contiguous buckets per thread ---------------------
         int V;
         {
-            const int NB = rbb[nr];
-            const int bpt = (NB + T - 1) / T;
-            const int b0 = min(NB, tid * bpt), b1 = min(NB, b0 + bpt);
-            int cnt = 0;
-            for (int b = b0; b < b1; ++b) cnt += hist[hidx(b)];
-            int ex = g.excl_sum1(cnt, sc, &V);
-            __syncthreads();   // (excl_sum1: the warp totals are read before the next write of sc)
-            for (int b = b0; b < b1; ++b) {
-                const int c = hist[hidx(b)];
-                hist[hidx(b)] = ex;
-                ex += c;
-            }
-            if (tid == 0) hist[hidx(NB)] = V;
-        }
-        __syncthreads();
-        if (tid < nr) rss[tid] = hist[hidx(rbb[tid])];
-        if (tid == 0) rss[nr] = V;   // (nr may equal T)
-        // ---- scatter by (bucket start + rank); binfo marks the slots that still have to rank -------
+            const int b0 = tid * BPT;
+            int cs = 0;
+            if (b0 < 2 * EPT * NTH) {
 #pragma unroll
-        for (int e = 0; e < EPT; ++e) {
-            if (bk[e] >= 0) {
-                const int b = bk[e] & ((1 << 30) - 1);
-                const int bs = hist[hidx(b)];
-                const int pos = bs + rk[e];
-                sk[pos] = key[e];
-                sv[pos] = val[e];
-                const int c = (bk[e] >> 30) ? 1 : hist[hidx(b + 1)] - bs;   // exact bucket: in place
-                binfo[pos] = (bs << 16) | c;
+                for (int v = 0; v < BPT / 4; ++v) {
+                    const int4 c = *reinterpret_cast<const int4 *>(hist + b0 + 4 * v);
+                    cs += c.x + c.y + c.z + c.w;
+                }
+            }
+            int ex = cta_excl_sum<NW>(cs, sc0, &V);   // (B4)
+            if (b0 < 2 * EPT * NTH) {
+#pragma unroll
+                for (int v = 0; v < BPT / 4; ++v) {
+                    int4 c = *reinterpret_cast<const int4 *>(hist + b0 + 4 * v);
+                    const int x = c.x, y = c.y, z = c.z, w = c.w;
+                    c = make_int4(ex, ex + x, ex + x + y, ex + x + y + z);
+                    ex += x + y + z + w;
+                    *reinterpret_cast<int4 *>(hist + b0 + 4 * v) = c;
+                }
+            }
+            if (tid == 0) hist[2 * EPT * NTH] = V;
+        }
+        __syncthreads();   // (B5)
+        TILE_PH(4);
+        if (tid < nr) rss[tid] = hist[2 * EPT * rth[tid]];
+        if (tid == 0) rss[nr] = V;
+        // ---- scatter by (bucket start + rank); binfo marks the slots that still have to rank -------
+        {
+            int32_t key[EPT];
+            float val[EPT];
+            load_keys(key);
+#pragma unroll
+            for (int v = 0; v < EPT / 4; ++v) {
+                float4 f = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (act && ps + 4 * v < n) f = *reinterpret_cast<const float4 *>(sv + ps + 4 * v);
+                val[4 * v] = f.x; val[4 * v + 1] = f.y; val[4 * v + 2] = f.z; val[4 * v + 3] = f.w;
+            }
+            __syncthreads();   // (B6: every slot read before the scatter overwrites the tile)
+#pragma unroll
+            for (int e = 0; e < EPT; ++e) {
+                if (bk[e] >= 0) {
+                    const int b = bk[e] & 0x1fff;
+                    const int bs = hist[b];
+                    const int pos = bs + ((bk[e] >> 13) & 0x1fff);
+                    sk[pos] = key[e];
+                    sv[pos] = val[e];
+                    const int c = (bk[e] >> 26) ? 1 : hist[b + 1] - bs;   // exact bucket: in place
+                    binfo[pos] = (bs << 16) | c;
+                }
             }
         }
-        __syncthreads();
-        // ---- rank inside the multi-key buckets, by slot: a warp covers 32 consecutive slots, so
-        //      the lanes of one bucket loop together (broadcast reads of the bucket's keys) ----------
-        int np[EPT];
-        int32_t mk[EPT];
-        float mv[EPT];
+        __syncthreads();   // (B7)
+        TILE_PH(5);
+        // ---- rank inside the multi-key buckets, by slot (a warp covers 32 consecutive slots, so the
+        //      lanes of one bucket loop together); every key is copied to its sorted slot in tk / tv --
 #pragma unroll
         for (int j = 0; j < EPT; ++j) {
             const int p = j * T + tid;
-            np[j] = -1;
             if (p < V) {
                 const int info = binfo[p];
                 const int c = info & 0xffff;
+                const int32_t kk = sk[p];
+                int dst = p;
                 if (c > 1) {
                     const int bs = info >> 16;
-                    const int32_t kk = sk[p];
                     int rank = 0;
-                    for (int q = bs; q < bs + c; ++q) {
-                        const int32_t kq = sk[q];
-                        rank += (kq < kk) | ((kq == kk) & (q < p));
+                    if (c <= 4) {   // the common case: straight-line comparisons, no divergent loop
+#pragma unroll
+                        for (int i = 0; i < 4; ++i) {
+                            const int q = bs + i;
+                            const int32_t kq = sk[min(q, bs + c - 1)];
+                            rank += (i < c) & ((kq < kk) | ((kq == kk) & (q < p)));
+                        }
+                    } else {
+                        for (int q = bs; q < bs + c; ++q) {
+                            const int32_t kq = sk[q];
+                            rank += (kq < kk) | ((kq == kk) & (q < p));
+                        }
                     }
-                    np[j] = bs + rank;
-                    mk[j] = kk;
-                    mv[j] = sv[p];
+                    dst = bs + rank;
                 }
+                tk[dst] = kk;
+                tv[dst] = sv[p];
             }
         }
-        __syncthreads();
-#pragma unroll
-        for (int j = 0; j < EPT; ++j)
-            if (np[j] >= 0) { sk[np[j]] = mk[j]; sv[np[j]] = mv[j]; }
-        __syncthreads();
-        // ---- fp64 segmented reduction over contiguous slices (odd stride: no bank conflicts).
-        //      A segment ends at a key change or a row start; a slice sums the segments that start
-        //      in it, and its leading positions (the tail of the previous slice's last segment) go
-        //      to lead[] for that slice to add ----------------------------------------------------------
+        __syncthreads();   // (B8)
+        TILE_PH(6);
+        // ---- fp64 segmented reduction: my row's sorted positions rss[r] + 9 k + [0, 9) (odd stride:
+        //      no bank conflicts; 9 (rth[r+1] - rth[r]) >= the row's products).  A segment ends at a
+        //      key change; a slice sums the segments that start in it, its leading positions (the
+        //      tail of the previous slice's last segment) go to lead[] for that slice ---------------------
         int U;
         {
-            const int E2 = ((V + T - 1) / T) | 1;
-            const int q0 = min(V, tid * E2), q1 = min(V, q0 + E2);
-            int row = 0;
-            if (q0 < q1 && nr > 1) {
-                int lo = 0, hi = nr;   // last row with rss <= q0 (empty rows share the next row's start)
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (rss[mid] <= q0) lo = mid; else hi = mid;
-                }
-                row = lo;
-            }
-            int32_t kr[E2M];
-            float vr[E2M];
-            unsigned hb = 0, rsb = 0;   // head bits and row-start bits of the slice
+            constexpr int E2 = EPT + 1;
+            const int rs = rss[row], re = rss[row + 1];
+            const int q0 = act ? min(re, rs + E2 * k_in_row) : 0, q1 = act ? min(re, q0 + E2) : 0;
+            int32_t kr[E2];
+            float vr[E2];
+            unsigned hb = 0;
             {
-                int st = rss[row], nx = rss[row + 1], rw = row;
-                int32_t prev = q0 > 0 ? sk[q0 - 1] : -1;
+                int32_t prev = q0 > rs ? tk[q0 - 1] : -1;   // (-1: no column; the row start is a head)
 #pragma unroll
-                for (int j = 0; j < E2M; ++j) {
+                for (int j = 0; j < E2; ++j) {
                     const int q = q0 + j;
-                    kr[j] = kKeyPad;
+                    kr[j] = 0;
                     vr[j] = 0.f;
                     if (q < q1) {
-                        kr[j] = sk[q];
-                        vr[j] = sv[q];
-                        while (q >= nx) { ++rw; st = nx; nx = rss[rw + 1]; }
-                        const bool rs = q == st;
-                        hb |= (unsigned)(rs | (kr[j] != prev)) << j;
-                        rsb |= (unsigned)rs << j;
+                        kr[j] = tk[q];
+                        vr[j] = tv[q];
+                        hb |= (unsigned)(kr[j] != prev) << j;
                         prev = kr[j];
                     }
                 }
             }
             const int nh = __popc(hb);
-            int o = g.excl_sum1(nh, sc, &U);
-            if (warp_id() == 0) lb_publish(a.status, t, U);
-            // slice partial sums: lead = positions before the first head; one sum per head
-            double accs = 0.0;
-            int last = -1;
-            {
-                double lsum = 0.0;
+            double accs = 0.0, lsum = 0.0;
+            int32_t lastk = 0;
 #pragma unroll
-                for (int j = 0; j < E2M; ++j) {
+            for (int j = 0; j < E2; ++j) {
+                if (q0 + j < q1) {
+                    if ((hb >> j) & 1u) {
+                        lastk = kr[j];
+                        accs = (double)vr[j];
+                    } else if (hb & ((1u << j) - 1u)) {
+                        accs += (double)vr[j];
+                    } else {
+                        lsum += (double)vr[j];
+                    }
+                }
+            }
+            lead[tid] = lsum;
+            hhead[tid] = hb != 0 || q0 >= q1;
+            int o = cta_excl_sum<NW>(nh, sc1, &U);   // (B9)
+            if (warp_id() == 0 && a.debug != 1) lb_publish(a.status, t, U);
+            if (act && k_in_row == 0 && re > rs) rout[row] = o;
+            if (nh) {
+                // completed segments (all heads but the last), then the last one with its carries
+                int oo = o;
+                double acc = 0.0;
+                int32_t hk = 0;
+                bool have = false;
+#pragma unroll
+                for (int j = 0; j < E2; ++j) {
                     if (q0 + j < q1) {
                         if ((hb >> j) & 1u) {
-                            if (last >= 0) {   // close the previous segment of the slice
-                                ok[o] = kr[last];
-                                ov[o] = (float)accs;
-                                ++o;
-                            }
-                            last = j;
-                            accs = (double)vr[j];
-                        } else if (last >= 0) {
-                            accs += (double)vr[j];
-                        } else {
-                            lsum += (double)vr[j];
+                            if (have) { ok[oo] = hk; ov[oo] = (float)acc; ++oo; }
+                            have = true;
+                            hk = kr[j];
+                            acc = (double)vr[j];
+                        } else if (have) {
+                            acc += (double)vr[j];
                         }
                     }
                 }
-                lead[tid] = lsum;
-                hhead[tid] = hb != 0 || q0 >= q1;
-            }
-            __syncthreads();
-            if (last >= 0) {   // the slice's last segment may continue through the next slices
-                for (int u = tid + 1; u < T; ++u) {
-                    accs += lead[u];
+                for (int u = tid + 1; u < NTH; ++u) {   // the last segment continues through slices
+                    accs += lead[u];                     // without a head (their lead is all theirs)
                     if (hhead[u]) break;
                 }
-                ok[o] = kr[last];
-                ov[o] = (float)accs;
-            }
-            // merged index of every row start (the row's first head)
-            if (rsb) {
-                const int o0 = o - (last >= 0 ? nh - 1 : 0);   // merged index of the slice's first head
-                int rw = row;
-                for (unsigned m = rsb; m; m &= m - 1) {
-                    const int j = __ffs(m) - 1;
-                    while (rss[rw + 1] <= q0 + j) ++rw;   // the (non-empty) row starting at q0 + j
-                    rout[rw] = o0 + __popc(hb & ((1u << j) - 1u));
-                }
+                ok[oo] = lastk;
+                ov[oo] = (float)accs;
             }
         }
-        __syncthreads();
+        TILE_PH(7);
         if (warp_id() == 0) {
-            const int64_t P = lb_resolve(a.status, t, U);
-            if (lane_id() == 0) s_P = P;
+            const int64_t P = a.debug == 1 ? S0 : lb_resolve(a.status, t, U);
+            if (lane_id() == 0) {
+                s_P = P;
+                s_t = (int64_t)atomicAdd(a.ticket, 1ull);   // next tile
+            }
         }
+        __syncthreads();   // (B10)
+        TILE_PH(8);
         // rows without products: the merged position of the next row with products (or U)
-        if (tid < nr && rout[tid] < 0) {
-            int q = tid + 1;
-            while (q < nr && rout[q] < 0) ++q;
-            rout[tid] = q < nr ? rout[q] : U;
-        }
-        __syncthreads();
         const int64_t P = s_P;
-        if (tid < nr && r0 >= 0) a.crowptr[r0 + tid] = P + rout[tid];
+        if (tid < nr && r0 >= 0) {
+            int q = tid, ro_ = rout[tid];
+            while (ro_ < 0 && ++q < nr) ro_ = rout[q];
+            a.crowptr[r0 + tid] = P + (ro_ < 0 ? U : ro_);
+        }
         if (tid == 0 && t == NT - 1) a.crowptr[a.M] = P + U;
         for (int q = tid; q < U; q += T) {
             a.col[P + q] = ok[q];
             a.val[P + q] = ov[q];
         }
+        if (prof_on) ph[11]++;
+        TILE_PH(9);
     }
+    if (prof_on)
+        for (int k = 0; k < 16; ++k) atomicAdd(a.prof + k, ph[k]);
 }
 
 }  // namespace spg

@@ -200,6 +200,7 @@ struct spgemm_plan_s {
     int64_t *tile_cnt = nullptr, *tile_base = nullptr;
     unsigned long long *tile_status = nullptr;
     int64_t tiles_max = 0;
+    unsigned long long *lbi = nullptr;   // options.reserved[8] = 1: [expansion | limited merge] x kLbiSlots
     int64_t nnz_c = -1;
     int state = 0;  // 1 planned, 2 expanded, 3 merged
 };
@@ -257,10 +258,10 @@ static inline unsigned grid_for(int64_t n, int threads, int64_t cap = 148 * 64) 
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>(cdiv(n, threads), cap));
 }
 
-// merge selection: the tile merge (merge_tiles.cuh, default) places C at the head of the Ĉ arrays;
-// options.reserved[5] = 1 or a legacy bin variant in reserved[0] selects the per-bin merge +
-// compaction (merge.cuh), reserved[0] = 4 the fused unit merge (merge_units.cuh)
-static inline bool use_tile_merge(const spgemm_options_t &o) { return o.reserved[0] == 0 && o.reserved[5] == 0; }
+// merge selection: default = per-bin merge + CSR compaction (merge.cuh); options.reserved[5] = 2 the
+// tile merge (merge_tiles.cuh + merge_long.cuh: C placed by look-back at the head of the Ĉ arrays, no
+// compaction); reserved[0] = 4 the fused unit merge (merge_units.cuh)
+static inline bool use_tile_merge(const spgemm_options_t &o) { return o.reserved[0] == 0 && o.reserved[5] == 2; }
 static inline bool c_in_place(const spgemm_options_t &o) { return use_tile_merge(o) || o.reserved[0] == kMergeFused; }
 
 // Large-smem kernels: opt-in shared memory size and resident blocks per SM, queried once per
@@ -604,7 +605,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     TRY(palloc(p, &p->piece_off, K + 1, s));
     int64_t *d_starts;
     TRY(palloc(p, &d_starts, kNumPairBuckets + kNumRowBuckets + 4, s));
-    SplitParams sp{o.piece_work, o.split_b_tile, o.split_ca_max};
+    SplitParams sp{o.piece_work, o.split_b_tile, o.split_ca_max, o.reserved[7]};
     {
         Temp tb(s), tr(s), tn(s);
         uint8_t *pb, *rbk;
@@ -769,6 +770,12 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     TRY(palloc(p, &p->fb_rows, M, s));
     TRY(palloc(p, &p->fb_count, 1, s));
     TRY(palloc(p, &p->crowptr, M + 1, s));
+    if (p->opt.reserved[8] == 1) {   // LBI recording (Eq. (3))
+        TRY(palloc(p, &p->lbi, 2 * kLbiSlots, s));
+        CK(cudaMemsetAsync(p->lbi, 0, 2 * kLbiSlots * 8, s));
+        CK(cudaMemsetAsync(p->lbi, 0xff, 8, s));
+        CK(cudaMemsetAsync(p->lbi + kLbiSlots, 0xff, 8, s));
+    }
     p->state = 1;
     return SPGEMM_OK;
 }
@@ -805,7 +812,7 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
         // expansion 1.34 -> 2.10 ms and the compaction 1.14 -> 1.48 ms on C2; not used)
         LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
             p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
-            p->base, p->chat_col, p->chat_val));
+            p->base, p->chat_col, p->chat_val, p->lbi));
     }
     p->state = 2;
     return SPGEMM_OK;
@@ -947,6 +954,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
         if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
         g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
+        g.lbi = p->lbi ? p->lbi + kLbiSlots : nullptr;
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
@@ -986,6 +994,7 @@ static int merge_limited_in_place(spgemm_plan_s *p, cudaStream_t s) {
     g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
     if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
     g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
+    g.lbi = p->lbi ? p->lbi + kLbiSlots : nullptr;
     // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
     // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
     TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
@@ -1077,6 +1086,9 @@ static int merge_tiles_path(spgemm_plan_s *p, cudaStream_t s) {
     ta.lt = lt;
     ta.scol = p->lg_scol;
     ta.sval = p->lg_sval;
+    ta.debug = p->opt.reserved[1];
+    ta.prof = p->unit_ticket + 2;
+    if (ta.debug == 2) CK(cudaMemsetAsync(ta.prof, 0, 16 * 8, s));
     using TS = TileSmem<kTileThreads, kTileEPT>;
     auto kern = k_merge_tiles<kTileThreads, kTileEPT>;
     int occ = 0;
@@ -1133,6 +1145,7 @@ static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
         g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
         if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
         g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
+        g.lbi = p->lbi ? p->lbi + kLbiSlots : nullptr;
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false, true));
@@ -1357,6 +1370,8 @@ int spgemm_inspect(spgemm_plan_t p, int32_t what, void *dst, int64_t cap, int64_
         case SPGEMM_VIEW_CROWPTR:
             if (p->state < 3) return fail(SPGEMM_ERR_STATE, "C row pointers exist after merge");
             src = p->crowptr; bytes = (p->m + 1) * 8; break;
+        case SPGEMM_VIEW_LBI:
+            src = p->lbi; bytes = p->lbi ? 2 * kLbiSlots * 8 : 0; break;
         case SPGEMM_VIEW_UNIT_PROFILE:
             if (p->state < 3) return fail(SPGEMM_ERR_STATE, "the unit profile exists after merge");
             src = p->unit_ticket + 2; bytes = 16 * 8; break;

@@ -14,7 +14,7 @@ from parity_util import cached_inputs, whole_matrix_check
 
 pytestmark = pytest.mark.gpu
 
-LEGACY = dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)   # per-bin merge + compaction (merge.cuh)
+TILES = dict(reserved=(0, 0, 0, 0, 0, 2) + (0,) * 10)   # tile merge: look-back placement, no compaction
 
 
 def _fresh():
@@ -23,7 +23,7 @@ def _fresh():
     spg.trim_pool()
 
 
-@pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", LEGACY), ("C4", {}), ("C3", {}), ("C5", {}),
+@pytest.mark.parametrize("name,opts", [("C2", {}), ("C2", TILES), ("C4", {}), ("C3", {}), ("C3", TILES), ("C5", {}),
                                        ("C5", {"chunks": 4}), ("AB17", {}), ("AB18", {})])
 def test_whole_matrix(name, opts):
     inp = cached_inputs(name)

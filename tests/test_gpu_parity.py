@@ -67,6 +67,8 @@ def _deg(inp):
 
 
 FUSED = dict(reserved=(4,) + (0,) * 15)   # merge variant: fused unit merge + look-back output
+TILES = dict(reserved=(0, 0, 0, 0, 0, 2) + (0,) * 10)   # tile merge (merge_tiles.cuh, merge_long.cuh)
+TILES_INPLACE = dict(reserved=(0, 0, 0, 0, 0, 2, 1) + (0,) * 9)   # tile merge, legacy long rows
 
 CASES = [
     ("C1", dict()),
@@ -86,6 +88,11 @@ CASES = [
     ("C1", dict(alpha=2.0)),
     ("C1", dict(beta=10.0)),
     ("C1", dict(beta=10.0, enable_limit=0)),
+    ("C1", dict(reserved=(0,) * 7 + (4,) + (0,) * 8)),   # fixed splitting factor 4 (Fig. 11 sweep)
+    ("C1", dict(reserved=(0,) * 7 + (64,) + (0,) * 8)),
+    ("C1", TILES),
+    ("C1", dict(beta=10.0, **TILES)),                # the paper's β: many long rows -> column groups
+    ("C1", dict(beta=10.0, **TILES_INPLACE)),        # ... or merged in place and moved
 ]
 
 
@@ -145,7 +152,7 @@ def test_stage2_reorganizer(name, opts):
     cls = stages.classify_pairs(ca, rb, work, t_dom, o.split_ca_max)
     np.testing.assert_array_equal(p.inspect(spg.VIEW_PAIR_CLASS, np.int8), cls)
     if o.enable_split:
-        want = stages.split_pieces(inp, cls, o.piece_work, o.split_b_tile, o.split_ca_max)
+        want = stages.split_pieces(inp, cls, o.piece_work, o.split_b_tile, o.split_ca_max, fixed_f=o.reserved[7])
         got = p.inspect(spg.VIEW_PIECES, np.int64).reshape(-1, 5)
         np.testing.assert_array_equal(got, want)
         assert st["n_pieces_split"] == len(want)
@@ -247,7 +254,7 @@ def test_random_tiny(shape, dens, seed, skew, values):
     A, B = spg.from_inputs(inp, "cuda")
     for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(1,) + (0,) * 15),
                  dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15), FUSED, dict(reserved=(6,) + (0,) * 15),
-                 dict(reserved=(10,) + (0,) * 15),
+                 dict(reserved=(10,) + (0,) * 15), TILES, dict(beta=1000.0, **TILES),
                  dict(beta=1000.0, piece_work=64, split_ca_max=3, **FUSED)):
         C = spg.matmul(A, B, **opts)
         assert_c_matches(C, inp, signed=(values == "signed"))
@@ -285,19 +292,20 @@ def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False,
     (16, 100, 30000, 0.3, 2000, False, False),     # dense rows: fp64 column windows
     (2, 10000, 1000000, 1.0, 21, True, False),     # column 0 in 10000 runs: single-column overflow
 ])
-@pytest.mark.parametrize("fused", [False, True])
+@pytest.mark.parametrize("fused", [False, True, "tiles", "tiles_inplace"])
 def test_limited_paths(m, k, n, dens, run_len, hub, narrow, fused):
     """B-Limited merge: rows longer than the non-limited capacity, through every sub-path."""
     inp = _wide_inputs(m, k, n, dens, run_len, 3, hub_col=hub, narrow=narrow)
     A, B = spg.from_inputs(inp, "cuda")
-    with spg.Plan(A, B, **(FUSED if fused else {})) as p:
+    opts = {False: {}, True: FUSED, "tiles": TILES, "tiles_inplace": TILES_INPLACE}[fused]
+    with spg.Plan(A, B, **opts) as p:
         st = p.stats()
         assert st["n_rows_bin"][5] > 0
         p.expand()
         p.merge()
         C = p.output()
     assert_c_matches(C, inp)
-    with spg.Plan(A, B, **(FUSED if fused else {})) as p:   # staged path with host output
+    with spg.Plan(A, B, **opts) as p:   # staged path with host output
         p.expand()
         p.merge()
         C = p.output(device="cpu")
@@ -449,14 +457,14 @@ def test_computed_zeros_hand():
     inp = synth.from_coo("cancel", 2, 2, 64, (np.array([0, 0, 1]), np.array([0, 1, 1]),
                                               np.array([1.0, -1.0, 2.0], dtype=np.float32)), (br, bc, bv))
     A, B = spg.from_inputs(inp, "cuda")
-    for opts in ({}, dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)):
+    for opts in ({}, TILES):
         C = spg.matmul(A, B, **opts)
         val = _assert_exact(C, inp)
         assert C.rowptr.cpu().tolist() == [0, 4, 8]
         assert np.all(val[:4] == 0) and np.all(C.val[:4].cpu().numpy() == 0)
 
 
-@pytest.mark.parametrize("opts", [{}, dict(beta=10.0), dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)])
+@pytest.mark.parametrize("opts", [{}, dict(beta=10.0), TILES])
 def test_computed_zeros_pm1(opts):
     """+-1 values (synth kind 'pm1'): thousands of entries cancel exactly; the structure keeps them and
     the values are exact (short rows, the paper's β-Limiting rows, and the legacy bins)."""
@@ -491,8 +499,24 @@ def test_limited_bucket_overflow_many_heavy_buckets():
     inp = synth.from_coo("heavy", 1, k, 130_000, (ar, ac, synth.edge_values(ar, ac, 1)),
                          (br, bc, synth.edge_values(br, bc, 2)))
     A, B = spg.from_inputs(inp, "cuda")
-    for opts in ({}, dict(reserved=(0, 0, 0, 0, 0, 1) + (0,) * 10)):
+    for opts in ({}, TILES):
         with spg.Plan(A, B, **opts) as p:
             assert p.stats()["n_rows_bin"][5] == 1   # the row is B-Limited (9108 padded slots)
             C = p.execute()
         assert_c_matches(C, inp)
+
+
+# ------------------------------------------------------------------ LBI (Eq. 3) ---------------
+def test_lbi_recording():
+    """PAPER.md Eq. (3): LBI = mean_i T_i / max_i T_i over the SMs, from per-SM busy times the
+    kernels record with options.reserved[8] = 1 (0 < LBI <= 1); recording does not change C."""
+    inp = _wide_inputs(40, 120, 70000, 0.25, 300, 3, narrow=True)
+    A, B = spg.from_inputs(inp, "cuda")
+    opts = dict(reserved=(0,) * 8 + (1,) + (0,) * 7)
+    with spg.Plan(A, B, **opts) as p:
+        C = p.execute()
+        lb = p.lbi()
+    assert_c_matches(C, inp)
+    for name in ("expand", "merge_limited"):
+        assert lb[name] is not None, name
+        assert 0.0 < lb[name]["lbi"] <= 1.0 and lb[name]["max_ms"] > 0

@@ -323,3 +323,17 @@ def test_gather_order_hand_list():
     lists = stages.gather_lists(ca, rb, cls)
     for b in range(6):
         np.testing.assert_array_equal(lists[b], kv[f"bin{b}"])
+
+
+@pytest.mark.parametrize("fixed_f,chunks", [(1, [5]), (2, [3, 2]), (4, [2, 2, 1]), (64, [1, 1, 1, 1, 1])])
+def test_fixed_splitting_factor_fig5_block(fixed_f, chunks):
+    """Fig. 11's sweep imposes the splitting factor 2^n (L640-L687 L): the Fig. 5 block (5 column
+    entries x 5 row entries, L386-L388 L) split by f gives greedy chunks of ceil(5/f) entries; f is
+    capped at the column's next power of two (8 -> one entry per piece)."""
+    inp = synth.from_coo("fig5", 5, 1, 5, (np.arange(5), np.zeros(5, int), np.ones(5, np.float32)),
+                         (np.zeros(5, int), np.arange(5), np.ones(5, np.float32)))
+    ca, rb, work = stages.pair_workload(inp)
+    cls = np.array([stages.DOMINATOR], dtype=np.int8)
+    pcs = stages.split_pieces(inp, cls, piece_work=10 ** 9, b_tile=4096, split_ca_max=10 ** 9, fixed_f=fixed_f)
+    assert [int(p[2] - p[1]) for p in pcs] == chunks
+    assert int(sum((p[2] - p[1]) * (p[4] - p[3]) for p in pcs)) == 25
