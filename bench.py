@@ -444,6 +444,11 @@ def main():
         del C, Cc, G
     # e2e through the C-ABI with host buffers (H2D of A, B and D2H of C inside the timed region)
     if not args.no_e2e:
+        # (the device-output steps' C arrays and plan workspaces stay cached by torch / the plan pool:
+        # a host-output product of C5 needs Ĉ plus a device staging copy of C, so release them first)
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+        spg.trim_pool()
         Ah, Bh = spg.from_inputs(inp, "cpu")
         h2d = sum(t.numel() * t.element_size() for t in (Ah.colptr, Ah.rowidx, Ah.val, Bh.rowptr, Bh.colidx, Bh.val))
         es = []

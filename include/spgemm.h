@@ -121,13 +121,9 @@ typedef struct {
                                  read from the first / last entry of b_k*) -- unsorted rows are
                                  then undefined behaviour, not an error                          */
     int32_t reserved[16];     /* tuning / comparison knobs, 0 = default:
-                                 [0] merge variant: 1 register-staged counting sort, 2 bucket sort
-                                     everywhere, 3 merge path everywhere, 4 fused unit merge (C
-                                     placed by decoupled look-back, see spgemm_execute), 6 register
-                                     bitonic <= 256 slots, 7 no software pipelining, 8 pipelined
-                                     2K / 4K bins too, 10 bucket-owner insertion sort;
-                                 [1] profiling: 1 unit merge without look-back (wrong C, timing
-                                     only), 2 unit-merge phase clocks, 3 B-Limited path clocks
+                                 [0] unused (round-1 merge variants, removed in round 2);
+                                 [1] profiling: 1 tile merge without look-back (wrong C, timing
+                                     only), 2 tile-merge phase clocks, 3 B-Limited path clocks
                                      (SPGEMM_VIEW_UNIT_PROFILE);
                                  [2] 1 = per-row compaction kernels instead of the chunked one;
                                  [3] 1 = row-product expansion (the paper's comparison order);
@@ -155,8 +151,8 @@ typedef struct {
     int64_t n_gather_bin[6];   /* low performers per gathering bin n (2^(n-1) < t <= 2^n)      */
     int64_t n_rows_bin[6];     /* empty, single-run, <=32 slots, <=1024 slots, <=4096 slots, limited */
     int64_t bytes_workspace;   /* device bytes held by the plan                                */
-    int64_t n_units;           /* merge units (short-row groups + long rows), after spgemm_merge */
-    int64_t n_units_fallback;  /* units merged by the natural-merge-sort fallback               */
+    int64_t n_units;           /* tile merge: tiles walked (after spgemm_merge), else -1          */
+    int64_t n_units_fallback;  /* tile merge: 0 (no fallback path), else -1                    */
 } spgemm_stats_t;
 
 /* spgemm_inspect selectors: copy a plan array to host memory (tests, tooling). */
@@ -172,7 +168,7 @@ typedef enum {
     SPGEMM_VIEW_CHAT_COL = 7,    /* int32[nnz_chat] after spgemm_expand (before merge)       */
     SPGEMM_VIEW_CHAT_VAL = 8,    /* fp32[nnz_chat]                                            */
     SPGEMM_VIEW_CROWPTR = 9,     /* int64[m+1] C row pointers after spgemm_merge             */
-    SPGEMM_VIEW_UNIT_PROFILE = 10,/* uint64[16] merge-unit phase clocks (options.reserved[1]=2) */
+    SPGEMM_VIEW_UNIT_PROFILE = 10,/* uint64[16] merge phase clocks (options.reserved[1] = 2 / 3)  */
     SPGEMM_VIEW_ROW_COLMIN = 11, /* int32[m]   first column of row i of C (the merge's bucket
                                     range; computed in spgemm_plan for rows whose padded Ĉ
                                     bucket exceeds 256 slots; other rows 0x7f7f7f7f = unknown;
@@ -200,6 +196,15 @@ void spgemm_default_options(spgemm_options_t *opt);
 int spgemm_plan(const spgemm_csc_t *A, const spgemm_csr_t *B, const spgemm_options_t *opt,
                 void *stream, spgemm_plan_t *plan);
 
+/* Rows [row_begin, row_end) of C = A x B, planned without a copy of A by the caller: the window's
+ * entries of every column of A (one contiguous range, rows being ascending) are packed on the
+ * device into the plan's own A' (row indices minus row_begin), so the plan computes the
+ * (row_end - row_begin) x n row block of C (the chunked expansion and the multi-GPU row blocks of
+ * DESIGN.md R8).  Synchronises `stream` once more than spgemm_plan (the window's nnz).
+ * spgemm_plan(A, B, ...) = spgemm_plan_rows(A, B, 0, A->nrows, ...). */
+int spgemm_plan_rows(const spgemm_csc_t *A, const spgemm_csr_t *B, int64_t row_begin, int64_t row_end,
+                     const spgemm_options_t *opt, void *stream, spgemm_plan_t *plan);
+
 /* Stage (3): writes Ĉ.  Asynchronous. */
 int spgemm_expand(spgemm_plan_t plan, void *stream);
 
@@ -214,8 +219,7 @@ int spgemm_output(spgemm_plan_t plan, spgemm_csr_out_t *C, void *stream);
 
 /* expand + merge + alloc(C arrays in `out_where`) + output.  C->rowptr/colidx/val are
  * set to the allocated buffers (owned by the caller).  Returns after `stream` holds C.
- * With a device C and the tile merge (options.reserved[5] = 2) or the fused unit merge
- * (options.reserved[0] = 4),
+ * With a device C and the tile merge (options.reserved[5] = 2),
  * colidx / val are requested BEFORE the expansion with capacity nnz(Ĉ) (padded slots) >= nnz(C):
  * they hold Ĉ during the merge and C in their first C->nnz entries afterwards (one buffer for
  * both: no second nnz(Ĉ)-sized allocation, no copy). */

@@ -28,7 +28,7 @@ VIEW_WORK, VIEW_ROWWORK, VIEW_ROWOFF, VIEW_PAIR_CLASS, VIEW_PIECES, VIEW_GATHER,
 EXPORTED = ["spgemm_abi_version", "spgemm_last_error", "spgemm_default_options", "spgemm_plan",
             "spgemm_expand", "spgemm_merge", "spgemm_output", "spgemm_execute", "spgemm_get_stats",
             "spgemm_inspect", "spgemm_destroy", "spgemm_set_timing", "spgemm_last_timings",
-            "spgemm_row_partition", "spgemm_trim_pool"]
+            "spgemm_row_partition", "spgemm_trim_pool", "spgemm_plan_rows"]
 
 
 class SpgemmError(RuntimeError):
@@ -87,6 +87,8 @@ def lib():
         L.spgemm_default_options.argtypes = [ctypes.POINTER(Options)]
         L.spgemm_plan.argtypes = [ctypes.POINTER(_CSC), ctypes.POINTER(_CSR), ctypes.POINTER(Options), vp,
                                   ctypes.POINTER(vp)]
+        L.spgemm_plan_rows.argtypes = [ctypes.POINTER(_CSC), ctypes.POINTER(_CSR), i64, i64, ctypes.POINTER(Options),
+                                       vp, ctypes.POINTER(vp)]
         L.spgemm_expand.argtypes = [vp, vp]
         L.spgemm_merge.argtypes = [vp, vp, ctypes.POINTER(i64)]
         L.spgemm_output.argtypes = [vp, ctypes.POINTER(_CSR), vp]
@@ -169,15 +171,18 @@ def _stream(stream) -> ctypes.c_void_p:
 class Plan:
     """One C = A x B problem: spgemm_plan (stages 1-2) on construction."""
 
-    def __init__(self, A: CSC, B: CSR, stream=None, **opts):
+    def __init__(self, A: CSC, B: CSR, stream=None, rows=None, **opts):
+        """rows=(r0, r1): plan rows [r0, r1) of C only (spgemm_plan_rows; A is windowed on the GPU)."""
         self._keep = (A, B)
         self.stream = _stream(stream)
-        self.m, self.n = A.nrows, B.ncols
+        r0, r1 = (0, A.nrows) if rows is None else (int(rows[0]), int(rows[1]))
+        self.m, self.n = r1 - r0, B.ncols
         a = _CSC(A.nrows, A.ncols, A.rowidx.numel(), _ptr(A.colptr), _ptr(A.rowidx), _ptr(A.val), _where(A.colptr))
         b = _CSR(B.nrows, B.ncols, B.colidx.numel(), _ptr(B.rowptr), _ptr(B.colidx), _ptr(B.val), _where(B.rowptr))
         o = options(**opts)
         h = ctypes.c_void_p()
-        _check(lib().spgemm_plan(ctypes.byref(a), ctypes.byref(b), ctypes.byref(o), self.stream, ctypes.byref(h)))
+        _check(lib().spgemm_plan_rows(ctypes.byref(a), ctypes.byref(b), r0, r1, ctypes.byref(o), self.stream,
+                                      ctypes.byref(h)))
         self.h = h
 
     def expand(self):
@@ -288,9 +293,10 @@ class HostBufferPool:
         return b[:nbytes]
 
 
-def matmul(A: CSC, B: CSR, device=None, stream=None, **opts) -> CSR:
-    """C = A x B (outer-product spGEMM with the Block Reorganizer); C is canonical CSR."""
-    with Plan(A, B, stream=stream, **opts) as p:
+def matmul(A: CSC, B: CSR, device=None, stream=None, rows=None, **opts) -> CSR:
+    """C = A x B (outer-product spGEMM with the Block Reorganizer); C is canonical CSR.
+    rows=(r0, r1): only rows [r0, r1) of C (the row block, renumbered from 0)."""
+    with Plan(A, B, stream=stream, rows=rows, **opts) as p:
         return p.execute(device=device)
 
 
@@ -303,9 +309,8 @@ def matmul_chunked(A: CSC, B: CSR, parts: int, device=None, stream=None, **opts)
         return matmul(A, B, device=device, stream=stream, **opts)
     bounds = row_partition(A, B, parts, stream=stream)
     blocks = []
-    for r in range(parts):
-        Ar = pdist.csc_row_slice(A, int(bounds[r]), int(bounds[r + 1]))
-        C = matmul(Ar, B, device=device, stream=stream, **opts)
+    for r in range(parts):   # (the row window is cut on the GPU by spgemm_plan_rows: no copy of A here)
+        C = matmul(A, B, device=device, stream=stream, rows=(int(bounds[r]), int(bounds[r + 1])), **opts)
         if C.colidx.untyped_storage().nbytes() > C.colidx.numel() * 4 * 1.05:   # release capacity slack
             C = CSR(C.nrows, C.ncols, C.rowptr, C.colidx.clone(), C.val.clone())
         blocks.append(C)

@@ -93,6 +93,39 @@ __global__ void k_validate_idx(const int64_t *__restrict__ ptr, const int32_t *_
     if (bad) atomicOr(flag, bit);
 }
 
+// ---------------------------------------------------------------- row window -------------
+// spgemm_plan_rows: rows [r0, r1) of A (CSC, rows ascending per column) are, in every column, one
+// contiguous range of entries -- found by two binary searches; the window's A' is those ranges
+// packed (row indices minus r0), so C' = A' x B is rows [r0, r1) of C.
+__global__ void k_window_count(const int64_t *__restrict__ colptr, const int32_t *__restrict__ rowidx, int64_t K,
+                               int32_t r0, int32_t r1, int64_t *__restrict__ lo, int64_t *__restrict__ cnt) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < K; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t a = colptr[k], b = colptr[k + 1];
+        int64_t l = a, h = b;   // first entry with row >= r0
+        while (l < h) { const int64_t m = (l + h) >> 1; if (rowidx[m] < r0) l = m + 1; else h = m; }
+        const int64_t first = l;
+        h = b;                  // first entry with row >= r1
+        while (l < h) { const int64_t m = (l + h) >> 1; if (rowidx[m] < r1) l = m + 1; else h = m; }
+        lo[k] = first;
+        cnt[k] = l - first;
+    }
+}
+
+// one warp per column copies its window range
+__global__ void k_window_copy(const int64_t *__restrict__ lo, const int64_t *__restrict__ newptr, int64_t K,
+                              const int32_t *__restrict__ rowidx, const float *__restrict__ val, int32_t r0,
+                              int32_t *__restrict__ out_idx, float *__restrict__ out_val) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t k = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; k < K;
+         k += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+        const int64_t src = lo[k], dst = newptr[k], n = newptr[k + 1] - dst;
+        for (int64_t q = lane; q < n; q += 32) {
+            out_idx[dst + q] = rowidx[src + q] - r0;
+            out_val[dst + q] = val[src + q];
+        }
+    }
+}
+
 // ---------------------------------------------------------------- stage (1) --------------
 // Block-wise nnz: work[k] = nnz(a_*k) * nnz(b_k*)  (L326-L330 L, L290-L291 R).
 __global__ void __launch_bounds__(256) k_pair_work(const int64_t *__restrict__ a_colptr,

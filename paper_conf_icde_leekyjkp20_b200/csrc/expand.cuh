@@ -120,7 +120,8 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     const Piece *__restrict__ pieces, const int64_t *__restrict__ uoff, int64_t npieces,
     const int64_t *__restrict__ tile_p0, const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ bp_col,
     const float *__restrict__ bp_val, const float *__restrict__ a_val, const int64_t *__restrict__ base,
-    int32_t *__restrict__ chat_col, float *__restrict__ chat_val, unsigned long long *lbi) {
+    int32_t *__restrict__ chat_col, float *__restrict__ chat_val, unsigned long long *lbi,
+    const int64_t *__restrict__ unit_lo_ptr) {
     lbi_start(lbi);
     __shared__ int64_t s_uoff[kExpPieceCache + 1];
     __shared__ int64_t s_alo[kExpPieceCache];
@@ -129,8 +130,10 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     __shared__ int32_t s_boff[kExpPieceCache];
     const int64_t total = uoff[npieces];
     const int64_t ntiles = (total + kExpTile - 1) / kExpTile;
-    for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const int64_t f0 = tile * kExpTile, f1 = min(total, f0 + kExpTile);
+    const int64_t unit_lo = *unit_lo_ptr;        // (units below unit_lo: the block kernel's)
+    const int64_t tile0 = unit_lo / kExpTile;
+    for (int64_t tile = tile0 + blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const int64_t f0 = max(unit_lo, tile * kExpTile), f1 = min(total, tile * kExpTile + kExpTile);
         const int64_t p0 = tile_p0[tile];
         const int64_t pend = tile_p0[tile + 1] + 1;   // blocks [p0, pend) overlap the tile
         const int np = (int)min(pend - p0, (int64_t)kExpPieceCache + 1);
@@ -200,6 +203,143 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
                            make_float4(av[u] * w4[u].x, av[u] * w4[u].y, av[u] * w4[u].z, av[u] * w4[u].w));
                 }
         }
+    }
+    lbi_end(lbi);
+}
+
+// ------------------------------------------------ block path: TMA-staged B' tiles -------
+// Split pieces and whole Normal blocks (>= 32 effective threads, L317-L318 R): one block at a
+// time per CTA, claimed in order.  The block's B' tile (nv 16-byte vectors of columns and of
+// values, <= 1024 each) is brought into shared memory by two bulk copies (cp.async.bulk, TMA
+// engine; double-buffered: the next block's tile streams in while this one is written), then
+// every A entry e of the block is written as one run Ĉ[base[e] + b_off ..) = (cols, a_e * vals):
+// groups of W = min(32, 2^ceil(log2 nv)) lanes take an A entry each and stride over its vectors
+// -- two 16-byte stores per 4 products, no per-unit search, division or global B' load.
+constexpr int kExpBlkThreads = 256;
+constexpr int kExpBlkVec = 1024;   // max vectors of one B tile (split_b_tile <= 4096)
+constexpr int kExpBlkSmem = 2 * 2 * kExpBlkVec * 16;   // 2 buffers x (cols, vals) = 64 KB
+
+__device__ __forceinline__ void exp_mbar_init(uint64_t *mbar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"((uint32_t)__cvta_generic_to_shared(mbar)), "r"(1)
+                 : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void exp_bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *mbar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     (uint32_t)__cvta_generic_to_shared(dst)),
+                 "l"(src), "r"(bytes), "r"((uint32_t)__cvta_generic_to_shared(mbar))
+                 : "memory");
+}
+__device__ __forceinline__ void exp_expect_tx(uint64_t *mbar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(
+                     (uint32_t)__cvta_generic_to_shared(mbar)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void exp_wait(uint64_t *mbar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"((uint32_t)__cvta_generic_to_shared(mbar)),
+        "r"(parity)
+        : "memory");
+}
+
+__global__ void __launch_bounds__(kExpBlkThreads) k_expand_blocks(
+    const Piece *__restrict__ pieces, int64_t nblk, const int64_t *__restrict__ b_rowptr,
+    const int32_t *__restrict__ bp_col, const float *__restrict__ bp_val, const float *__restrict__ a_val,
+    const int64_t *__restrict__ base, int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
+    unsigned long long *ticket, unsigned long long *lbi) {
+    lbi_start(lbi);
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ uint64_t mbar[2];
+    __shared__ int64_t s_next;
+    __shared__ float s_av[kExpBlkThreads];      // the block's A values and run bases (a_len <= 256:
+    __shared__ int64_t s_dst[kExpBlkThreads];   //  split_ca_max bounds every block's A range)
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        exp_mbar_init(&mbar[0]);
+        exp_mbar_init(&mbar[1]);
+    }
+    __syncthreads();
+    uint32_t phases = 0;   // mbarrier parity of buffer b in bit b
+    // issue the bulk copies of vectors [v0, v0 + min(rest, kExpBlkVec)) of block q into buffer b
+    auto issue = [&](int64_t q, int b, int v0) {
+        const Piece pc = pieces[q];
+        const int nv = min(piece_nvec(pc) - v0, kExpBlkVec);
+        const int64_t src = bp_start(b_rowptr[pc.k], pc.k) + pc.b_off + 4 * (int64_t)v0;
+        int4 *dc = reinterpret_cast<int4 *>(smem_raw + (size_t)b * 2 * kExpBlkVec * 16);
+        float4 *dv = reinterpret_cast<float4 *>(dc + kExpBlkVec);
+        exp_expect_tx(&mbar[b], (uint32_t)nv * 32u);
+        exp_bulk_load(dc, bp_col + src, (uint32_t)nv * 16u, &mbar[b]);
+        exp_bulk_load(dv, bp_val + src, (uint32_t)nv * 16u, &mbar[b]);
+    };
+    int64_t cur = 0;
+    if (tid == 0) {
+        cur = (int64_t)atomicAdd(ticket, 1ull);
+        if (cur < nblk) issue(cur, 0, 0);
+        s_next = cur;
+    }
+    __syncthreads();
+    cur = s_next;
+    int b = 0;
+    while (cur < nblk) {
+        __syncthreads();   // (s_next of the previous round read; the other buffer's readers done)
+        if (tid == 0) {    // prefetch the next block into the other buffer
+            const int64_t nx = (int64_t)atomicAdd(ticket, 1ull);
+            if (nx < nblk) issue(nx, b ^ 1, 0);
+            s_next = nx;
+        }
+        const Piece pc = pieces[cur];
+        const int nvall = piece_nvec(pc);
+
+        const int4 *sc = reinterpret_cast<const int4 *>(smem_raw + (size_t)b * 2 * kExpBlkVec * 16);
+        const float4 *sv = reinterpret_cast<const float4 *>(sc + kExpBlkVec);
+        // (a whole Normal block's B row can exceed one buffer: its further sub-tiles reuse this one)
+        for (int v0 = 0; v0 < nvall; v0 += kExpBlkVec) {
+            if (v0 > 0) {
+                __syncthreads();   // the previous sub-tile's readers are done
+                if (tid == 0) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    issue(cur, b, v0);
+                }
+            }
+            exp_wait(&mbar[b], (phases >> b) & 1u);
+            phases ^= 1u << b;
+            const int nv = min(nvall - v0, kExpBlkVec);
+            const int lw = nv >= 32 ? 5 : (nv <= 1 ? 0 : 32 - __clz(nv - 1));   // lanes per A entry: 2^lw
+            const int W = 1 << lw;
+            const int sub = tid >> lw;                          // entry slot of this lane group
+            const int nsub = kExpBlkThreads >> lw;
+            const int li = tid & (W - 1);
+            for (int a0 = 0; a0 < pc.a_len; a0 += kExpBlkThreads) {   // A entries in chunks of 256
+                const int na = min(pc.a_len - a0, kExpBlkThreads);
+                __syncthreads();   // (the previous chunk's readers are done)
+                if (tid < na) {    // one coalesced load per A entry
+                    s_av[tid] = __ldg(a_val + pc.a_lo + a0 + tid);
+                    s_dst[tid] = __ldg(base + pc.a_lo + a0 + tid) + pc.b_off;
+                }
+                __syncthreads();
+                for (int a = sub; a < na; a += nsub) {
+                    const float av = s_av[a];
+                    const int64_t dst = s_dst[a] + 4 * (int64_t)v0;
+                    int4 *oc = reinterpret_cast<int4 *>(chat_col + dst);
+                    float4 *ov = reinterpret_cast<float4 *>(chat_val + dst);
+                    for (int v = li; v < nv; v += W) {
+                        const float4 w = sv[v];
+                        __stcs(oc + v, sc[v]);
+                        __stcs(ov + v, make_float4(av * w.x, av * w.y, av * w.z, av * w.w));
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        if (tid == 0) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // before the next prefetch
+        cur = s_next;
+        b ^= 1;
     }
     lbi_end(lbi);
 }

@@ -80,125 +80,6 @@ __global__ void __launch_bounds__(256) k_merge_warp(const int32_t *__restrict__ 
     if (lane == 0 && !out_col) ccount[i] = __popc(tails);
 }
 
-// ------------------------------------------------------------ warp bins, E slots/lane ---
-// One warp per row of <= 32E padded slots, held in registers in blocked order (lane l owns
-// slots [lE, lE + E)): bitonic network over the 32E (col, val) pairs (partners at distance >= E
-// by shuffles, closer ones inside the lane), then an fp64 segmented reduction -- in-lane running
-// sums plus a segmented scan of the lanes' open tails -- and the segment ends are written back
-// in place (the row is in registers).  No shared memory: rows of <= 256 slots with few runs
-// (C4: 8 runs of 8) cost ~log2(32E)^2/2 shuffle stages instead of merge levels in smem.
-template <int E>
-__global__ void __launch_bounds__(256) k_merge_warpE(const int32_t *__restrict__ rows, int64_t nrows,
-                                                     const int64_t *__restrict__ rowoff, int32_t *__restrict__ chat_col,
-                                                     float *__restrict__ chat_val, int64_t *__restrict__ ccount) {
-    constexpr int N = 32 * E;
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (gw >= nrows) return;
-    const int lane = lane_id();
-    const int i = rows[gw];
-    const int64_t s = rowoff[i];
-    const int L = (int)(rowoff[i + 1] - s);   // multiple of 4 (padded runs)
-    int32_t k[E];
-    float v[E];
-    if constexpr (E % 4 == 0) {
-#pragma unroll
-        for (int q = 0; q < E / 4; ++q) {
-            const int p = lane * E + 4 * q;
-            int4 c = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
-            float4 f = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (p < L) {
-                c = __ldcs(reinterpret_cast<const int4 *>(chat_col + s + p));
-                f = __ldcs(reinterpret_cast<const float4 *>(chat_val + s + p));
-            }
-            k[4 * q] = c.x; k[4 * q + 1] = c.y; k[4 * q + 2] = c.z; k[4 * q + 3] = c.w;
-            v[4 * q] = f.x; v[4 * q + 1] = f.y; v[4 * q + 2] = f.z; v[4 * q + 3] = f.w;
-        }
-    } else {
-#pragma unroll
-        for (int e = 0; e < E; ++e) {
-            const int p = lane * E + e;
-            k[e] = p < L ? chat_col[s + p] : kKeyPad;
-            v[e] = p < L ? chat_val[s + p] : 0.f;
-        }
-    }
-#pragma unroll
-    for (int kk = 2; kk <= N; kk <<= 1) {
-#pragma unroll
-        for (int j = kk >> 1; j > 0; j >>= 1) {
-            if (j >= E) {
-#pragma unroll
-                for (int e = 0; e < E; ++e) {
-                    const int idx = lane * E + e;
-                    const int32_t pk = __shfl_xor_sync(kFull, k[e], j / E);
-                    const float pv = __shfl_xor_sync(kFull, v[e], j / E);
-                    const bool up = (idx & kk) == 0, lower = (idx & j) == 0;
-                    if (lower == up ? (pk < k[e]) : (pk > k[e])) { k[e] = pk; v[e] = pv; }
-                }
-            } else {
-#pragma unroll
-                for (int e = 0; e < E; ++e) {
-                    const int f = e ^ j;
-                    if (f > e) {
-                        const bool up = ((lane * E + e) & kk) == 0;
-                        if (up ? (k[f] < k[e]) : (k[f] > k[e])) {
-                            const int32_t tk = k[e]; k[e] = k[f]; k[f] = tk;
-                            const float tv = v[e]; v[e] = v[f]; v[f] = tv;
-                        }
-                    }
-                }
-            }
-        }
-    }
-    // fp64 segmented sums: a segment starts where the key changes
-    const int32_t prev_last = __shfl_up_sync(kFull, k[E - 1], 1);
-    double acc[E];
-    double run = 0.0;
-    bool any_head = false;
-#pragma unroll
-    for (int e = 0; e < E; ++e) {
-        const bool head = e == 0 ? (lane == 0 || k[0] != prev_last) : (k[e] != k[e - 1]);
-        run = head ? (double)v[e] : run + (double)v[e];
-        any_head |= head;
-        acc[e] = run;
-    }
-    // segmented inclusive scan over lanes of (open tail sum, lane has a head)
-    double sc = run;
-    bool fl = any_head;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const double os = __shfl_up_sync(kFull, sc, d);
-        const bool of = __shfl_up_sync(kFull, (int)fl, d) != 0;
-        if (lane >= d && !fl) { sc += os; fl = of; }
-    }
-    double carry = __shfl_up_sync(kFull, sc, 1);
-    if (lane == 0) carry = 0.0;
-    bool open = true;   // slots before the lane's first head continue the previous lane's segment
-#pragma unroll
-    for (int e = 0; e < E; ++e) {
-        open &= !(e == 0 ? (lane == 0 || k[0] != prev_last) : (k[e] != k[e - 1]));
-        if (open) acc[e] += carry;
-    }
-    // segment ends (valid keys only) -> in place, in order
-    const int32_t next_first = __shfl_down_sync(kFull, k[0], 1);
-    int nt = 0;
-    bool tail[E];
-#pragma unroll
-    for (int e = 0; e < E; ++e) {
-        const int32_t nk = e < E - 1 ? k[e + 1] : (lane == 31 ? kKeyPad : next_first);
-        tail[e] = k[e] != kKeyPad && (nk != k[e] || (e == E - 1 && lane == 31));
-        nt += tail[e];
-    }
-    const int inc = warp_incl_sum(nt);
-    int o = inc - nt;
-#pragma unroll
-    for (int e = 0; e < E; ++e)
-        if (tail[e]) {
-            chat_col[s + o] = k[e];
-            chat_val[s + o] = (float)acc[e];
-            ++o;
-        }
-    if (lane == 31) ccount[i] = inc;
-}
 
 // ------------------------------------------------------------------ thread groups ---
 // A group of NW warps works on one row; GROUPS groups share a CTA.  Groups synchronise with
@@ -441,32 +322,6 @@ __device__ __forceinline__ int nextpow2_log(int x) { return x <= 1 ? 0 : 32 - __
 // ranges (stride = buckets per thread) hit distinct banks
 __host__ __device__ __forceinline__ constexpr int hidx(int b) { return b + (b >> 5); }
 
-// Copy a warp's contiguous output slice: lane l staged u_l entries at (sk, sv)[st_l ..) and
-// they go to out[wbase + ex_l ..), ex_l = exclusive prefix of u over the warp's lanes.
-__device__ __forceinline__ int warp_copy_out(int st, int u, int64_t wbase, const int32_t *sk, const float *sv,
-                                             int32_t *__restrict__ out_col, float *__restrict__ out_val) {
-    const int lane = lane_id();
-    const int inc = warp_incl_sum(u);
-    const int ex = inc - u;
-    const int wtot = __shfl_sync(kFull, inc, 31);
-    for (int o0 = 0; o0 < wtot; o0 += 32) {      // warp-uniform trip count (shuffles below)
-        const int o = o0 + lane;
-        int pos = 0;   // owner = number of lanes with inc <= o
-#pragma unroll
-        for (int step = 16; step > 0; step >>= 1) {
-            const int probe = __shfl_sync(kFull, inc, min(pos + step - 1, 31));
-            if (pos + step <= 32 && probe <= o) pos += step;
-        }
-        const int owner = min(pos, 31);
-        const int src = __shfl_sync(kFull, st, owner) + (o - __shfl_sync(kFull, ex, owner));
-        if (o < wtot) {
-            out_col[wbase + o] = sk[src];
-            out_val[wbase + o] = sv[src];
-        }
-    }
-    return wtot;
-}
-
 // striped load of a row into registers (slot gtid + e*T); sentinel (padding) entries stay kKeyPad
 template <int NW, int GROUPS, int EPT>
 __device__ __forceinline__ void bsr_load(const Group<NW, GROUPS> &g, const int32_t *sk, const float *sv, int L,
@@ -486,100 +341,6 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
                                                        float *dv2, int *hist, int32_t *out_col, float *out_val,
                                                        int *sc, int32_t pmn = 1, int32_t pmx = 0);
 
-// Bucket-owner variant: after the scatter, every thread owns the contiguous bucket range it
-// scanned, insertion-sorts its multi-key buckets in place and reduces them (equal keys never
-// leave a bucket) into the head of its slot range; a group scan of the per-thread counts places
-// them and each warp copies its lanes' ranges out coalesced.  No second (dk2, dv2) buffer and no
-// per-element ranking loop.  Returns -1 on a bucket of > kBucketMax keys.
-template <int NW, int GROUPS, int EPT>
-__device__ __forceinline__ int bucket_walk_reduce_regs(const Group<NW, GROUPS> &g, int32_t (&key)[EPT],
-                                                       float (&val)[EPT], int L, int32_t *dk, float *dv, int *hist,
-                                                       int32_t *out_col, float *out_val, int *sc) {
-    constexpr int T = NW * 32;
-    int32_t mn = kKeyPad, mx = 0;
-#pragma unroll
-    for (int e = 0; e < EPT; ++e)
-        if (key[e] != kKeyPad) { mn = min(mn, key[e]); mx = max(mx, key[e]); }
-    mn = g.reduce_min(mn, sc);
-    mx = g.reduce_max(mx, sc);
-    const uint32_t span = (uint32_t)(mx - mn);
-    const int lognb = nextpow2_log(L);
-    const int nb = 1 << lognb;
-    const int bits = span ? 32 - __clz(span) : 0;
-    const int sh = max(0, bits - lognb);
-    for (int b = g.gtid; b <= hidx(nb); b += T) hist[b] = 0;
-    g.sync();
-    int rk[EPT];
-#pragma unroll
-    for (int e = 0; e < EPT; ++e)
-        rk[e] = key[e] != kKeyPad ? atomicAdd(&hist[hidx((key[e] - mn) >> sh)], 1) : 0;
-    g.sync();
-    const int bpt = (nb + T - 1) / T;
-    const int b0 = min(nb, g.gtid * bpt), b1 = min(nb, b0 + bpt);
-    int cnt = 0, mxc = 0;
-    for (int b = b0; b < b1; ++b) {
-        const int c = hist[hidx(b)];
-        cnt += c;
-        mxc = max(mxc, c);
-    }
-    int tot;
-    int ex = g.excl_sum(cnt, sc, &tot);
-    if (g.reduce_max(mxc, sc) > kBucketMax) return -1;
-    const int S = ex, E = ex + cnt;
-    for (int b = b0; b < b1; ++b) {
-        const int c = hist[hidx(b)];
-        hist[hidx(b)] = ex;
-        ex += c;
-    }
-    if (g.gtid == 0) hist[hidx(nb)] = tot;
-    g.sync();
-#pragma unroll
-    for (int e = 0; e < EPT; ++e)
-        if (key[e] != kKeyPad) {
-            const int pos = hist[hidx((key[e] - mn) >> sh)] + rk[e];
-            dk[pos] = key[e];
-            dv[pos] = val[e];
-        }
-    g.sync();
-    // owner walk: sort each multi-key bucket (insertion), then reduce the range in place
-    {
-        int bs = S;
-        for (int b = b0; b < b1; ++b) {
-            const int be = b + 1 < b1 ? hist[hidx(b + 1)] : E;
-            for (int p = bs + 1; p < be; ++p) {
-                const int32_t kk = dk[p];
-                const float vv = dv[p];
-                int q = p - 1;
-                while (q >= bs && dk[q] > kk) { dk[q + 1] = dk[q]; dv[q + 1] = dv[q]; --q; }
-                dk[q + 1] = kk;
-                dv[q + 1] = vv;
-            }
-            bs = be;
-        }
-    }
-    int u = 0;
-    {
-        int32_t cur = -1;
-        double acc = 0.0;
-        for (int p = S; p < E; ++p) {
-            const int32_t k = dk[p];
-            const float v = dv[p];
-            if (k != cur) {
-                if (cur != -1) { dk[S + u] = cur; dv[S + u] = (float)acc; ++u; }
-                cur = k;
-                acc = (double)v;
-            } else {
-                acc += (double)v;
-            }
-        }
-        if (cur != -1) { dk[S + u] = cur; dv[S + u] = (float)acc; ++u; }
-    }
-    int U;
-    const int o = g.excl_sum(u, sc, &U);
-    const int64_t wbase = __shfl_sync(kFull, o, 0);
-    warp_copy_out(S, u, wbase, dk, dv, out_col, out_val);
-    return U;
-}
 
 // LS: buckets = 2^LS x (slots rounded up to a power of two); more buckets, fewer shared ones.
 // UNR2: in-bucket ranking two keys per step (the B-Limited groups' wider buckets: C3 -5 %; the
@@ -825,7 +586,7 @@ __global__ void k_row_meta(const int32_t *__restrict__ order, int64_t n, const i
     }
 }
 
-template <int NW, int GROUPS, int EPT, int LS = 0, bool WALK = false>
+template <int NW, int GROUPS, int EPT, int LS = 0>
 __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k_merge_bucket_pipe(
     const RowMeta *__restrict__ meta, int64_t nrows, int32_t *__restrict__ chat_col, float *__restrict__ chat_val,
     int64_t *__restrict__ ccount, int32_t *__restrict__ fb_rows, unsigned *__restrict__ fb_count,
@@ -848,10 +609,9 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
     int32_t key[EPT];
     float val[EPT];
     bsr_load<NW, GROUPS, EPT>(g, chat_col + m0.s, chat_val + m0.s, min(m0.L, S::kCap), key, val);
-    if constexpr (!WALK) {   // PRECLEAR: hist starts zeroed, every row leaves it zeroed
-        for (int b = g.gtid; b <= hidx(S::kNb); b += NW * 32) hist[b] = 0;
-        g.sync();
-    }
+    // PRECLEAR: hist starts zeroed, every row leaves it zeroed
+    for (int b = g.gtid; b <= hidx(S::kNb); b += NW * 32) hist[b] = 0;
+    g.sync();
     while (r < nrows) {
         const int2 rg = rng ? rng[r] : make_int2(1, 0);
         int32_t kn[EPT];
@@ -859,20 +619,14 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
         bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, min(m1.L, S::kCap), kn, vn);
         const RowMeta m2 = r + 2 * stride < nrows ? meta[r + 2 * stride] : none;
         if (m0.L <= S::kCap) {
-            int U;
-            if constexpr (WALK)
-                U = bucket_walk_reduce_regs<NW, GROUPS, EPT>(g, key, val, m0.L, dk, dv, hist, chat_col + m0.s,
-                                                             chat_val + m0.s, sc_all[g.gid]);
-            else
-                U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, false, hidx(S::kNb)>(g, key, val, m0.L, dk, dv, dk2, dv2, hist,
-                                                                 chat_col + m0.s, chat_val + m0.s, sc_all[g.gid],
-                                                                 rg.x, rg.y);
+            const int U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, false, hidx(S::kNb)>(
+                g, key, val, m0.L, dk, dv, dk2, dv2, hist, chat_col + m0.s, chat_val + m0.s, sc_all[g.gid], rg.x, rg.y);
             if (g.gtid == 0) {
                 if (U >= 0) ccount[m0.i] = U;
                 else fb_rows[atomicAdd(fb_count, 1u)] = m0.i;
             }
         }
-        if constexpr (WALK) g.sync();   // (bucket sort: no barrier needed between rows, see k_merge_bucket)
+        // (no barrier needed between rows, see k_merge_bucket)
 #pragma unroll
         for (int e = 0; e < EPT; ++e) { key[e] = kn[e]; val[e] = vn[e]; }
         m0 = m1;
@@ -881,272 +635,6 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
     }
 }
 
-// ------------------------------------------- register-staged counting sort (WCS) ---
-// One warp per row; the row is held in registers (VPT int4 + float4 vectors per lane, CAP =
-// 128*VPT slots) and shared memory holds only the scattered keys / values, the histogram and a
-// bitmap of bucket starts: ~12.3 B per slot, so CAP = 1024 is 12.4 KB and ~17 rows are in
-// flight per SM.
-//   1. vector loads of the padded row (runs are 16-byte aligned); min / max of its columns;
-//   2. nb = max(32, 2^ceil(log2 L)) buckets over the column span, bucket = (col - min) >> sh;
-//      histogram by shared-memory integer atomics;
-//   3. lane l owns nb/32 consecutive buckets (stored at b + b/32, so the 32 lanes' walks hit
-//      distinct banks): exclusive scan -> bucket starts; non-empty bucket starts are marked in
-//      the bitmap;
-//   4. scatter by atomic cursor (order inside a bucket is arbitrary);
-//   5. warp_merge_buckets: 32 slots at a time, cut at the last bucket start, so a chunk holds
-//      whole buckets; keys of a bucket are compared by shuffles (only chunks with a bucket of
-//      >= 2 keys loop), each distinct key's fp64 sum is written at its sorted output index.
-// Segments never cross buckets (equal keys share a bucket), so each chunk is independent.
-constexpr int kBitsPad = 3;   // bitmap words read past the end by bits64()
-
-// bits [p, p + 64) of the bucket-start bitmap
-__device__ __forceinline__ uint64_t bits64(const uint32_t *bits, int p) {
-    const int w = p >> 5, sh = p & 31;
-    const uint32_t a = bits[w], b = bits[w + 1], c = bits[w + 2];
-    const uint32_t lo = __funnelshift_r(a, b, sh), hi = __funnelshift_r(b, c, sh);
-    return (uint64_t)lo | ((uint64_t)hi << 32);
-}
-
-// Ascending bitonic sort of (k, v)[0, n) in shared memory by one warp; indices >= n act as +inf
-// (every comparator puts the minimum at the lower index, so virtual padding never moves).
-__device__ __noinline__ void warp_bitonic_smem(int32_t *k, float *v, int n) {
-    int N = 1;
-    while (N < n) N <<= 1;
-    const int lane = lane_id();
-    auto cmpswap = [&](int i, int j) {
-        if (j < n) {
-            const int32_t ki = k[i], kj = k[j];
-            if (kj < ki) {
-                const float vi = v[i];
-                k[i] = kj; k[j] = ki;
-                v[i] = v[j]; v[j] = vi;
-            }
-        }
-    };
-    for (int size = 2; size <= N; size <<= 1) {
-        const int half = size >> 1;
-        for (int t = lane; t < (N >> 1); t += 32) {     // flip: i <-> mirror in its block
-            const int blk = (t / half) * size, off = t % half;
-            cmpswap(blk + off, blk + size - 1 - off);
-        }
-        __syncwarp();
-        for (int d = half >> 1; d >= 1; d >>= 1) {      // half-cleaners
-            for (int t = lane; t < (N >> 1); t += 32) {
-                const int blk = (t / d) * (2 * d), off = t % d;
-                cmpswap(blk + off, blk + off + d);
-            }
-            __syncwarp();
-        }
-    }
-}
-
-// Merge the slots [lo, hi) of a row (or of a tile of rows) whose buckets are contiguous and
-// marked in `bits` (lo is a bucket start): every distinct key of a bucket is emitted once, in
-// ascending key order, with the fp64 sum of its values, through emit(o, key, value) with
-// o = 0, 1, ... (warp-uniform call sites; o is relative to the range).  Returns the count.
-template <typename Emit>
-__device__ __forceinline__ int warp_merge_buckets(int32_t *sk, float *sv, const uint32_t *bits, int lo, int hi,
-                                                  Emit emit) {
-    const int lane = lane_id();
-    int ob = 0;
-    int p0 = lo;
-    while (p0 < hi) {
-        uint64_t m = bits64(bits, p0) | 1ull;
-        const int rem = hi - p0;
-        if (rem < 64) m = (m & ((1ull << rem) - 1)) | (1ull << rem);   // hi is a boundary
-        const uint64_t m33 = m & 0x1FFFFFFFEull;                        // boundaries in [1, 32]
-        if (m33 == 0) {
-            // one bucket of more than 32 keys: find its end, sort it (unless single-valued)
-            int e = p0 + 64;
-            while (e < hi) {
-                const uint64_t mm = bits64(bits, e);
-                if (mm) { e += __ffsll((long long)mm) - 1; break; }
-                e += 64;
-            }
-            e = min(e, hi);
-            int32_t kmin = kKeyPad, kmax = 0;
-            for (int p = p0 + lane; p < e; p += 32) { kmin = min(kmin, sk[p]); kmax = max(kmax, sk[p]); }
-            kmin = __reduce_min_sync(kFull, kmin);
-            kmax = __reduce_max_sync(kFull, kmax);
-            if (kmin != kmax) warp_bitonic_smem(sk + p0, sv + p0, e - p0);
-            __syncwarp();
-            for (int q0 = p0; q0 < e; q0 += 32) {
-                const int p = q0 + lane;
-                const bool in = p < e;
-                const int32_t k = in ? sk[p] : kKeyPad;
-                int32_t prev = __shfl_up_sync(kFull, k, 1);
-                if (lane == 0) prev = q0 > p0 ? sk[q0 - 1] : ~k;
-                const bool head = in && k != prev;
-                double acc = 0.0;
-                if (head) {
-                    acc = (double)sv[p];
-                    for (int q = p + 1; q < e && sk[q] == k; ++q) acc += (double)sv[q];
-                }
-                const unsigned hm = __ballot_sync(kFull, head);
-                __syncwarp();
-                if (head) emit(ob + __popc(hm & lanemask_lt()), k, acc);
-                ob += __popc(hm);
-            }
-            __syncwarp();
-            p0 = e;
-            continue;
-        }
-        const int n = 63 - __clzll((long long)m33);   // lanes [0, n) hold whole buckets
-        const bool ok = lane < n;
-        const int p = p0 + lane;
-        const int32_t k = ok ? sk[p] : kKeyPad;
-        const float v = ok ? sv[p] : 0.f;
-        const uint32_t mlo = (uint32_t)m;
-        const int bs = 31 - __clz(mlo & (lane == 31 ? kFull : ((2u << lane) - 1)));   // bucket start lane
-        const uint64_t above = m & ~((2ull << lane) - 1);
-        const int be = __ffsll((long long)above) - 1;                                 // bucket end lane
-        const int c = ok ? be - bs : 0;
-        bool rep = ok;
-        double acc = (double)v;
-        int nless = 0;
-        const int maxc = __reduce_max_sync(kFull, c);
-        if (maxc > 1) {
-            const int myq = lane - bs;
-            acc = 0.0;
-            for (int q = 0; q < maxc; ++q) {
-                const int src = min(bs + q, 31);
-                const int32_t kq = __shfl_sync(kFull, k, src);
-                const float vq = __shfl_sync(kFull, v, src);
-                if (q < c && kq == k) {
-                    acc += (double)vq;
-                    if (q < myq) rep = false;
-                }
-            }
-            for (int q = 0; q < maxc; ++q) {
-                const int src = min(bs + q, 31);
-                const int32_t kq = __shfl_sync(kFull, k, src);
-                const bool rq = __shfl_sync(kFull, (int)rep, src) != 0;
-                nless += (q < c && rq && kq < k);
-            }
-        }
-        const unsigned rm = __ballot_sync(kFull, rep);
-        __syncwarp();
-        if (rep) emit(ob + __popc(rm & ((1u << bs) - 1)) + nless, k, acc);
-        ob += __popc(rm);
-        p0 += n;
-    }
-    __syncwarp();
-    return ob;
-}
-
-template <int VPT>
-struct WcsSmem {
-    static constexpr int kCap = 32 * VPT * 4;      // power of two
-    static constexpr int kHist = kCap + kCap / 32;
-    static constexpr int kBits = kCap / 32 + kBitsPad;
-    static constexpr int kBytes = kCap * 8 + kHist * 4 + kBits * 4;
-};
-
-__device__ __forceinline__ int wcs_hidx(int b) { return b + (b >> 5); }
-
-template <int GROUPS, int VPT>
-__global__ void __launch_bounds__(32 * GROUPS) k_merge_wcs(const int32_t *__restrict__ rows, int64_t nrows,
-                                                          const int64_t *__restrict__ rowoff,
-                                                          const int64_t *__restrict__ rowwork,
-                                                          int32_t *__restrict__ chat_col,
-                                                          float *__restrict__ chat_val,
-                                                          int64_t *__restrict__ ccount,
-                                                          const int64_t *__restrict__ crowptr,
-                                                          int32_t *__restrict__ out_col_all,
-                                                          float *__restrict__ out_val_all) {
-    using S = WcsSmem<VPT>;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    const int gid = threadIdx.x >> 5;
-    unsigned char *slice = smem_raw + (size_t)gid * S::kBytes;
-    int32_t *sk = (int32_t *)slice;
-    float *sv = (float *)(slice + S::kCap * 4);
-    int *hist = (int *)(slice + S::kCap * 8);
-    uint32_t *bits = (uint32_t *)(slice + S::kCap * 8 + S::kHist * 4);
-    const int lane = lane_id();
-    for (int64_t r = (int64_t)blockIdx.x * GROUPS + gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
-        const int i = rows[r];
-        const int64_t s = rowoff[i];
-        const int nv = (int)((rowoff[i + 1] - s) >> 2);
-        const int L = (int)rowwork[i];
-        int4 kc[VPT];
-        float4 kv[VPT];
-#pragma unroll
-        for (int j = 0; j < VPT; ++j) {
-            const int v = lane + j * 32;
-            if (v < nv) {
-                kc[j] = __ldcs(reinterpret_cast<const int4 *>(chat_col + s) + v);
-                kv[j] = __ldcs(reinterpret_cast<const float4 *>(chat_val + s) + v);
-            } else {
-                kc[j] = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
-            }
-        }
-        int32_t mn = kKeyPad, mx = 0;
-#pragma unroll
-        for (int j = 0; j < VPT; ++j) {
-            const int32_t c4[4] = {kc[j].x, kc[j].y, kc[j].z, kc[j].w};
-#pragma unroll
-            for (int u = 0; u < 4; ++u)
-                if (c4[u] != kKeyPad) { mn = min(mn, c4[u]); mx = max(mx, c4[u]); }
-        }
-        mn = __reduce_min_sync(kFull, mn);
-        mx = __reduce_max_sync(kFull, mx);
-        const int lognb = max(nextpow2_log(L), 5);
-        const int nb = 1 << lognb;
-        const uint32_t span = (uint32_t)(mx - mn);
-        const int bits_span = span ? 32 - __clz(span) : 0;
-        const int sh = max(0, bits_span - lognb);
-        const int nbh = nb + (nb >> 5);
-        for (int b = lane; b < nbh; b += 32) hist[b] = 0;
-        for (int w = lane; w < min(S::kBits, (L >> 5) + kBitsPad); w += 32) bits[w] = 0;
-        __syncwarp();
-#pragma unroll
-        for (int j = 0; j < VPT; ++j) {
-            const int32_t c4[4] = {kc[j].x, kc[j].y, kc[j].z, kc[j].w};
-#pragma unroll
-            for (int u = 0; u < 4; ++u)
-                if (c4[u] != kKeyPad) atomicAdd(&hist[wcs_hidx((c4[u] - mn) >> sh)], 1);
-        }
-        __syncwarp();
-        const int bpt = nb >> 5;
-        const int b0 = lane * bpt;
-        int cnt = 0;
-        for (int q = 0; q < bpt; ++q) cnt += hist[wcs_hidx(b0 + q)];
-        const int inc = warp_incl_sum(cnt);
-        {
-            int run = inc - cnt;
-            for (int q = 0; q < bpt; ++q) {
-                const int h = wcs_hidx(b0 + q);
-                const int c = hist[h];
-                hist[h] = run;
-                if (c) atomicOr(&bits[run >> 5], 1u << (run & 31));
-                run += c;
-            }
-        }
-        __syncwarp();
-#pragma unroll
-        for (int j = 0; j < VPT; ++j) {
-            const int32_t c4[4] = {kc[j].x, kc[j].y, kc[j].z, kc[j].w};
-            const float v4[4] = {kv[j].x, kv[j].y, kv[j].z, kv[j].w};
-#pragma unroll
-            for (int u = 0; u < 4; ++u)
-                if (c4[u] != kKeyPad) {
-                    const int p = atomicAdd(&hist[wcs_hidx((c4[u] - mn) >> sh)], 1);
-                    sk[p] = c4[u];
-                    sv[p] = v4[u];
-                }
-        }
-        __syncwarp();
-        const int64_t o0 = out_col_all ? crowptr[i] : s;
-        int32_t *__restrict__ out_col = (out_col_all ? out_col_all : chat_col) + o0;
-        float *__restrict__ out_val = (out_col_all ? out_val_all : chat_val) + o0;
-        const int U = warp_merge_buckets(sk, sv, bits, 0, L, [&](int o, int32_t k, double acc) {
-            out_col[o] = k;
-            out_val[o] = (float)acc;
-        });
-        if (lane == 0 && !out_col_all) ccount[i] = U;
-        __syncwarp();
-    }
-}
 
 // -------------------------------------------- warp merge-path natural merge sort (WMP) ---
 // No shared-memory atomics (see k_count_rows).  A row's bucket is a concatenation of runs (one
@@ -1176,232 +664,6 @@ struct WmpSmem {
     static constexpr int kBytes = CAP * 16 + 2 * kRuns * 4;
 };
 
-template <int NW, int GROUPS, int CAP>
-__global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_wmp(const int32_t *__restrict__ rows, int64_t nrows,
-                                                               const int64_t *__restrict__ rowoff,
-                                                               const int64_t *__restrict__ rowwork,
-                                                               int32_t *__restrict__ chat_col,
-                                                               float *__restrict__ chat_val,
-                                                               int64_t *__restrict__ ccount,
-                                                               const int64_t *__restrict__ crowptr,
-                                                               int32_t *__restrict__ out_col_all,
-                                                               float *__restrict__ out_val_all) {
-    using S = WmpSmem<CAP>;
-    constexpr int T = NW * 32;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ int sc_all[GROUPS][NW + 1];
-    __shared__ int wcnt_all[GROUPS][NW + 1];
-    const Group<NW, GROUPS> g;
-    int *sc = sc_all[g.gid];
-    int *wcnt = wcnt_all[g.gid];
-    const int lane = lane_id(), wg = g.gtid >> 5;
-    unsigned char *slice = smem_raw + (size_t)g.gid * S::kBytes;
-    uint64_t *bufA = (uint64_t *)slice;
-    uint64_t *bufB = bufA + CAP;
-    int *runsA = (int *)(bufB + CAP);
-    int *runsB = runsA + S::kRuns;
-    const unsigned lt = lanemask_lt();
-    for (int64_t r = (int64_t)blockIdx.x * GROUPS + g.gid; r < nrows; r += (int64_t)gridDim.x * GROUPS) {
-        const int i = rows[r];
-        const int64_t s = rowoff[i];
-        const int Lp = (int)(rowoff[i + 1] - s);
-        const int Lv = (int)rowwork[i];
-        const int nv = Lp >> 2;
-        const int4 *__restrict__ c4p = reinterpret_cast<const int4 *>(chat_col + s);
-        const float4 *__restrict__ v4p = reinterpret_cast<const float4 *>(chat_val + s);
-        // 1. load + pack; run starts
-        int R = 0;
-        if constexpr (NW == 1) {
-            int32_t carry = kKeyPad;
-            for (int v0 = 0; v0 < nv; v0 += 64) {
-                int4 c[2];
-                float4 f[2];
-#pragma unroll
-                for (int u = 0; u < 2; ++u) {
-                    const int v = v0 + 32 * u + lane;
-                    if (v < nv) { c[u] = __ldcs(c4p + v); f[u] = __ldcs(v4p + v); }
-                    else c[u] = make_int4(kKeyPad, kKeyPad, kKeyPad, kKeyPad);
-                }
-#pragma unroll
-                for (int u = 0; u < 2; ++u) {
-                    const int v = v0 + 32 * u + lane;
-                    int32_t prev = __shfl_up_sync(kFull, c[u].w, 1);
-                    if (lane == 0) prev = carry;
-                    carry = __shfl_sync(kFull, c[u].w, 31);
-                    const bool start = v < nv && (v == 0 || c[u].x < prev);
-                    const unsigned m = __ballot_sync(kFull, start);
-                    if (start) runsA[R + __popc(m & lt)] = 4 * v;
-                    R += __popc(m);
-                    if (v < nv) {
-                        ulonglong2 *d = reinterpret_cast<ulonglong2 *>(bufA + 4 * v);
-                        d[0] = make_ulonglong2(pack_kv(c[u].x, f[u].x), pack_kv(c[u].y, f[u].y));
-                        d[1] = make_ulonglong2(pack_kv(c[u].z, f[u].z), pack_kv(c[u].w, f[u].w));
-                    }
-                }
-            }
-            if (lane == 0) runsA[R] = Lp;
-            __syncwarp();
-        } else {
-            for (int v0 = 0; v0 < nv; v0 += 2 * T) {
-                int4 c[2];
-                float4 f[2];
-#pragma unroll
-                for (int u = 0; u < 2; ++u) {
-                    const int v = v0 + T * u + g.gtid;
-                    if (v < nv) { c[u] = __ldcs(c4p + v); f[u] = __ldcs(v4p + v); }
-                }
-#pragma unroll
-                for (int u = 0; u < 2; ++u) {
-                    const int v = v0 + T * u + g.gtid;
-                    if (v < nv) {
-                        ulonglong2 *d = reinterpret_cast<ulonglong2 *>(bufA + 4 * v);
-                        d[0] = make_ulonglong2(pack_kv(c[u].x, f[u].x), pack_kv(c[u].y, f[u].y));
-                        d[1] = make_ulonglong2(pack_kv(c[u].z, f[u].z), pack_kv(c[u].w, f[u].w));
-                    }
-                }
-            }
-            g.sync();
-            // run starts over contiguous vector ranges per thread, compacted by a group scan
-            const int vpt = (nv + T - 1) / T;
-            const int va = min(nv, g.gtid * vpt), vb = min(nv, va + vpt);
-            int ns = 0;
-            for (int v = va; v < vb; ++v) ns += (v == 0 || kv_key(bufA[4 * v]) < kv_key(bufA[4 * v - 1]));
-            int tot;
-            int pos = g.excl_sum(ns, sc, &tot);
-            for (int v = va; v < vb; ++v)
-                if (v == 0 || kv_key(bufA[4 * v]) < kv_key(bufA[4 * v - 1])) runsA[pos++] = 4 * v;
-            R = tot;
-            if (g.gtid == 0) runsA[R] = Lp;
-            g.sync();
-        }
-        // 2. merge levels
-        uint64_t *src = bufA, *dst = bufB;
-        int *rs = runsA, *rd = runsB;
-        const int E = (Lp + T - 1) / T;
-        while (R > 1) {
-            const int npairs = (R + 1) >> 1;
-            int o = min(Lp, g.gtid * E);
-            const int oend = min(Lp, o + E);
-            if (o < oend) {
-                int lo = 0, hi = npairs;      // pair holding output o: last q with rs[2q] <= o
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (rs[2 * mid] <= o) lo = mid; else hi = mid;
-                }
-                int q = lo;
-                while (o < oend) {
-                    const int a0 = rs[2 * q], a1 = rs[min(2 * q + 1, R)], b1 = rs[min(2 * q + 2, R)];
-                    const int d = o - a0;
-                    int ilo = max(0, d - (b1 - a1)), ihi = min(d, a1 - a0);
-                    while (ilo < ihi) {        // merge path: first i with A[i] > B[d - i - 1] (keys)
-                        const int mi = (ilo + ihi) >> 1;
-                        if (kv_key(src[a0 + mi]) <= kv_key(src[a1 + d - mi - 1])) ilo = mi + 1; else ihi = mi;
-                    }
-                    int ia = a0 + ilo, jb = a1 + d - ilo;
-                    uint64_t xa = ia < a1 ? src[ia] : kKvMax;
-                    uint64_t xb = jb < b1 ? src[jb] : kKvMax;
-                    const int pend = min(oend, b1);
-                    for (; o < pend; ++o) {
-                        const bool tA = kv_key(xa) <= kv_key(xb);
-                        dst[o] = tA ? xa : xb;
-                        const int nxt = tA ? ia + 1 : jb + 1;
-                        const uint64_t y = nxt < (tA ? a1 : b1) ? src[nxt] : kKvMax;
-                        ia = tA ? nxt : ia;
-                        jb = tA ? jb : nxt;
-                        xa = tA ? y : xa;
-                        xb = tA ? xb : y;
-                    }
-                    ++q;
-                }
-            }
-            for (int q = g.gtid; q <= npairs; q += T) rd[q] = q < npairs ? rs[2 * q] : Lp;
-            g.sync();
-            { uint64_t *t = src; src = dst; dst = t; }
-            { int *t = rs; rs = rd; rd = t; }
-            R = npairs;
-        }
-        // 3. reduction of the sorted products (sentinels sorted last) into C
-        int wlo = 0, whi = Lv;
-        if constexpr (NW > 1) {
-            const int per = (Lv + NW - 1) / NW;
-            wlo = min(Lv, wg * per);
-            whi = min(Lv, wlo + per);
-            // shares start at segment heads
-            if (lane == 0) {
-                while (wlo > 0 && wlo < Lv && kv_key(src[wlo]) == kv_key(src[wlo - 1])) ++wlo;
-                while (whi < Lv && kv_key(src[whi]) == kv_key(src[whi - 1])) ++whi;
-            }
-            wlo = __shfl_sync(kFull, wlo, 0);
-            whi = __shfl_sync(kFull, whi, 0);
-        }
-        // output: C at crowptr[i], or in place at the head of the row's Ĉ bucket (the whole row
-        // is in shared memory by now)
-        const int64_t obase = out_col_all ? crowptr[i] : s;
-        int32_t *__restrict__ out_col = out_col_all ? out_col_all : chat_col;
-        float *__restrict__ out_val = out_col_all ? out_val_all : chat_val;
-        int ob = 0;
-        uint64_t *stage = dst + wlo;   // NW > 1: the free buffer, at the warp's share
-        for (int p0 = wlo; p0 < whi; p0 += 32) {
-            const int p = p0 + lane;
-            const bool in = p < whi;
-            const uint64_t x = in ? src[p] : kKvMax;
-            const int32_t k = kv_key(x);
-            int32_t prev = __shfl_up_sync(kFull, k, 1);
-            if (lane == 0) prev = p0 > wlo ? kv_key(src[p0 - 1]) : ~k;
-            int32_t next = __shfl_down_sync(kFull, k, 1);
-            if (lane == 31) next = p + 1 < whi ? kv_key(src[p + 1]) : kKeyPad;
-            const bool head = in && k != prev;
-            const unsigned hm = __ballot_sync(kFull, head);
-            const bool dup = in && next == k;
-            if (hm == kFull && !__any_sync(kFull, dup)) {         // common case: 32 distinct keys
-                if constexpr (NW == 1) {
-                    out_col[obase + ob + lane] = k;
-                    out_val[obase + ob + lane] = kv_val(x);
-                } else {
-                    stage[ob + lane] = x;
-                }
-                ob += 32;
-                continue;
-            }
-            double acc = (double)kv_val(x);
-            if (head && dup)
-                for (int q = p + 1; q < whi; ++q) {
-                    const uint64_t y = src[q];
-                    if (kv_key(y) != k) break;
-                    acc += (double)kv_val(y);
-                }
-            if (head) {
-                const int o = ob + __popc(hm & lt);
-                if constexpr (NW == 1) {
-                    out_col[obase + o] = k;
-                    out_val[obase + o] = (float)acc;
-                } else {
-                    stage[o] = pack_kv(k, (float)acc);
-                }
-            }
-            ob += __popc(hm);
-        }
-        if constexpr (NW > 1) {
-            if (lane == 0) wcnt[wg] = ob;
-            g.sync();
-            int wb = 0;
-            for (int w = 0; w < wg; ++w) wb += wcnt[w];
-            for (int q = lane; q < ob; q += 32) {
-                const uint64_t x = stage[q];
-                out_col[obase + wb + q] = kv_key(x);
-                out_val[obase + wb + q] = kv_val(x);
-            }
-            if (g.gtid == 0 && !out_col_all) {
-                int U = 0;
-                for (int w = 0; w < NW; ++w) U += wcnt[w];
-                ccount[i] = U;
-            }
-        } else {
-            if (lane == 0 && !out_col_all) ccount[i] = ob;
-        }
-        g.sync();
-    }
-}
 
 // Software-pipelined warp merge-path bin (rows of <= 256 slots, one warp per row, in place):
 // a warp holds the next row's slots (2 vectors per lane) in registers and the row after that's

@@ -16,7 +16,6 @@
 #include "analysis.cuh"
 #include "expand.cuh"
 #include "merge.cuh"
-#include "merge_units.cuh"
 #include "merge_tiles.cuh"
 #include "merge_long.cuh"
 #include "scan.cuh"
@@ -178,15 +177,8 @@ struct spgemm_plan_s {
     int32_t *rowmn = nullptr, *rowmx = nullptr;   // exact column range per row of C (bucket mapping)
     int64_t *row_rng = nullptr;    // (rowmn, rowmx) as int2 in row_order (pipelined bucket bins)
     bool chat_external = false;
-    bool c_in_chat = false;        // C compact at the head of the Ĉ arrays (fused merge)    // Ĉ lives in the caller's C buffers (spgemm_execute, device C)
-    // merge units (merge_units.cuh): long rows merged into the side buffer, then one unit kernel
-    int64_t long_slots = 0;
-    int32_t *side_col = nullptr;
-    float *side_val = nullptr;
-    int64_t *side_off = nullptr;
-    int32_t *unit_row = nullptr;
-    int64_t *nunits = nullptr;
-    unsigned long long *unit_status = nullptr, *unit_ticket = nullptr;
+    bool c_in_chat = false;        // C compact at the head of the Ĉ arrays (tile merge)
+    unsigned long long *unit_ticket = nullptr;   // profile buffer of the merge kernels (options.reserved[1])
     // merge tiles (merge_tiles.cuh): tile table, look-back words
     TileDesc *tiles = nullptr;
     // long rows by column groups (merge_long.cuh)
@@ -201,6 +193,7 @@ struct spgemm_plan_s {
     unsigned long long *tile_status = nullptr;
     int64_t tiles_max = 0;
     unsigned long long *lbi = nullptr;   // options.reserved[8] = 1: [expansion | limited merge] x kLbiSlots
+    unsigned long long *exp_ticket = nullptr;   // block-path expansion claim counter
     int64_t nnz_c = -1;
     int state = 0;  // 1 planned, 2 expanded, 3 merged
 };
@@ -260,9 +253,9 @@ static inline unsigned grid_for(int64_t n, int threads, int64_t cap = 148 * 64) 
 
 // merge selection: default = per-bin merge + CSR compaction (merge.cuh); options.reserved[5] = 2 the
 // tile merge (merge_tiles.cuh + merge_long.cuh: C placed by look-back at the head of the Ĉ arrays, no
-// compaction); reserved[0] = 4 the fused unit merge (merge_units.cuh)
-static inline bool use_tile_merge(const spgemm_options_t &o) { return o.reserved[0] == 0 && o.reserved[5] == 2; }
-static inline bool c_in_place(const spgemm_options_t &o) { return use_tile_merge(o) || o.reserved[0] == kMergeFused; }
+// compaction)
+static inline bool use_tile_merge(const spgemm_options_t &o) { return o.reserved[5] == 2; }
+static inline bool c_in_place(const spgemm_options_t &o) { return use_tile_merge(o); }
 
 // Large-smem kernels: opt-in shared memory size and resident blocks per SM, queried once per
 // (kernel, device, smem, threads) -- these runtime calls cost host microseconds on every step.
@@ -323,12 +316,12 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
 }
 
 // software-pipelined in-place bucket bin over rows [b0, b1) of row_order (meta table in p->row_meta)
-template <int NW, int GROUPS, int EPT, bool WALK = false>
+template <int NW, int GROUPS, int EPT>
 static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int64_t cnt, const char *name,
                               int ctas_per_sm) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, 0>::kBytes * GROUPS;
-    auto kern = k_merge_bucket_pipe<NW, GROUPS, EPT, 0, WALK>;
+    auto kern = k_merge_bucket_pipe<NW, GROUPS, EPT, 0>;
     int occ = 0;
     TRY(kernel_occupancy((const void *)kern, smem, NW * 32 * GROUPS, &occ));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
@@ -339,44 +332,17 @@ static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int6
     return SPGEMM_OK;
 }
 
-// merged rows go to the side buffer (long rows) when `side`, else in place
+// merged rows are written in place at the head of their Ĉ bucket
 template <int NW, int GROUPS, int EPT, int LS = 0>
 static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name,
-                             int ctas_per_sm, bool fallback_list = true, bool side = false) {
+                             int ctas_per_sm, bool fallback_list = true) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, LS>::kBytes * GROUPS;
     TRY(kernel_occupancy((const void *)k_merge_bucket<NW, GROUPS, EPT, LS>, smem, 0, nullptr));
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * ctas_per_sm * 4);
     LAUNCH(name, s, k_merge_bucket<NW, GROUPS, EPT, LS><<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
         rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count, 0,
-        side ? p->side_off : nullptr, side ? p->side_col : nullptr, side ? p->side_val : nullptr, p->rowmn, p->rowmx));
-    return SPGEMM_OK;
-}
-
-template <int GROUPS, int VPT>
-static int launch_wcs_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name) {
-    if (cnt == 0) return SPGEMM_OK;
-    const int smem = WcsSmem<VPT>::kBytes * GROUPS;
-    auto kern = k_merge_wcs<GROUPS, VPT>;
-    int occ = 0;
-    TRY(kernel_occupancy((const void *)kern, smem, 32 * GROUPS, &occ));
-    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
-    LAUNCH(name, s, kern<<<(unsigned)grid, 32 * GROUPS, smem, s>>>(rows, cnt, p->rowoff, p->rowwork, p->chat_col,
-                                                                  p->chat_val, p->ccount, nullptr, nullptr, nullptr));
-    return SPGEMM_OK;
-}
-
-template <int NW, int GROUPS, int CAP>
-static int launch_wmp_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *rows, int64_t cnt, const char *name) {
-    if (cnt == 0) return SPGEMM_OK;
-    const int smem = WmpSmem<CAP>::kBytes * GROUPS;
-    auto kern = k_merge_wmp<NW, GROUPS, CAP>;
-    int occ = 0;
-    TRY(kernel_occupancy((const void *)kern, smem, NW * 32 * GROUPS, &occ));
-    const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
-    LAUNCH(name, s, kern<<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(rows, cnt, p->rowoff, p->rowwork, p->chat_col,
-                                                                       p->chat_val, p->ccount, nullptr, nullptr,
-                                                                       nullptr));
+        nullptr, nullptr, nullptr, p->rowmn, p->rowmx));
     return SPGEMM_OK;
 }
 
@@ -442,16 +408,25 @@ static int check_csx(int64_t nseg, int64_t other, int64_t nnz, const void *ptr, 
     return SPGEMM_OK;
 }
 
-static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t *B, cudaStream_t s);
+static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t *B, cudaStream_t s, int64_t r0,
+                     int64_t r1);
 
 int spgemm_plan(const spgemm_csc_t *A, const spgemm_csr_t *B, const spgemm_options_t *opt, void *stream,
                 spgemm_plan_t *out) {
+    if (!A) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "A or B is NULL");
+    return spgemm_plan_rows(A, B, 0, A->nrows, opt, stream, out);
+}
+
+int spgemm_plan_rows(const spgemm_csc_t *A, const spgemm_csr_t *B, int64_t row_begin, int64_t row_end,
+                     const spgemm_options_t *opt, void *stream, spgemm_plan_t *out) {
     if (!out) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan out-pointer is NULL");
     *out = nullptr;
     if (!A || !B) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "A or B is NULL");
     TRY(check_csx(A->ncols, A->nrows, A->nnz, A->colptr, A->rowidx, A->val, A->where, "A"));
     TRY(check_csx(B->nrows, B->ncols, B->nnz, B->rowptr, B->colidx, B->val, B->where, "B"));
     if (A->ncols != B->nrows) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "A.ncols != B.nrows");
+    if (row_begin < 0 || row_end < row_begin || row_end > A->nrows)
+        return fail(SPGEMM_ERR_INVALID_ARGUMENT, "bad row window");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) return fail(SPGEMM_ERR_NO_DEVICE, "no CUDA device");
     spgemm_plan_s *p = new spgemm_plan_s();
@@ -465,7 +440,7 @@ int spgemm_plan(const spgemm_csc_t *A, const spgemm_csr_t *B, const spgemm_optio
     if (p->opt.split_b_tile <= 0) p->opt.split_b_tile = d.split_b_tile;
     p->opt.split_b_tile = (int32_t)pad_run(p->opt.split_b_tile);   // R4: whole 16-byte vectors
     if (p->opt.limit_ctas_per_sm <= 0) p->opt.limit_ctas_per_sm = d.limit_ctas_per_sm;
-    int r = plan_impl(p, A, B, (cudaStream_t)stream);
+    int r = plan_impl(p, A, B, (cudaStream_t)stream, row_begin, row_end);
     if (r != SPGEMM_OK) {
         std::string keep = g_err;
         spgemm_destroy(p);
@@ -488,7 +463,8 @@ static int upload(spgemm_plan_s *p, const void *src, int64_t bytes, int32_t wher
     return SPGEMM_OK;
 }
 
-static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t *B, cudaStream_t s) {
+static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t *B, cudaStream_t s, int64_t r0,
+                     int64_t r1) {
     CK(cudaGetDevice(&p->dev));
     CK(cudaDeviceGetAttribute(&p->num_sms, cudaDevAttrMultiProcessorCount, p->dev));
     p->pool = pool_for_device(p->dev);
@@ -499,7 +475,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     p->n = B->ncols;
     p->nnz_a = A->nnz;
     p->nnz_b = B->nnz;
-    const int64_t M = p->m, K = p->k;
+    int64_t M = p->m;
+    const int64_t K = p->k;
     TRY(upload(p, A->colptr, (K + 1) * 8, A->where, (const void **)&p->a_colptr, s));
     TRY(upload(p, A->rowidx, p->nnz_a * 4, A->where, (const void **)&p->a_rowidx, s));
     TRY(upload(p, A->val, p->nnz_a * 4, A->where, (const void **)&p->a_val, s));
@@ -528,6 +505,35 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         CK(cudaMemcpyAsync(&hs, p->scal, sizeof(hs), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
         if (hs.invalid) return fail(SPGEMM_ERR_INVALID_INPUT, "malformed indices (range / order) in A or B");
+    }
+
+    // ---- row window (spgemm_plan_rows): A' = rows [r0, r1) of A, packed on the device -----
+    if (r0 != 0 || r1 != A->nrows) {
+        int64_t *lo, *cnt, *nptr;
+        TRY(palloc(p, &lo, K, s));
+        TRY(palloc(p, &cnt, K, s));
+        TRY(palloc(p, &nptr, K + 1, s));
+        if (K > 0)
+            LAUNCH("row_window", s, k_window_count<<<grid_for(K, 256), 256, 0, s>>>(p->a_colptr, p->a_rowidx, K,
+                                                                                    (int32_t)r0, (int32_t)r1, lo, cnt));
+        TRY(scan_excl(p, cnt, K, nptr, s, "row_window"));
+        int64_t nnz_w = 0;
+        CK(cudaMemcpyAsync(&nnz_w, nptr + K, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));   // (the window's nnz sizes every A-entry array below)
+        int32_t *widx;
+        float *wval;
+        TRY(palloc(p, &widx, nnz_w, s));
+        TRY(palloc(p, &wval, nnz_w, s));
+        if (K > 0 && nnz_w > 0)
+            LAUNCH("row_window", s, k_window_copy<<<grid_for(K * 32, 256), 256, 0, s>>>(lo, nptr, K, p->a_rowidx,
+                                                                                       p->a_val, (int32_t)r0, widx,
+                                                                                       wval));
+        p->a_colptr = nptr;
+        p->a_rowidx = widx;
+        p->a_val = wval;
+        p->m = r1 - r0;
+        p->nnz_a = nnz_w;
+        M = p->m;
     }
 
     // ---- stage (1): workload analysis -------------------------------------------------
@@ -742,34 +748,12 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         }
     }
     // merge state; Ĉ itself is allocated by spgemm_expand (or is the caller's C, spgemm_execute)
-    const bool fused = p->opt.reserved[0] == kMergeFused;
-    p->long_slots = fused ? (int64_t)p->h_scal.long_slots : 0;
-    TRY(palloc(p, &p->side_col, p->long_slots, s));
-    TRY(palloc(p, &p->side_val, p->long_slots, s));
-    TRY(palloc(p, &p->side_off, M + 1, s));
-    TRY(palloc(p, &p->unit_row, M + 1, s));
-    TRY(palloc(p, &p->nunits, 1, s));
-    TRY(palloc(p, &p->unit_status, M + 1, s));
-    TRY(palloc(p, &p->unit_ticket, 18, s));
-    if (M > 0 && fused) {
-        Temp tf(s), tl(s), tu(s);
-        int32_t *flag;
-        int64_t *longcap, *uoff;
-        TRY(talloc(p, tf, &flag, M));
-        TRY(talloc(p, tl, &longcap, M));
-        TRY(talloc(p, tu, &uoff, M + 1));
-        LAUNCH("units", s, k_unit_flags<<<grid_for(M, 256), 256, 0, s>>>(p->rowoff, p->row_cls, M, kUnitThreads, flag,
-                                                                          longcap));
-        TRY(scan_excl(p, longcap, M, p->side_off, s, "units"));
-        TRY(scan_excl(p, flag, M, uoff, s, "units"));
-        LAUNCH("units", s, k_unit_rows<<<grid_for(M, 256), 256, 0, s>>>(flag, uoff, M, p->unit_row, p->nunits));
-    } else {
-        CK(cudaMemsetAsync(p->nunits, 0, 8, s));
-    }
+    TRY(palloc(p, &p->unit_ticket, 18, s));   // [2, 18): per-phase / per-path profile (tuning)
     TRY(palloc(p, &p->ccount, M, s));
     TRY(palloc(p, &p->fb_rows, M, s));
     TRY(palloc(p, &p->fb_count, 1, s));
     TRY(palloc(p, &p->crowptr, M + 1, s));
+    TRY(palloc(p, &p->exp_ticket, 1, s));
     if (p->opt.reserved[8] == 1) {   // LBI recording (Eq. (3))
         TRY(palloc(p, &p->lbi, 2 * kLbiSlots, s));
         CK(cudaMemsetAsync(p->lbi, 0, 2 * kLbiSlots * 8, s));
@@ -810,9 +794,20 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
     } else if (p->n_pieces_all > 0) {
         // (measured: an L2 persistence window over B' -- half of L2 set aside -- made the
         // expansion 1.34 -> 2.10 ms and the compaction 1.14 -> 1.48 ms on C2; not used)
-        LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
-            p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
-            p->base, p->chat_col, p->chat_val, p->lbi));
+        // block path (split pieces + whole Normal blocks, TMA-staged B' tiles) unless disabled
+        // (options.reserved[9] = 1: every block through the flat unit kernel)
+        const int64_t nblk = p->opt.reserved[9] == 1 ? 0 : p->n_split_pieces + p->n_whole;
+        if (nblk > 0) {
+            CK(cudaMemsetAsync(p->exp_ticket, 0, 8, s));
+            TRY(kernel_occupancy((const void *)k_expand_blocks, kExpBlkSmem, kExpBlkThreads, nullptr));
+            LAUNCH("expand_blocks", s, k_expand_blocks<<<(unsigned)p->num_sms * 3, kExpBlkThreads, kExpBlkSmem, s>>>(
+                p->pieces, nblk, p->b_rowptr, p->bp_col, p->bp_val, p->a_val, p->base, p->chat_col, p->chat_val,
+                p->exp_ticket, p->lbi));
+        }
+        if (nblk < p->n_pieces_all)
+            LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
+                p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
+                p->base, p->chat_col, p->chat_val, p->lbi, p->piece_uoff + nblk));
     }
     p->state = 2;
     return SPGEMM_OK;
@@ -820,7 +815,7 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
 
 static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     const int64_t M = p->m;
-    if (M > 0 && p->opt.reserved[0] != 7) {
+    if (M > 0) {
         if (!p->row_meta) TRY(palloc(p, &p->row_meta, M, s));
         if (p->rowmn && !p->row_rng) TRY(palloc(p, &p->row_rng, M, s));
         LAUNCH("merge_meta", s, k_row_meta<<<grid_for(M, 256), 256, 0, s>>>(p->row_order, M, p->rowoff, p->rowwork,
@@ -841,34 +836,12 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         LAUNCH("merge_warp", s, k_merge_warp<<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
             rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount, nullptr, nullptr, nullptr));
     CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
-    // merge_variant (options.reserved[0], tuning): 0 default (warp merge-path natural merge sort
-    // for the <= 256 bin, per-row bucket sort for the <= 4096 bins, software-pipelined for <= 1024),
-    // 1 register-staged counting sort for the <= 256 / <= 1024 bins, 2 bucket sort everywhere,
-    // 3 merge-path everywhere, 4 fused unit merge (merge_units.cuh), 6 register bitonic for
-    // <= 256, 7 no pipelining, 8 pipelined <= 4096 bins too
-    const int variant = p->opt.reserved[0];
-    if (variant == 6) {
-        // register bitonic, 2 / 4 / 8 slots per lane (measured slower than the merge-path warp:
-        // C4 2.24 vs 2.11 ms, C2's <= 256 bin 0.80 vs 0.37 ms -- latency-bound, one row per warp)
-        rows = rows_of(kRowBucketWarp64, kRowBucketWarp64 + 1, &cnt);
-        if (cnt > 0)
-            LAUNCH("merge_warp64", s, k_merge_warpE<2><<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
-                rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
-        rows = rows_of(kRowBucketWarp128, kRowBucketWarp128 + 1, &cnt);
-        if (cnt > 0)
-            LAUNCH("merge_warp128", s, k_merge_warpE<4><<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
-                rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
-        rows = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &cnt);
-        if (cnt > 0)
-            LAUNCH("merge_warp256", s, k_merge_warpE<8><<<(unsigned)cdiv(cnt * 32, 256), 256, 0, s>>>(
-                rows, cnt, p->rowoff, p->chat_col, p->chat_val, p->ccount));
-    }
+    // <= 256 slots: software-pipelined warp merge path; <= 1024: pipelined per-row bucket sort;
+    // <= 4096: per-row bucket sort (8 / 16 warps).  (The slower alternatives measured in round 1 --
+    // register-staged counting sort, bucket sort or merge path everywhere, register bitonic, the
+    // bucket-owner walk, the fused unit merge -- were removed in round 2.)
     rows = rows_of(kRowBucketWarp64, kRowBucketSort256 + 1, &cnt);   // 32 < slots <= 256
-    if (variant == 6) {
-    } else if (variant == 1) TRY(launch_wcs_bin<4, 2>(p, s, rows, cnt, "merge_wcs256"));
-    else if (variant == 2) TRY(launch_bucket_bin<1, 8, 8>(p, s, rows, cnt, "merge_bucket256", 8));
-    else if (variant == 7) TRY(launch_wmp_bin<1, 8, 256>(p, s, rows, cnt, "merge_wmp256"));
-    else if (cnt > 0) {   // software-pipelined warp merge path
+    if (cnt > 0) {
         constexpr int G = 8;
         const int smem = WmpSmem<256>::kBytes * G;
         int occ = 0;
@@ -878,47 +851,16 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         LAUNCH("merge_wmp256", s, k_merge_wmp_pipe<G><<<(unsigned)grid, 32 * G, smem, s>>>(
             p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount));
     }
-    if (variant == 1) {
-        rows = rows_of(kRowBucketSort512, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_wcs_bin<1, 8>(p, s, rows, cnt, "merge_wcs1k"));
-    } else if (variant == 3) {
-        rows = rows_of(kRowBucketSort512, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_wmp_bin<1, 4, 1024>(p, s, rows, cnt, "merge_wmp1k"));
-    } else if (variant == 7) {
-        rows = rows_of(kRowBucketSort512, kRowBucketSort512 + 1, &cnt);
-        TRY(launch_bucket_bin<2, 4, 8>(p, s, rows, cnt, "merge_bucket512", 8));
-        rows = rows_of(kRowBucketSort1K, kRowBucketSort1K + 1, &cnt);
-        TRY(launch_bucket_bin<4, 2, 8>(p, s, rows, cnt, "merge_bucket1k", 8));
-    } else if (variant == 10) {   // bucket-owner insertion sort + walk reduction
-        const int64_t q = p->row_starts[kRowBucketSort512];
-        TRY(launch_bucket_pipe<2, 4, 8, true>(p, s, q, p->row_starts[kRowBucketSort512 + 1] - q, "merge_bucket512", 8));
-        const int64_t q2 = p->row_starts[kRowBucketSort1K];
-        TRY(launch_bucket_pipe<4, 2, 8, true>(p, s, q2, p->row_starts[kRowBucketSort1K + 1] - q2, "merge_bucket1k", 8));
-    } else {
+    {
         const int64_t q = p->row_starts[kRowBucketSort512];
         TRY(launch_bucket_pipe<2, 4, 8>(p, s, q, p->row_starts[kRowBucketSort512 + 1] - q, "merge_bucket512", 8));
         const int64_t q2 = p->row_starts[kRowBucketSort1K];
         TRY(launch_bucket_pipe<4, 2, 8>(p, s, q2, p->row_starts[kRowBucketSort1K + 1] - q2, "merge_bucket1k", 8));
     }
-    if (variant == 3) {
-        rows = rows_of(kRowBucketSort2K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_wmp_bin<4, 1, 4096>(p, s, rows, cnt, "merge_wmp4k"));
-    } else if (variant == 7) {
-        rows = rows_of(kRowBucketSort2K, kRowBucketSort2K + 1, &cnt);
-        TRY(launch_bucket_bin<8, 1, 8>(p, s, rows, cnt, "merge_bucket2k", 8));
-        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
-    } else if (variant == 8) {   // pipelined 2K / 4K bins (measured: 0.88 / 0.53 ms vs 0.85 / 0.50 unpipelined)
-        const int64_t q = p->row_starts[kRowBucketSort2K];
-        TRY(launch_bucket_pipe<8, 1, 8>(p, s, q, p->row_starts[kRowBucketSort2K + 1] - q, "merge_bucket2k", 8));
-        const int64_t q2 = p->row_starts[kRowBucketSort4K];
-        TRY(launch_bucket_pipe<16, 1, 8>(p, s, q2, p->row_starts[kRowBucketSort4K + 1] - q2, "merge_bucket4k", 4));
-    } else {
-        rows = rows_of(kRowBucketSort2K, kRowBucketSort2K + 1, &cnt);
-        TRY(launch_bucket_bin<8, 1, 8>(p, s, rows, cnt, "merge_bucket2k", 8));
-        rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-        TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
-    }
+    rows = rows_of(kRowBucketSort2K, kRowBucketSort2K + 1, &cnt);
+    TRY(launch_bucket_bin<8, 1, 8>(p, s, rows, cnt, "merge_bucket2k", 8));
+    rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+    TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
@@ -1097,100 +1039,6 @@ static int merge_tiles_path(spgemm_plan_s *p, cudaStream_t s) {
     return SPGEMM_OK;
 }
 
-static int merge_fused(spgemm_plan_s *p, cudaStream_t s) {
-    const int64_t M = p->m;
-    if (M > 0) CK(cudaMemsetAsync(p->ccount, 0, M * 8, s));
-    auto rows_of = [&](int b0, int b1, int64_t *cnt) {
-        *cnt = p->row_starts[b1] - p->row_starts[b0];
-        return p->row_order + p->row_starts[b0];
-    };
-    int64_t cnt;
-    CK(cudaMemsetAsync(p->fb_count, 0, sizeof(unsigned), s));
-    // (a) long rows (padded bucket > kUnitRowMax, or B-Limited), merged into the side buffer:
-    //     <= 4096 slots by a 16-warp bucket-sort block per row; the limited rows B-Limited
-    const int32_t *rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
-    TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_long4k", 4, true, true));
-    {   // rows whose buckets overflowed: natural merge sort (count read on the device)
-        constexpr int CAP = 4096;
-        const int smem = SortSmem<CAP>::kBytes;
-        TRY(kernel_occupancy((const void *)k_merge_rows<8, 1, CAP>, smem, 0, nullptr));
-        LAUNCH("merge_fallback", s, k_merge_rows<8, 1, CAP><<<(unsigned)p->num_sms * 2, 256, smem, s>>>(
-            p->fb_rows, 0, p->rowoff, p->rowwork, p->chat_col, p->chat_val, p->ccount, p->fb_count, p->side_off,
-            p->side_col, p->side_val));
-    }
-    if (p->nlim > 0) {
-        CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
-        LimitedArgs g;
-        g.rows = p->row_order + p->row_starts[kRowBucketLim0];
-        g.nrows = p->nlim;
-        g.rowoff = p->rowoff;
-        g.rowwork = p->rowwork;
-        g.run_start = p->run_start;
-        g.run_base = p->run_base;
-        g.run_len = p->run_len;
-        g.chat_col = p->chat_col;
-        g.chat_val = p->chat_val;
-        g.ccount = p->ccount;
-        g.scratch_cursor = p->scr_cursor;
-        g.scratch_cnt = p->scr_cnt;
-        g.scratch_col = p->scr_col;
-        g.scratch_val = p->scr_val;
-        g.max_deg = p->lim_max_deg;
-        g.stage_cap = p->stage_cap;
-        g.row_counter = p->row_counter;
-        g.out_col = p->side_col;
-        g.out_val = p->side_val;
-        g.out_off = p->side_off;
-        g.skip_small = 1;
-        g.prof = p->opt.reserved[1] == 3 ? p->unit_ticket + 2 : nullptr;
-        if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
-        g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
-        g.lbi = p->lbi ? p->lbi + kLbiSlots : nullptr;
-        // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
-        // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
-        TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false, true));
-        TRY(kernel_occupancy((const void *)k_merge_limited, kLimSmem, 0, nullptr));
-        LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
-    }
-    // (b) every unit of short rows (and the long rows' copies), in row order, straight into C
-    if (M > 0) {
-        CK(cudaMemsetAsync(p->unit_status, 0, (M + 1) * 8, s));
-        CK(cudaMemsetAsync(p->unit_ticket, 0, 18 * 8, s));
-        UnitArgs ua;
-        ua.unit_row = p->unit_row;
-        ua.nunits = p->nunits;
-        ua.rowoff = p->rowoff;
-        ua.rowwork = p->rowwork;
-        ua.rcls = p->row_cls;
-        ua.chat_col = p->chat_col;
-        ua.chat_val = p->chat_val;
-        ua.side_col = p->side_col;
-        ua.side_val = p->side_val;
-        ua.side_off = p->side_off;
-        ua.ccount = p->ccount;
-        ua.crowptr = p->crowptr;
-        ua.M = M;
-        ua.status = p->unit_status;
-        ua.ticket = p->unit_ticket;
-        ua.n_fallback = p->unit_ticket + 1;
-        ua.debug = p->opt.reserved[1];
-        ua.prof = p->unit_ticket + 2;
-        constexpr int smem = UnitSmem<kUnitThreads>::kBytes;
-        int occ = 0;
-        TRY(kernel_occupancy((const void *)k_merge_units<kUnitThreads>, smem, kUnitThreads, &occ));
-        LAUNCH("merge_units", s, k_merge_units<kUnitThreads><<<(unsigned)(p->num_sms * std::max(occ, 1)), kUnitThreads,
-                                                                 smem, s>>>(ua));
-        const int64_t nlong = p->row_starts[kRowBucketEmpty] - p->row_starts[kRowBucketSort4K];
-        if (nlong > 0)
-            LAUNCH("merge_copy_long", s, k_copy_long<<<grid_for(nlong, 1, (int64_t)p->num_sms * 8), kCopyThreads, 0, s>>>(
-                p->row_order + p->row_starts[kRowBucketSort4K], nlong, p->crowptr, p->ccount, p->side_off, p->side_col,
-                p->side_val, p->chat_col, p->chat_val));
-    } else {
-        CK(cudaMemsetAsync(p->crowptr, 0, 8, s));
-    }
-    return SPGEMM_OK;
-}
-
 int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     if (!p) return fail(SPGEMM_ERR_INVALID_ARGUMENT, "plan is NULL");
     if (p->state < 2) return fail(SPGEMM_ERR_STATE, "spgemm_merge before spgemm_expand");
@@ -1201,7 +1049,6 @@ int spgemm_merge(spgemm_plan_t p, void *stream, int64_t *nnz_c) {
     const int64_t M = p->m;
     p->c_in_chat = c_in_place(p->opt);
     if (use_tile_merge(p->opt)) TRY(merge_tiles_path(p, s));
-    else if (p->opt.reserved[0] == kMergeFused) TRY(merge_fused(p, s));
     else TRY(merge_bins(p, s));
     CK(cudaMemcpyAsync(&p->nnz_c, p->crowptr + M, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
@@ -1223,7 +1070,7 @@ int spgemm_output(spgemm_plan_t p, spgemm_csr_out_t *C, void *stream) {
     C->nnz = p->nnz_c;
     const int64_t nnz = p->nnz_c;
     if (p->c_in_chat) {
-        // tile / fused merge: C is compact at the head of the Ĉ arrays (merge_tiles.cuh, merge_units.cuh)
+        // tile merge: C is compact at the head of the Ĉ arrays (merge_tiles.cuh)
         const cudaMemcpyKind kind = C->where == SPGEMM_HOST ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
         CK(cudaMemcpyAsync(C->rowptr, p->crowptr, (p->m + 1) * 8, kind, s));
         if (nnz > 0 && C->colidx != p->chat_col) {
@@ -1337,11 +1184,9 @@ int spgemm_get_stats(spgemm_plan_t p, spgemm_stats_t *st) {
     st->n_rows_bin[5] = p->nlim;
     st->bytes_workspace = p->bytes;
     st->n_units = st->n_units_fallback = -1;
-    if (p->state >= 3 && p->m > 0 && p->c_in_chat) {
-        unsigned long long t[2];
-        CK(cudaMemcpy(&st->n_units, p->nunits, 8, cudaMemcpyDeviceToHost));
-        CK(cudaMemcpy(t, p->unit_ticket, 16, cudaMemcpyDeviceToHost));
-        st->n_units_fallback = (int64_t)t[1];
+    if (p->state >= 3 && p->m > 0 && p->tiles) {   // tile merge: number of tiles walked
+        CK(cudaMemcpy(&st->n_units, p->tile_base + cdiv(p->m, kTileRowChunk), 8, cudaMemcpyDeviceToHost));
+        st->n_units_fallback = 0;
     }
     return SPGEMM_OK;
 }

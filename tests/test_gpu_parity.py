@@ -66,28 +66,21 @@ def _deg(inp):
     return d
 
 
-FUSED = dict(reserved=(4,) + (0,) * 15)   # merge variant: fused unit merge + look-back output
 TILES = dict(reserved=(0, 0, 0, 0, 0, 2) + (0,) * 10)   # tile merge (merge_tiles.cuh, merge_long.cuh)
 TILES_INPLACE = dict(reserved=(0, 0, 0, 0, 0, 2, 1) + (0,) * 9)   # tile merge, legacy long rows
 
 CASES = [
     ("C1", dict()),
-    ("C1", FUSED),
-    ("C1", dict(beta=10.0, **FUSED)),
-    ("C1", dict(reserved=(1,) + (0,) * 15)),   # merge variant: register-staged counting sort
-    ("C1", dict(reserved=(2,) + (0,) * 15)),   # merge variant: smem bucket sort everywhere
-    ("C1", dict(reserved=(3,) + (0,) * 15)),   # merge variant: merge-path everywhere
-    ("C1", dict(reserved=(6,) + (0,) * 15)),   # merge variant: register bitonic for <= 256 slots
-    ("C1", dict(reserved=(7,) + (0,) * 15)),   # merge variant: bucket bins without pipelining
-    ("C1", dict(reserved=(8,) + (0,) * 15)),   # merge variant: all bucket bins pipelined
-    ("C1", dict(reserved=(10,) + (0,) * 15)),  # merge variant: bucket-owner insertion sort
     ("C1", dict(reserved=(0, 0, 0, 1) + (0,) * 12)),   # row-product expansion (comparison order)
+    ("C1", dict(reserved=(0, 0, 1) + (0,) * 13)),      # per-row compaction kernels
+    ("C1", dict(reserved=(0, 0, 0, 0, 1) + (0,) * 11)),   # no per-row column range from the plan
     ("C1", dict(enable_gather=0)),
     ("C1", dict(enable_split=0)),
     ("C1", dict(piece_work=300, split_b_tile=37, split_ca_max=5)),
     ("C1", dict(alpha=2.0)),
     ("C1", dict(beta=10.0)),
     ("C1", dict(beta=10.0, enable_limit=0)),
+    ("C1", dict(reserved=(0,) * 9 + (1,) + (0,) * 6)),   # expansion: every block through the flat kernel
     ("C1", dict(reserved=(0,) * 7 + (4,) + (0,) * 8)),   # fixed splitting factor 4 (Fig. 11 sweep)
     ("C1", dict(reserved=(0,) * 7 + (64,) + (0,) * 8)),
     ("C1", TILES),
@@ -196,7 +189,7 @@ def _rows_sorted(m, rowoff, cols, vals):
 
 
 EXPAND_CASES = [c for c in CASES if not c[1] or {"enable_gather", "enable_split", "piece_work"} & set(c[1])
-                or c[1].get("reserved", (0,) * 4)[3] == 1]
+                or c[1].get("reserved", (0,) * 16)[3] == 1 or c[1].get("reserved", (0,) * 16)[9] == 1]
 
 
 @pytest.mark.parametrize("name,opts", EXPAND_CASES)
@@ -252,10 +245,8 @@ def test_c_matches_oracle(name, opts):
 def test_random_tiny(shape, dens, seed, skew, values):
     inp = synth.random_tiny(*shape, dens[0], dens[1], seed, values=values, skew=skew)
     A, B = spg.from_inputs(inp, "cuda")
-    for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(1,) + (0,) * 15),
-                 dict(reserved=(2,) + (0,) * 15), dict(reserved=(3,) + (0,) * 15), FUSED, dict(reserved=(6,) + (0,) * 15),
-                 dict(reserved=(10,) + (0,) * 15), TILES, dict(beta=1000.0, **TILES),
-                 dict(beta=1000.0, piece_work=64, split_ca_max=3, **FUSED)):
+    for opts in (dict(), dict(beta=1000.0, piece_work=64, split_ca_max=3), dict(reserved=(0, 0, 1) + (0,) * 13),
+                 TILES, dict(beta=1000.0, **TILES), dict(beta=1000.0, piece_work=64, split_ca_max=3, **TILES)):
         C = spg.matmul(A, B, **opts)
         assert_c_matches(C, inp, signed=(values == "signed"))
 
@@ -292,12 +283,12 @@ def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False,
     (16, 100, 30000, 0.3, 2000, False, False),     # dense rows: fp64 column windows
     (2, 10000, 1000000, 1.0, 21, True, False),     # column 0 in 10000 runs: single-column overflow
 ])
-@pytest.mark.parametrize("fused", [False, True, "tiles", "tiles_inplace"])
+@pytest.mark.parametrize("fused", [False, "tiles", "tiles_inplace"])
 def test_limited_paths(m, k, n, dens, run_len, hub, narrow, fused):
     """B-Limited merge: rows longer than the non-limited capacity, through every sub-path."""
     inp = _wide_inputs(m, k, n, dens, run_len, 3, hub_col=hub, narrow=narrow)
     A, B = spg.from_inputs(inp, "cuda")
-    opts = {False: {}, True: FUSED, "tiles": TILES, "tiles_inplace": TILES_INPLACE}[fused]
+    opts = {False: {}, "tiles": TILES, "tiles_inplace": TILES_INPLACE}[fused]
     with spg.Plan(A, B, **opts) as p:
         st = p.stats()
         assert st["n_rows_bin"][5] > 0
@@ -315,7 +306,8 @@ def test_limited_paths(m, k, n, dens, run_len, hub, narrow, fused):
 @pytest.mark.parametrize("k,cluster,spread", [(10, 20, 10), (40, 40, 60), (60, 100, 2)])
 def test_clustered_columns_fallback(k, cluster, spread):
     """Rows whose columns cluster in a narrow range of a wide span overflow the bucket sort's
-    buckets; the natural merge sort fallback (and the limited kernel's inline fallback) take them."""
+    buckets; the natural merge sort fallback (and the limited kernel's inline fallback) take them;
+    the tile merge ranks the crowded buckets."""
     rng = np.random.default_rng(5)
     m, n = 6, 1_000_000
     ar, ac = np.nonzero(np.ones((m, k), dtype=bool))
@@ -332,11 +324,7 @@ def test_clustered_columns_fallback(k, cluster, spread):
     A, B = spg.from_inputs(inp, "cuda")
     C = spg.matmul(A, B)
     assert_c_matches(C, inp)
-    with spg.Plan(A, B, **FUSED) as p:
-        C = p.execute()
-        if k * (cluster + spread) <= 2048:           # short rows: the unit merge's fallback ran
-            assert p.stats()["n_units_fallback"] > 0
-    assert_c_matches(C, inp)
+    assert_c_matches(spg.matmul(A, B, **TILES), inp)
 
 
 def test_row_partition_and_row_blocks():
@@ -520,3 +508,35 @@ def test_lbi_recording():
     for name in ("expand", "merge_limited"):
         assert lb[name] is not None, name
         assert 0.0 < lb[name]["lbi"] <= 1.0 and lb[name]["max_ms"] > 0
+
+
+@pytest.mark.parametrize("ca,rb", [(1, 6000), (3, 6000), (2, 4097), (40, 1)])
+def test_expansion_block_shapes(ca, rb):
+    """The block-path expansion (TMA-staged B' tiles): a Normal block whose B row exceeds one
+    shared-memory buffer (1 x 6000: sub-tiles), a split Dominator with B tiles, a row one past a
+    tile, and thin blocks -- Ĉ against Eq. (2) through the full C."""
+    rng = np.random.default_rng(ca * 7 + rb)
+    ar = np.arange(ca, dtype=np.int32)
+    ac = np.zeros(ca, dtype=np.int32)
+    bc = np.sort(rng.choice(10 * rb + 10, rb, replace=False)).astype(np.int32)
+    br = np.zeros(rb, dtype=np.int32)
+    inp = synth.from_coo("blk", ca, 1, 10 * rb + 10, (ar, ac, synth.edge_values(ar, ac, 1)),
+                         (br, bc, synth.edge_values(br, bc, 2)))
+    A, B = spg.from_inputs(inp, "cuda")
+    for opts in ({}, dict(reserved=(0,) * 9 + (1,) + (0,) * 6), dict(split_b_tile=1000)):
+        assert_c_matches(spg.matmul(A, B, **opts), inp)
+
+
+@pytest.mark.parametrize("r0,r1", [(0, 1024), (0, 1), (100, 300), (512, 512), (1000, 1024), (7, 1021)])
+def test_row_window_plan(r0, r1):
+    """spgemm_plan_rows: rows [r0, r1) of C (A windowed on the GPU, no copy by the caller) equal the
+    oracle's rows [r0, r1) -- the chunked expansion and multi-GPU row blocks (R8)."""
+    inp = synth.make_inputs("C1", seed=3)
+    A, B = spg.from_inputs(inp, "cuda")
+    C = spg.matmul(A, B, rows=(r0, r1))
+    rows = np.arange(r0, r1, dtype=np.int32)
+    orp, ocol, oval = oracle.gustavson(inp, rows=rows) if r1 > r0 else (np.zeros(1, np.int64), [], np.zeros(0))
+    np.testing.assert_array_equal(C.rowptr.cpu().numpy(), orp)
+    np.testing.assert_array_equal(C.colidx.cpu().numpy(), ocol)
+    got = C.val.cpu().numpy().astype(np.float64)
+    assert np.all(np.abs(got - oval) <= RTOL * np.abs(oval))
