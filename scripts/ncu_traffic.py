@@ -26,7 +26,12 @@ def main(rep, config):
     hdr, units, data = rows[0], rows[1], rows[2:]
     ki = hdr.index("Kernel Name")
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9}
-    out = {"report": rep, "config": config, "groups": {}, "kernels": []}
+    out = {"report": rep, "config": config, "groups": {}, "kernels": [],
+           "step": "launches from the first k_pair_work up to (not including) the next one: one bench step"}
+    names = [d[ki].split("(")[0] for d in data]
+    starts = [q for q, nm in enumerate(names) if nm.split("::")[-1].startswith("k_pair_work")]
+    if starts:
+        data = data[starts[0]:starts[1]] if len(starts) > 1 else data[starts[0]:]
     for d in data:
         name = d[ki].split("(")[0]
         b = 0.0
@@ -52,7 +57,8 @@ def main(rep, config):
                     pass
         out["kernels"].append(rec)
         for g, pre in GROUPS.items():
-            if any(name.split("<")[0].split()[-1].startswith(p) for p in pre):
+            base = name.split("<")[0].split()[-1].split("::")[-1]
+            if any(base.startswith(p) for p in pre):
                 e = out["groups"].setdefault(g, {"dram_bytes": 0, "ms": 0.0, "launches": 0})
                 e["dram_bytes"] += int(b)
                 e["ms"] += ms
