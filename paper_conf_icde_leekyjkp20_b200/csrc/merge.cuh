@@ -497,12 +497,11 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
         }
     }
     g.sync();
-    // 4. coalesced copy of the merged row (out_col == NULL: the caller copies dk / dv [0, U) itself)
-    if (out_col)
-        for (int q = g.gtid; q < U; q += T) {
-            out_col[q] = dk[q];
-            out_val[q] = dv[q];
-        }
+    // 4. coalesced copy of the merged row
+    for (int q = g.gtid; q < U; q += T) {
+        out_col[q] = dk[q];
+        out_val[q] = dv[q];
+    }
     return U;
 }
 
@@ -905,12 +904,7 @@ constexpr int kLimNW = kLimThreads / 32;
 constexpr int kLimEPT = kLimCap / kLimThreads;
 constexpr int kLimBucketCap = 9216;               // rows up to this were merged by the bucket launch
 constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
-// coarse groups of <= kHalfCap products are sorted two at a time, one per 512-thread half of the
-// block (named barriers), each in its own half of the sorter memory
-constexpr int kHalfNW = kLimNW / 2;
-constexpr int kHalfCap = kHalfNW * 32 * kLimEPT;   // 4608
-constexpr int kHalfBytes = kHalfCap * 16 + (hidx(ceil_pow2(kHalfCap)) + 4) * 4;
-constexpr int kLimSortBytes = cmax3(cmax3(SortSmem<kLimCap>::kBytes, 0, 2 * kHalfBytes),   // fallback / halves
+constexpr int kLimSortBytes = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
                                     kLimCap * 16 + (hidx(ceil_pow2(kLimCap)) + 4) * 4,  // bucket sort
                                     kLimWindow * 8 + (kLimWindow / 32) * 4);   // dense window
 constexpr int kCoarseLog = 10;
@@ -1053,9 +1047,11 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
                 const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
 #pragma unroll
-                for (int u = 0; u < 4; ++u)   // (one shared atomic per product: MATCH.ANY, ~63 SM-cycles
-                    if (cc[u] != kKeyPad)      //  per warp on B200, cost more than it saved)
-                        atomicAdd(&fh[(cc[u] - mn) >> kLimWinLog], 1);
+                for (int u = 0; u < 4; ++u) {
+                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> kLimWinLog;
+                    const unsigned peers = __match_any_sync(__activemask(), wid);
+                    if (wid >= 0 && lane_id() == __ffs(peers) - 1) atomicAdd(&fh[wid], __popc(peers));
+                }
             }
             __syncthreads();
             {
@@ -1080,9 +1076,15 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
                 const float vv[4] = {v4.x, v4.y, v4.z, v4.w};
 #pragma unroll
-                for (int u = 0; u < 4; ++u) {     // cursor bump per product (order inside a window is free)
-                    if (cc[u] != kKeyPad) {
-                        const int q = atomicAdd(&wcur[(cc[u] - mn) >> kLimWinLog], 1);
+                for (int u = 0; u < 4; ++u) {     // warp-aggregated cursor bumps per window
+                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> kLimWinLog;
+                    const unsigned peers = __match_any_sync(__activemask(), wid);
+                    if (wid >= 0) {
+                        const int leader = __ffs(peers) - 1;
+                        int q0 = 0;
+                        if (lane_id() == leader) q0 = atomicAdd(&wcur[wid], __popc(peers));
+                        q0 = __shfl_sync(peers, q0, leader);
+                        const int q = q0 + __popc(peers & lanemask_lt());
                         sc_col[q] = cc[u];
                         sc_val[q] = vv[u];
                     }
@@ -1245,10 +1247,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     // (fewer, fuller sorts: C3 182 -> 159 ms; 7/8: same speed), else 1/2, so rows
                     // with one heavy column range still take this path (C5: 3/4 alone sent them to
                     // the window path, limited merge 86 -> 115 ms)
-                    // rows whose bins are all small take groups of < kHalfCap (sorted in pairs by the two
-                    // halves of the block)
-                    const int T = mxb <= kHalfCap / 8 ? kHalfCap - kHalfCap / 8
-                                  : (mxb <= kLimCap / 4 ? kLimCap * 3 / 4 : kLimCap / 2);
+                    const int T = mxb <= kLimCap / 4 ? kLimCap * 3 / 4 : kLimCap / 2;
 #pragma unroll
                     for (int u = 0; u < BPT; ++u) {
                         fh[threadIdx.x * BPT + u] = ex / T;     // group id of the bin
@@ -1290,9 +1289,15 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                         const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
                         const float vv[4] = {v4.x, v4.y, v4.z, v4.w};
 #pragma unroll
-                        for (int u = 0; u < 4; ++u) {     // cursor bump per product (a group is sorted anyway;
-                            if (cc[u] != kKeyPad) {        //  MATCH.ANY costs ~63 SM-cycles per warp on B200)
-                                const int q = atomicAdd(&gcur[fh[(cc[u] - mn) >> shc]], 1);
+                        for (int u = 0; u < 4; ++u) {     // warp-aggregated cursor bumps per group
+                            const int gid = cc[u] == kKeyPad ? -1 - lane_id() : fh[(cc[u] - mn) >> shc];
+                            const unsigned peers = __match_any_sync(__activemask(), gid);
+                            if (gid >= 0) {
+                                const int leader = __ffs(peers) - 1;
+                                int q0 = 0;
+                                if (lane_id() == leader) q0 = atomicAdd(&gcur[gid], __popc(peers));
+                                q0 = __shfl_sync(peers, q0, leader);
+                                const int q = q0 + __popc(peers & lanemask_lt());
                                 sc_col[q] = cc[u];
                                 sc_val[q] = vv[u];
                             }
@@ -1300,40 +1305,9 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     }
                     __syncthreads();
                     sub(11);   // scatter into scratch
-                    __shared__ int sch[2][2 * kHalfNW + 2], s_hu[2];
-                    const Group<kHalfNW, 2> hg;
                     for (int gi = 0; gi < ng; ++gi) {
                         const int g0 = gstart[gi], n = gstart[gi + 1] - g0;
                         if (n == 0) continue;
-                        if (gi + 1 < ng && n <= kHalfCap && gstart[gi + 2] - gstart[gi + 1] <= kHalfCap) {
-                            // two groups at once: half h sorts group gi + h into its half of the memory
-                            const int a0 = gstart[gi + hg.gid], na = gstart[gi + hg.gid + 1] - a0;
-                            unsigned char *hs = smem_raw + (size_t)hg.gid * kHalfBytes;
-                            int Uh = 0;
-                            if (na > 0)
-                                Uh = bucket_sort_reduce<kHalfNW, 2, kLimEPT, 0, true>(
-                                    hg, sc_col + a0, sc_val + a0, na, (int32_t *)hs, (float *)(hs + kHalfCap * 4),
-                                    (int32_t *)(hs + kHalfCap * 8), (float *)(hs + kHalfCap * 12),
-                                    (int *)(hs + kHalfCap * 16), nullptr, nullptr, sch[hg.gid]);
-                            if (hg.gtid == 0) s_hu[hg.gid] = Uh;
-                            __syncthreads();
-                            const int U0 = s_hu[0], U1 = s_hu[1];
-                            if (U0 >= 0 && U1 >= 0) {   // copy both merged groups out, in order
-                                const int32_t *k0h = (const int32_t *)smem_raw;
-                                const float *v0h = (const float *)(smem_raw + kHalfCap * 4);
-                                const int32_t *k1h = (const int32_t *)(smem_raw + kHalfBytes);
-                                const float *v1h = (const float *)(smem_raw + kHalfBytes + kHalfCap * 4);
-                                for (int q = threadIdx.x; q < U0 + U1; q += kLimThreads) {
-                                    oc[nout + q] = q < U0 ? k0h[q] : k1h[q - U0];
-                                    ov[nout + q] = q < U0 ? v0h[q] : v1h[q - U0];
-                                }
-                                nout += U0 + U1;
-                                __syncthreads();
-                                ++gi;
-                                continue;
-                            }
-                            // (a bucket overflowed: both groups again, one after the other, below)
-                        }
                         int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(
                             grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + kLimCap * 4),
                             (int32_t *)(smem_raw + kLimCap * 8), (float *)(smem_raw + kLimCap * 12),
