@@ -19,7 +19,7 @@ from typing import Optional
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libspgemm.so")
+LIB_PATH = os.environ.get("SPGEMM_LIB") or os.path.join(_HERE, "libspgemm.so")   # (override: A/B builds)
 
 SPGEMM_DEVICE, SPGEMM_HOST = 0, 1
 VIEW_WORK, VIEW_ROWWORK, VIEW_ROWOFF, VIEW_PAIR_CLASS, VIEW_PIECES, VIEW_GATHER, VIEW_ROW_CLASS, \

@@ -10,7 +10,7 @@ SO = os.path.join(HERE, "libspgemm.so")
 MAIN = os.path.join(HERE, "csrc", "spgemm.cu")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",
-         "-Xcompiler", "-fPIC", "-shared"]
+         "-Xcompiler", "-fPIC", "-shared"] + os.environ.get("SPGEMM_NVCC_EXTRA", "").split()
 
 
 def sources():

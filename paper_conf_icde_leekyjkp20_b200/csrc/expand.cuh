@@ -215,8 +215,11 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
 // every A entry e of the block is written as one run Ĉ[base[e] + b_off ..) = (cols, a_e * vals):
 // groups of W = min(32, 2^ceil(log2 nv)) lanes take an A entry each and stride over its vectors
 // -- two 16-byte stores per 4 products, no per-unit search, division or global B' load.
+#ifndef EXP_BLK_VEC
+#define EXP_BLK_VEC 1024
+#endif
 constexpr int kExpBlkThreads = 256;
-constexpr int kExpBlkVec = 1024;   // max vectors of one B tile (split_b_tile <= 4096)
+constexpr int kExpBlkVec = EXP_BLK_VEC;   // vectors of one B' buffer (longer B tiles: sub-tiles)
 constexpr int kExpBlkSmem = 2 * 2 * kExpBlkVec * 16;   // 2 buffers x (cols, vals) = 64 KB
 
 __device__ __forceinline__ void exp_mbar_init(uint64_t *mbar) {

@@ -799,8 +799,9 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
         const int64_t nblk = p->opt.reserved[9] == 1 ? 0 : p->n_split_pieces + p->n_whole;
         if (nblk > 0) {
             CK(cudaMemsetAsync(p->exp_ticket, 0, 8, s));
-            TRY(kernel_occupancy((const void *)k_expand_blocks, kExpBlkSmem, kExpBlkThreads, nullptr));
-            LAUNCH("expand_blocks", s, k_expand_blocks<<<(unsigned)p->num_sms * 3, kExpBlkThreads, kExpBlkSmem, s>>>(
+            int occ = 0;
+            TRY(kernel_occupancy((const void *)k_expand_blocks, kExpBlkSmem, kExpBlkThreads, &occ));
+            LAUNCH("expand_blocks", s, k_expand_blocks<<<(unsigned)(p->num_sms * std::max(occ, 1)), kExpBlkThreads, kExpBlkSmem, s>>>(
                 p->pieces, nblk, p->b_rowptr, p->bp_col, p->bp_val, p->a_val, p->base, p->chat_col, p->chat_val,
                 p->exp_ticket, p->lbi));
         }

@@ -78,3 +78,24 @@ def test_two_ranks_one_gpu_cuda_path(name):
     status, info = q.get(timeout=10)
     assert status == "ok", info
     assert info[0] == 0 and 0 < info[1] < info[2]
+
+
+def test_bench_two_ranks_share_gpu():
+    """bench.py --gpus 2 (re-launching itself under torch.distributed.run) with both ranks on this
+    B200 (SPGEMM_BENCH_SHARE_GPU: gloo instead of NCCL): rank 0 prints one JSON line with n_gpus 2,
+    the per-rank step times, the C gather timing and the e2e leg."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SPGEMM_BENCH_SHARE_GPU="1")
+    env.pop("WORLD_SIZE", None)
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--config", "C1",
+                          "--steps", "2", "--warmup", "1", "--no-cpu-baseline"], capture_output=True, text=True,
+                         timeout=900, cwd=root, env=env)
+    assert out.returncode == 0, out.stderr[-3000:]
+    line = [ln for ln in out.stdout.splitlines() if ln.startswith("{")][-1]
+    d = json.loads(line)
+    assert d["n_gpus"] == 2 and len(d["rank_ms_per_step"]) == 2 and d["value"] > 0
+    assert d["c_gather"]["ms"] > 0 and d["e2e"]["value"] > 0
+    assert d["config"]["products"] > 0 and d["config"]["m"] == 1024
