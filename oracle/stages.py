@@ -105,9 +105,9 @@ def split_pieces(inp, cls, piece_work: int, b_tile: int, split_ca_max: int, fixe
     ("several elements from each column vector are shifted to the next vector
     sequentially", L374-L376 L); empty trailing pieces are not emitted (Fig. 5: a
     25-computation block split into three blocks, L386-L388 L).  The B row is cut
-    into tiles of b_tile entries (rounded up to a multiple of 4) only when it exceeds
-    b_tile (R4)."""
-    b_tile = -(-b_tile // 4) * 4   # R4: a tile is whole 16-byte vectors (4 slots) of the run
+    into tiles of b_tile entries (rounded up to a multiple of 8) only when it exceeds
+    b_tile (R4, R16)."""
+    b_tile = -(-b_tile // 8) * 8   # R4 / R16: a tile is whole 32-byte sectors (8 slots) of the run
     out = []
     for k in np.nonzero(cls == DOMINATOR)[0]:
         a0, a1 = int(inp.a_colptr[k]), int(inp.a_colptr[k + 1])

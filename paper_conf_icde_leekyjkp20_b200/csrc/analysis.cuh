@@ -34,9 +34,12 @@ constexpr int kRowBucketLim0 = 9;      // 9 + (39 - floor(log2 L)): longest rows
 constexpr int kRowBucketEmpty = 49;
 constexpr int kNumRowBuckets = 50;
 constexpr int kWarpRowMax = 32;
-// Ĉ runs are padded to multiples of kRunAlign slots (16 B) with sentinel entries
-// (col = INT32_MAX, val = 0) so that every run starts 16-byte aligned (vector stores).
-constexpr int kRunAlign = 4;
+// Ĉ runs are padded to multiples of kRunAlign slots (32 B: one DRAM sector of columns and one of
+// values) with sentinel entries (col = INT32_MAX, val = 0), so that every run starts 16-byte
+// aligned (vector stores, bulk copies) and no 32-byte sector is shared by two runs -- two runs of
+// a row are written by different blocks at different times, and a sector written half by each
+// used to cost a read-modify-write in DRAM (R16).
+constexpr int kRunAlign = 8;
 __host__ __device__ __forceinline__ int64_t pad_run(int64_t x) { return (x + kRunAlign - 1) & ~(int64_t)(kRunAlign - 1); }
 constexpr int kSort256Max = 256;
 constexpr int kSort512Max = 512;
@@ -393,7 +396,9 @@ __global__ void k_piece_whole(const int32_t *__restrict__ list, int64_t n, const
 // B' (B with rows padded to 4 slots) row k starts at bp_start(b_rowptr[k], k) = b_rowptr[k] + 7k
 // rounded up to 4 slots: 16-byte aligned and clear of row k + 1 (row k ends by b_rowptr[k+1] + 7k + 6)
 // without a scan over the padded lengths; B' holds nnz(B) + 7K + 4 slots.
-__host__ __device__ __forceinline__ int64_t bp_start(int64_t rp, int64_t k) { return (rp + 7 * k + 3) & ~(int64_t)3; }
+__host__ __device__ __forceinline__ int64_t bp_start(int64_t rp, int64_t k) {
+    return (rp + (2 * kRunAlign - 1) * k + kRunAlign - 1) & ~(int64_t)(kRunAlign - 1);
+}
 
 // Merge row classes.  Limited rows (L > t_lim, L452-L477 L) get B-Limited merge blocks;
 // a row made of a single run (one A entry) is already sorted and duplicate-free.

@@ -33,7 +33,7 @@ constexpr int kExpCtasPerSM = 3;   // 80 registers: 3 x 256 threads resident per
 
 // vectors of one run written by a block: the B sub-row rounded up to 4 slots (B tiles start on
 // 4-slot boundaries, so the last tile of a row also writes the run's sentinel padding)
-__device__ __forceinline__ int piece_nvec(const Piece &pc) { return (pc.b_len + 3) >> 2; }
+__device__ __forceinline__ int piece_nvec(const Piece &pc) { return (int)(pad_run(pc.b_len) >> 2); }
 
 __global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64_t *__restrict__ units) {
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
@@ -42,7 +42,7 @@ __global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64
     }
 }
 
-// B' = B with every row padded to a multiple of 4 slots (col = INT32_MAX, val = 0), 16-byte
+// B' = B with every row padded to a multiple of kRunAlign slots (col = INT32_MAX, val = 0), 16-byte
 // stores.  Lane per row for rows of <= 64 entries; the warp's longer rows (hub rows of thousands
 // of entries) are then copied by the whole warp, one after another (a thread per row alone left
 // AB18's 100K-entry rows on one thread: 1.2 ms).
@@ -71,14 +71,14 @@ __global__ void k_pad_b(const int64_t *__restrict__ b_rowptr, const int32_t *__r
         if (k < K) { b0 = b_rowptr[k]; rb = b_rowptr[k + 1] - b0; }
         const bool lng = rb > 64;
         if (!lng)
-            for (int64_t j = 0; j < rb; j += 4) pad_b_vec(b_colidx, b_val, b0, rb, bp_start(b0, k), j, bp_col, bp_val);
+            for (int64_t j = 0; j < pad_run(rb); j += 4) pad_b_vec(b_colidx, b_val, b0, rb, bp_start(b0, k), j, bp_col, bp_val);
         unsigned m = __ballot_sync(0xffffffffu, lng);
         while (m) {
             const int l = __ffs(m) - 1;
             m &= m - 1;
             const int64_t kl = kb + l;
             const int64_t bl = __shfl_sync(0xffffffffu, b0, l), rl = __shfl_sync(0xffffffffu, rb, l);
-            for (int64_t j = 4 * lane; j < rl; j += 128) pad_b_vec(b_colidx, b_val, bl, rl, bp_start(bl, kl), j, bp_col, bp_val);
+            for (int64_t j = 4 * lane; j < pad_run(rl); j += 128) pad_b_vec(b_colidx, b_val, bl, rl, bp_start(bl, kl), j, bp_col, bp_val);
         }
     }
 }
@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
 // groups of W = min(32, 2^ceil(log2 nv)) lanes take an A entry each and stride over its vectors
 // -- two 16-byte stores per 4 products, no per-unit search, division or global B' load.
 #ifndef EXP_BLK_VEC
-#define EXP_BLK_VEC 1024
+#define EXP_BLK_VEC 512
 #endif
 constexpr int kExpBlkThreads = 256;
 constexpr int kExpBlkVec = EXP_BLK_VEC;   // vectors of one B' buffer (longer B tiles: sub-tiles)
@@ -394,7 +394,7 @@ __global__ void __launch_bounds__(256) k_expand_rows(const int64_t *__restrict__
                 const int64_t e = list_e[q];
                 const int32_t k = list_k[q];
                 const int64_t b0 = __ldg(b_rowptr + k);
-                nv = (int)((__ldg(b_rowptr + k + 1) - b0 + 3) >> 2);
+                nv = (int)(pad_run(__ldg(b_rowptr + k + 1) - b0) >> 2);
                 src = bp_start(b0, k);
                 dst = base[e];
                 av = a_val[e];

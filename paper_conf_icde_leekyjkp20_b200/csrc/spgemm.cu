@@ -438,7 +438,7 @@ int spgemm_plan_rows(const spgemm_csc_t *A, const spgemm_csr_t *B, int64_t row_b
     if (p->opt.split_ca_max <= 0) p->opt.split_ca_max = d.split_ca_max;
     if (p->opt.piece_work <= 0) p->opt.piece_work = d.piece_work;
     if (p->opt.split_b_tile <= 0) p->opt.split_b_tile = d.split_b_tile;
-    p->opt.split_b_tile = (int32_t)pad_run(p->opt.split_b_tile);   // R4: whole 16-byte vectors
+    p->opt.split_b_tile = (int32_t)pad_run(p->opt.split_b_tile);   // R4: whole 32-byte sectors (8 slots)
     if (p->opt.limit_ctas_per_sm <= 0) p->opt.limit_ctas_per_sm = d.limit_ctas_per_sm;
     int r = plan_impl(p, A, B, (cudaStream_t)stream, row_begin, row_end);
     if (r != SPGEMM_OK) {
@@ -673,7 +673,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     }
     // B' = B with rows padded to 4 slots (16-byte aligned vector loads in the expansion)
     {   // one allocation: cols then values
-        const int64_t nbp = (p->nnz_b + 7 * K + 4 + 63) & ~(int64_t)63;
+        const int64_t nbp = (p->nnz_b + (2 * kRunAlign - 1) * K + kRunAlign + 63) & ~(int64_t)63;   // (bp_start)
         TRY(palloc(p, &p->bp_col, 2 * nbp, s));
         p->bp_val = (float *)(p->bp_col + nbp);
         p->bp_bytes = (size_t)(2 * nbp) * 4;

@@ -43,7 +43,9 @@ def run(A, B, reps, **opts):
         lbis.append(lb)
     med = {nm: statistics.median(v[1:]) for nm, v in times.items()}
     lb = lbis[-1]
-    return {"expand_ms": round(med.get("expand", 0.0), 4),
+    return {"expand_ms": round(med.get("expand", 0.0) + med.get("expand_blocks", 0.0), 4),
+            "long_partition_ms": round(med.get("merge_long_partition", 0.0), 4),
+            "tiles_ms": round(med.get("merge_tiles", 0.0), 4),
             "merge_limited_ms": round(sum(v for k, v in med.items() if k.startswith("merge_limited")), 4),
             "step_kernels_ms": round(sum(med.values()), 4),
             "lbi_expand": lb["expand"] and round(lb["expand"]["lbi"], 4),
@@ -67,6 +69,11 @@ def main():
     for cap in [1, 2, 3]:
         r = run(A, B, args.reps, limit_ctas_per_sm=cap)
         print(json.dumps({"sweep": "limit_ctas_per_sm", "config": args.config, "cap": cap, **r}), flush=True)
+    tiles = (0,) * 5 + (2,) + (0,) * 10   # tile merge: the long-row partition kernel's residency
+    for cap in [1, 2]:
+        r = run(A, B, args.reps, limit_ctas_per_sm=cap, reserved=tiles)
+        print(json.dumps({"sweep": "limit_ctas_per_sm (tile merge)", "config": args.config, "cap": cap, **r}),
+              flush=True)
     for beta in [10.0, 0.0]:
         r = run(A, B, args.reps, beta=beta)
         print(json.dumps({"sweep": "beta", "config": args.config, "beta": beta, **r}), flush=True)

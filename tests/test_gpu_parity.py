@@ -49,12 +49,12 @@ PAD_KEY = 0x7FFFFFFF
 
 
 def _caps(inp):
-    """Padded Ĉ bucket length of every row: runs rounded up to 4 slots (16-byte alignment of the
-    kernel's vector stores); not method arithmetic, the layout of the buffer."""
+    """Padded Ĉ bucket length of every row: runs rounded up to 8 slots (32-byte sectors, DESIGN.md
+    §4, R16); not method arithmetic, the layout of the buffer."""
     ca, rb, _ = stages.pair_workload(inp)
     col_of = np.repeat(np.arange(inp.k), ca)
     cap = np.zeros(inp.m, dtype=np.int64)
-    np.add.at(cap, inp.a_rowidx.astype(np.int64), (rb[col_of] + 3) // 4 * 4)
+    np.add.at(cap, inp.a_rowidx.astype(np.int64), (rb[col_of] + 7) // 8 * 8)
     return cap
 
 
