@@ -136,7 +136,10 @@ typedef struct {
                                      (merged in place, then moved) instead of column groups;
                                  [7] > 0: fixed B-Splitting factor for every Dominator (the
                                      Fig. 11 sweep; capped at the column's power of two);
-                                 [8] 1 = record per-SM busy times for the LBI (SPGEMM_VIEW_LBI) */
+                                 [8] 1 = record per-SM busy times for the LBI (SPGEMM_VIEW_LBI);
+                                 [9] expansion mapping: 0 block path + a run per thread for the
+                                     gathered Low performers, 1 every block one vector per thread
+                                     (round 1), 2 block path + a vector per thread               */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */

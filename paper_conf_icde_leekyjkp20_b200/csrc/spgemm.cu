@@ -151,6 +151,8 @@ struct spgemm_plan_s {
     Piece *pieces = nullptr;       // split pieces, whole Normal blocks, gathered Low-performer blocks
     int64_t *piece_uoff = nullptr; // unit (16-byte vector) prefix over pieces
     int64_t *tile_p0 = nullptr;    // first piece of every expansion tile
+    int64_t *piece_eoff = nullptr; // A-entry prefix over pieces (run-per-thread expansion)
+    int64_t *tile_e0 = nullptr;    // first piece of every run tile
     int64_t n_low = 0, n_pieces_all = 0;
     // B' (rows padded to 4 slots, row k at bp_start(b_rowptr[k], k)): cols, values
     int32_t *bp_col = nullptr;
@@ -656,20 +658,28 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_low, 256), 256, 0, s>>>(
             p->pair_order + g_lo, p->n_low, p->a_colptr, p->b_rowptr, p->pieces + p->n_split_pieces + p->n_whole));
     TRY(palloc(p, &p->piece_uoff, p->n_pieces_all + 1, s));
+    TRY(palloc(p, &p->piece_eoff, p->n_pieces_all + 1, s));
     if (p->n_pieces_all > 0) {
-        Temp tu(s);
-        int64_t *units;
+        Temp tu(s), ta(s);
+        int64_t *units, *alen;
         TRY(talloc(p, tu, &units, p->n_pieces_all));
+        TRY(talloc(p, ta, &alen, p->n_pieces_all));
         LAUNCH("piece_units", s, k_piece_units<<<grid_for(p->n_pieces_all, 256), 256, 0, s>>>(
-            p->pieces, p->n_pieces_all, units));
+            p->pieces, p->n_pieces_all, units, alen));
         TRY(scan_excl(p, units, p->n_pieces_all, p->piece_uoff, s, "piece_scan"));
-        // (units <= nnz(Ĉ)/4 + #pieces; the tile map is sized for that bound, no host sync)
+        TRY(scan_excl(p, alen, p->n_pieces_all, p->piece_eoff, s, "piece_scan"));
+        // (units <= nnz(Ĉ)/4 + #pieces and A entries <= units; the tile maps are sized for that
+        // bound, no host sync)
         const int64_t ntiles_max = cdiv(p->chat_cap / 4 + p->n_pieces_all, kExpTile);
         TRY(palloc(p, &p->tile_p0, ntiles_max + 1, s));
+        TRY(palloc(p, &p->tile_e0, ntiles_max + 1, s));
         LAUNCH("piece_scan", s, k_tile_first_piece<<<grid_for(ntiles_max + 1, 256), 256, 0, s>>>(
             p->piece_uoff, p->n_pieces_all, ntiles_max, p->tile_p0));
+        LAUNCH("piece_scan", s, k_tile_first_piece<<<grid_for(ntiles_max + 1, 256), 256, 0, s>>>(
+            p->piece_eoff, p->n_pieces_all, ntiles_max, p->tile_e0));
     } else {
         CK(cudaMemsetAsync(p->piece_uoff, 0, 8, s));
+        CK(cudaMemsetAsync(p->piece_eoff, 0, 8, s));
     }
     // B' = B with rows padded to 4 slots (16-byte aligned vector loads in the expansion)
     {   // one allocation: cols then values
@@ -795,7 +805,7 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
         // (measured: an L2 persistence window over B' -- half of L2 set aside -- made the
         // expansion 1.34 -> 2.10 ms and the compaction 1.14 -> 1.48 ms on C2; not used)
         // block path (split pieces + whole Normal blocks, TMA-staged B' tiles) unless disabled
-        // (options.reserved[9] = 1: every block through the flat unit kernel)
+        // (options.reserved[9] = 1: every block through the flat unit kernel, round 1's mapping)
         const int64_t nblk = p->opt.reserved[9] == 1 ? 0 : p->n_split_pieces + p->n_whole;
         if (nblk > 0) {
             CK(cudaMemsetAsync(p->exp_ticket, 0, 8, s));
@@ -805,8 +815,14 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
                 p->pieces, nblk, p->b_rowptr, p->bp_col, p->bp_val, p->a_val, p->base, p->chat_col, p->chat_val,
                 p->exp_ticket, p->lbi));
         }
-        if (nblk < p->n_pieces_all)
-            LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
+        // the gathered Low performers: a run per thread (options.reserved[9] = 2: a vector per
+        // thread, the round-1 unit mapping)
+        if (nblk < p->n_pieces_all && p->opt.reserved[9] == 0)
+            LAUNCH("expand", s, k_expand_flat<true><<<(unsigned)p->num_sms * 5, kExpThreads, 0, s>>>(
+                p->pieces, p->piece_eoff, p->n_pieces_all, p->tile_e0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
+                p->base, p->chat_col, p->chat_val, p->lbi, p->piece_eoff + nblk));
+        else if (nblk < p->n_pieces_all)
+            LAUNCH("expand", s, k_expand_flat<false><<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
                 p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
                 p->base, p->chat_col, p->chat_val, p->lbi, p->piece_uoff + nblk));
     }

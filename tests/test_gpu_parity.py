@@ -81,6 +81,7 @@ CASES = [
     ("C1", dict(beta=10.0)),
     ("C1", dict(beta=10.0, enable_limit=0)),
     ("C1", dict(reserved=(0,) * 9 + (1,) + (0,) * 6)),   # expansion: every block through the flat kernel
+    ("C1", dict(reserved=(0,) * 9 + (2,) + (0,) * 6)),   # expansion: Low performers a vector per thread
     ("C1", dict(reserved=(0,) * 7 + (4,) + (0,) * 8)),   # fixed splitting factor 4 (Fig. 11 sweep)
     ("C1", dict(reserved=(0,) * 7 + (64,) + (0,) * 8)),
     ("C1", TILES),
@@ -189,7 +190,7 @@ def _rows_sorted(m, rowoff, cols, vals):
 
 
 EXPAND_CASES = [c for c in CASES if not c[1] or {"enable_gather", "enable_split", "piece_work"} & set(c[1])
-                or c[1].get("reserved", (0,) * 16)[3] == 1 or c[1].get("reserved", (0,) * 16)[9] == 1]
+                or c[1].get("reserved", (0,) * 16)[3] == 1 or c[1].get("reserved", (0,) * 16)[9] != 0]
 
 
 @pytest.mark.parametrize("name,opts", EXPAND_CASES)
