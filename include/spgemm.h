@@ -109,7 +109,12 @@ typedef struct {
     int32_t split_b_tile;     /* max B-row entries per piece (default 4096)                     */
     double beta;              /* >0: limiting threshold min(cap, nnz(Ĉ)/(#rows × β)) (L475-L477 L);
                                  0: B200 default = non-limited merge capacity (4096)            */
-    int32_t limit_ctas_per_sm;/* B-Limiting: resident limited-merge blocks per SM (default 1)   */
+    int32_t limit_ctas_per_sm;/* B-Limiting (PAPER.md L463-L469 L, Fig. 14): resident limited-
+                                 merge blocks per SM, 1 / 2 / 4 = blocks of 1024 / 512 / 256
+                                 threads sorting column groups of <= 9216 / 4096 / 2048
+                                 products (other values round down to these; default 1).  With
+                                 2 or 4, rows with a column range too heavy for the smaller
+                                 sorter are deferred to a second launch at 1 per SM.        */
     int32_t enable_split;     /* ablation switches (Fig. 10): 0 disables the technique; for
                                  enable_limit = 0 the β threshold is ignored and only rows above
                                  the non-limited kernels' capacity take the long-row kernels     */
@@ -137,9 +142,9 @@ typedef struct {
                                  [7] > 0: fixed B-Splitting factor for every Dominator (the
                                      Fig. 11 sweep; capped at the column's power of two);
                                  [8] 1 = record per-SM busy times for the LBI (SPGEMM_VIEW_LBI);
-                                 [9] expansion mapping: 0 block path + a run per thread for the
-                                     gathered Low performers, 1 every block one vector per thread
-                                     (round 1), 2 block path + a vector per thread               */
+                                 [9] expansion mapping: 0 block path (split pieces + Normal blocks,
+                                     TMA-staged) + a 16-byte vector per thread for the gathered
+                                     Low performers, 1 every block a vector per thread (round 1) */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */

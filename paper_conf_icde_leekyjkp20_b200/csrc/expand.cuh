@@ -35,12 +35,10 @@ constexpr int kExpCtasPerSM = 3;   // 80 registers: 3 x 256 threads resident per
 // 4-slot boundaries, so the last tile of a row also writes the run's sentinel padding)
 __device__ __forceinline__ int piece_nvec(const Piece &pc) { return (int)(pad_run(pc.b_len) >> 2); }
 
-__global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64_t *__restrict__ units,
-                              int64_t *__restrict__ alen) {
+__global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64_t *__restrict__ units) {
     for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < n; q += (int64_t)gridDim.x * blockDim.x) {
         const Piece pc = pieces[q];
         units[q] = (int64_t)pc.a_len * piece_nvec(pc);
-        alen[q] = pc.a_len;
     }
 }
 
@@ -118,10 +116,6 @@ __device__ __forceinline__ int64_t div_units(int64_t r, int nv) {
 // searches the block list in global memory instead.
 constexpr int kExpPieceCache = 1024;
 
-// RUNS = true (the gathered Low performers: runs of <= 32 products): a unit is a whole run (one A
-// entry of a block, nv <= 8 vectors) instead of one vector -- no per-vector search or division;
-// uoff / tile_p0 are then the prefix of the blocks' A lengths and its tile map.
-template <bool RUNS>
 __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
     const Piece *__restrict__ pieces, const int64_t *__restrict__ uoff, int64_t npieces,
     const int64_t *__restrict__ tile_p0, const int64_t *__restrict__ b_rowptr, const int32_t *__restrict__ bp_col,
@@ -191,22 +185,6 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
                     nv = piece_nvec(pc); boff = pc.b_off;
                 }
                 const int64_t r = f - uo;
-                if constexpr (RUNS) {   // the whole run of A entry alo + r: nv (<= 8) vector pairs
-                    const int64_t e = alo + r;
-                    const float a = __ldg(a_val + e);
-                    const int64_t d0 = __ldg(base + e) + boff;
-                    ok[u] = false;
-#pragma unroll
-                    for (int v = 0; v < 8; ++v)
-                        if (v < nv) {
-                            const int4 cc = __ldg(reinterpret_cast<const int4 *>(bp_col + bsrc + 4 * v));
-                            const float4 ww = __ldg(reinterpret_cast<const float4 *>(bp_val + bsrc + 4 * v));
-                            __stcs(reinterpret_cast<int4 *>(chat_col + d0 + 4 * v), cc);
-                            __stcs(reinterpret_cast<float4 *>(chat_val + d0 + 4 * v),
-                                   make_float4(a * ww.x, a * ww.y, a * ww.z, a * ww.w));
-                        }
-                    continue;
-                }
                 const int64_t a = div_units(r, nv);
                 const int v = (int)(r - a * nv);
                 const int64_t e = alo + a;

@@ -374,10 +374,12 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
         g.reduce_minmax(mn, mx, sc);
     }
     const uint32_t span = (uint32_t)(mx - mn);
-    const int lognb = nextpow2_log(L) + LS;
+    // (>= 64 buckets: sh <= 25, so a key's in-bucket bits and its 7-bit atomic rank fit 32 bits)
+    const int lognb = max(6, nextpow2_log(L) + LS);
     const int nb = 1 << lognb;
     const int bits = span ? 32 - __clz(span) : 0;
     const int sh = max(0, bits - lognb);
+    const uint32_t lowmask = (1u << sh) - 1u;
     // PRECLEAR > 0: the caller zeroed hist[0, PRECLEAR] (and the previous row cleared it after its
     // ranking), so the row starts with its atomics -- one barrier less per row
     if constexpr (PRECLEAR == 0) {
@@ -419,40 +421,37 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
     }
     if (g.gtid == 0) hist[hidx(nb)] = tot;
     g.sync();
-    // 1. scatter: bucket start + atomic rank (unordered inside a bucket)
+    // 1. scatter: bucket start + atomic rank (unordered inside a bucket).  What is scattered is the
+    //    element's in-bucket sort code c = (key's low sh bits) << 7 | atomic rank: the keys of one
+    //    bucket share their high bits, so c orders them by key, ties by scatter order, and is unique
+    //    (ranks < 2^7: buckets above kBucketMax took the fallback)
     int pos[EPT];
+    uint32_t *dc = reinterpret_cast<uint32_t *>(dk);
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
         pos[e] = -1;
         if (key[e] != kKeyPad) {
             pos[e] = hist[hidx((key[e] - mn) >> sh)] + rk[e];
-            dk[pos[e]] = key[e];
+            dc[pos[e]] = ((((uint32_t)(key[e] - mn)) & lowmask) << 7) | (uint32_t)rk[e];
         }
     }
     g.sync();
-    // 2. bucket b = [hist[b], hist[b+1]).  Every element counts the keys of its bucket that sort
-    //    before it (smaller, or equal and scattered earlier) and moves to its sorted slot.
+    // 2. bucket b = [hist[b], hist[b+1]).  Every element counts the codes of its bucket below its own
+    //    (one load and one compare per key) and moves to its sorted slot.
 #pragma unroll
     for (int e = 0; e < EPT; ++e) {
         if (pos[e] >= 0) {
             const int b = (key[e] - mn) >> sh;
             const int bs = hist[hidx(b)], be = hist[hidx(b + 1)];
-            const int32_t kk = key[e];
+            const uint32_t ce = ((((uint32_t)(key[e] - mn)) & lowmask) << 7) | (uint32_t)rk[e];
             int rank = 0;
             if (be - bs > 1) {   // (a bucket of one key is already in place)
                 int q = bs;
                 if constexpr (UNR2)
-                    for (; q + 1 < be; q += 2) {
-                        const int32_t k0 = dk[q], k1 = dk[q + 1];
-                        rank += ((k0 < kk) | ((k0 == kk) & (q < pos[e]))) +
-                                ((k1 < kk) | ((k1 == kk) & (q + 1 < pos[e])));
-                    }
-                for (; q < be; ++q) {
-                    const int32_t kq = dk[q];
-                    rank += (kq < kk) | ((kq == kk) & (q < pos[e]));
-                }
+                    for (; q + 1 < be; q += 2) rank += (dc[q] < ce) + (dc[q + 1] < ce);
+                for (; q < be; ++q) rank += dc[q] < ce;
             }
-            dk2[bs + rank] = kk;
+            dk2[bs + rank] = key[e];
             dv2[bs + rank] = val[e];
         }
     }
@@ -895,22 +894,28 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
 // copied to the head of the row's bucket after the whole row has been read.
 // (measured: 256 threads / 3584 slots at 2 blocks per SM made C3's long rows 8.6x slower -- bins
 // of the coarse partition overflow the smaller sorter and fall back to the window search)
-constexpr int kLimThreads = 1024;
-constexpr int kLimCap = 9216;                     // 1 limited block per SM (B-Limiting)
-constexpr int kLimWinLog = 14;
-constexpr int kLimWindow = 1 << kLimWinLog;
-constexpr int kLimWords = kLimWindow / 32;         // touched-column bitmap words of a window
-constexpr int kLimNW = kLimThreads / 32;
-constexpr int kLimEPT = kLimCap / kLimThreads;
 constexpr int kLimBucketCap = 9216;               // rows up to this were merged by the bucket launch
 constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
-constexpr int kLimSortBytes = cmax3(SortSmem<kLimCap>::kBytes,                 // merge-path fallback
-                                    kLimCap * 16 + (hidx(ceil_pow2(kLimCap)) + 4) * 4,  // bucket sort
-                                    kLimWindow * 8 + (kLimWindow / 32) * 4);   // dense window
 constexpr int kCoarseLog = 10;
 constexpr int kCoarseBins = 1 << kCoarseLog;
-constexpr int kLimSmem = kLimSortBytes + (3 * kCoarseBins + 1) * 4;           // + coarse partition tables
-constexpr int kLimCtasPerSM = 228 * 1024 / (kLimSmem + 1024);   // B-Limiting: limited blocks resident per SM
+// B-Limiting (Fig. 14's "number of blocks per SM"): a limited merge block of NT threads sorts
+// column groups of <= NT * EPT products and takes ~1/(1024/NT) of an SM's shared memory, so
+// 1024 / NT blocks are resident per SM (options.limit_ctas_per_sm = 1, 2, 4).
+template <int NT>
+struct LimCfg {
+    static constexpr int kThreads = NT;
+    static constexpr int kNW = NT / 32;
+    static constexpr int kEPT = NT >= 1024 ? 9 : 8;
+    static constexpr int kCap = NT * kEPT;                  // 9216 / 4096 / 2048 products
+    static constexpr int kWinLog = NT >= 1024 ? 14 : (NT >= 512 ? 13 : 12);
+    static constexpr int kWindow = 1 << kWinLog;            // dense-path column window
+    static constexpr int kWords = kWindow / 32;             // touched-column bitmap words of a window
+    static constexpr int kSortBytes = cmax3(SortSmem<kCap>::kBytes,                  // merge-path fallback
+                                            kCap * 16 + (hidx(ceil_pow2(kCap)) + 4) * 4,   // bucket sort
+                                            kWindow * 8 + kWords * 4);               // dense window
+    static constexpr int kSmem = kSortBytes + (4 * kCoarseBins + 2) * 4;           // + coarse partition tables
+    static constexpr int kPerSM = 1024 / NT;
+};
 
 struct LimitedArgs {
     const int32_t *rows;          // limited rows, longest first
@@ -937,6 +942,10 @@ struct LimitedArgs {
     unsigned long long *prof;     // NULL, or per-path clock totals [0..10) (tuning)
     int64_t coarse_cap;           // rows up to this many slots take the coarse-partition path
     unsigned long long *lbi;      // NULL, or per-SM busy times (LBI, Eq. (3))
+    int32_t *defer_list;          // non-NULL: rows the coarse partition cannot take go here (row list index)
+    unsigned *defer_count;
+    const int32_t *rlist;         // non-NULL: process only these row list indices (*rlist_count of them)
+    const unsigned *rlist_count;
 };
 
 __device__ __forceinline__ void smem_add_f64(double *addr, double v) {
@@ -961,12 +970,14 @@ __device__ __forceinline__ int count_below(const int32_t *__restrict__ col, int6
     return lo - cur;
 }
 
-__global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g) {
+template <int NT>
+__global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) {
+    using C = LimCfg<NT>;
     lbi_start(g.lbi);
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ int sc[2 * kLimNW + 2];
+    __shared__ int sc[2 * C::kNW + 2];
     __shared__ int64_t row_sm;
-    const Group<kLimNW, 1> grp;
+    const Group<C::kNW, 1> grp;
     const int lane = lane_id(), w = warp_id();
     int32_t *cursor = g.scratch_cursor + (int64_t)blockIdx.x * g.max_deg;
     int32_t *cnt = g.scratch_cnt + (int64_t)blockIdx.x * g.max_deg;
@@ -975,9 +986,13 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
     while (true) {
         if (threadIdx.x == 0) row_sm = (int64_t)atomicAdd(g.row_counter, 1ull);
         __syncthreads();
-        const int64_t r = row_sm;
+        int64_t r = row_sm;
         __syncthreads();
         if (r >= g.nrows) break;
+        if (g.rlist) {
+            if (r >= (int64_t)*g.rlist_count) break;
+            r = g.rlist[r];
+        }
         const int i = g.rows[r];
         const int64_t s = g.rowoff[i];
         const int64_t cap = g.rowoff[i + 1] - s;   // padded bucket length
@@ -994,16 +1009,16 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         if (cap <= kLimBucketCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
         int32_t *const oc = g.out_col ? g.out_col + g.out_off[i] : g.chat_col + s;
         float *const ov = g.out_col ? g.out_val + g.out_off[i] : g.chat_val + s;
-        if (cap <= kLimCap) {
+        if (cap <= C::kCap) {
             int32_t *dk = (int32_t *)smem_raw;
-            float *dv = (float *)(smem_raw + kLimCap * 4);
-            int32_t *dk2 = (int32_t *)(smem_raw + kLimCap * 8);
-            float *dv2 = (float *)(smem_raw + kLimCap * 12);
-            int *hist = (int *)(smem_raw + kLimCap * 16);
-            int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
+            float *dv = (float *)(smem_raw + C::kCap * 4);
+            int32_t *dk2 = (int32_t *)(smem_raw + C::kCap * 8);
+            float *dv2 = (float *)(smem_raw + C::kCap * 12);
+            int *hist = (int *)(smem_raw + C::kCap * 16);
+            int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, true>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
                                                             dv2, hist, oc, ov, sc);
             if (U < 0)
-                U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
+                U = merge_row_in_smem<C::kNW, 1, C::kCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
                                                           oc, ov);
             if (threadIdx.x == 0) g.ccount[i] = U;
             __syncthreads();
@@ -1015,7 +1030,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         const int64_t *rbase = g.run_base + rs;
         const int32_t *rlen = g.run_len + rs;
         int32_t mn = kKeyPad, mx = 0;
-        for (int q = threadIdx.x; q < R; q += kLimThreads) {
+        for (int q = threadIdx.x; q < R; q += C::kThreads) {
             const int64_t b = rbase[q];
             mn = min(mn, g.chat_col[b]);
             mx = max(mx, g.chat_col[b + rlen[q] - 1]);
@@ -1024,38 +1039,38 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         mn = grp.reduce_min(mn, sc);
         mx = grp.reduce_max(mx, sc);
         const int64_t span = (int64_t)mx - mn + 1;
-        const int64_t nwin_dense = (span + kLimWindow - 1) / kLimWindow;
+        const int64_t nwin_dense = (span + C::kWindow - 1) / C::kWindow;
         const bool dense = L * 4 >= span && (int64_t)R * nwin_dense <= 2 * L;
         int64_t nout = 0;
-        const int64_t nwin_pow = (span + kLimWindow - 1) >> kLimWinLog;
+        const int64_t nwin_pow = (span + C::kWindow - 1) >> C::kWinLog;
         if (dense && cap <= g.stage_cap && nwin_pow <= kCoarseBins) {
-            // dense row, streamed: (1) histogram of the row's column windows (2^kLimWinLog columns),
+            // dense row, streamed: (1) histogram of the row's column windows (2^C::kWinLog columns),
             // (2) scatter into the block's scratch grouped by window, (3) per window, coalesced
             // sweep of its products into the fp64 shared accumulator + touched bits, extracted in
             // column order straight to the row's output (the row now lives in scratch).  Every
             // load is independent (the per-run cursor walk below is one dependent load per run
             // per window: C3's hub rows, 38K runs x 104 windows, took 250 ms in one block).
             const int nwin = (int)nwin_pow;
-            int *fh = (int *)(smem_raw + kLimSortBytes);       // [kCoarseBins] counts -> starts
+            int *fh = (int *)(smem_raw + C::kSortBytes);       // [kCoarseBins] counts -> starts
             int *wst = fh + kCoarseBins;                        // [kCoarseBins + 1]
             int *wcur = wst + kCoarseBins + 1;                  // [kCoarseBins]
             int32_t *sc_col = g.scratch_col + (int64_t)blockIdx.x * g.stage_cap;
             float *sc_val = g.scratch_val + (int64_t)blockIdx.x * g.stage_cap;
-            for (int t = threadIdx.x; t < kCoarseBins; t += kLimThreads) fh[t] = 0;
+            for (int t = threadIdx.x; t < kCoarseBins; t += C::kThreads) fh[t] = 0;
             __syncthreads();
-            for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+            for (int64_t p = threadIdx.x; p < (cap >> 2); p += C::kThreads) {
                 const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
                 const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
 #pragma unroll
                 for (int u = 0; u < 4; ++u) {
-                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> kLimWinLog;
+                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> C::kWinLog;
                     const unsigned peers = __match_any_sync(__activemask(), wid);
                     if (wid >= 0 && lane_id() == __ffs(peers) - 1) atomicAdd(&fh[wid], __popc(peers));
                 }
             }
             __syncthreads();
             {
-                constexpr int BPT = kCoarseBins / kLimThreads;
+                constexpr int BPT = kCoarseBins / C::kThreads;
                 int c[BPT], cnt = 0;
 #pragma unroll
                 for (int u = 0; u < BPT; ++u) { c[u] = fh[threadIdx.x * BPT + u]; cnt += c[u]; }
@@ -1070,14 +1085,14 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 if (threadIdx.x == 0) wst[kCoarseBins] = tot;
             }
             __syncthreads();
-            for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+            for (int64_t p = threadIdx.x; p < (cap >> 2); p += C::kThreads) {
                 const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
                 const float4 v4 = *reinterpret_cast<const float4 *>(g.chat_val + s + 4 * p);
                 const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
                 const float vv[4] = {v4.x, v4.y, v4.z, v4.w};
 #pragma unroll
                 for (int u = 0; u < 4; ++u) {     // warp-aggregated cursor bumps per window
-                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> kLimWinLog;
+                    const int wid = cc[u] == kKeyPad ? -1 - lane_id() : (cc[u] - mn) >> C::kWinLog;
                     const unsigned peers = __match_any_sync(__activemask(), wid);
                     if (wid >= 0) {
                         const int leader = __ffs(peers) - 1;
@@ -1091,22 +1106,22 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
             }
             double *acc = (double *)smem_raw;
-            uint32_t *bits = (uint32_t *)(smem_raw + kLimWindow * 8);
-            for (int t = threadIdx.x; t < kLimWindow; t += kLimThreads) acc[t] = 0.0;
-            for (int t = threadIdx.x; t < kLimWindow / 32; t += kLimThreads) bits[t] = 0u;
+            uint32_t *bits = (uint32_t *)(smem_raw + C::kWindow * 8);
+            for (int t = threadIdx.x; t < C::kWindow; t += C::kThreads) acc[t] = 0.0;
+            for (int t = threadIdx.x; t < C::kWindow / 32; t += C::kThreads) bits[t] = 0u;
             __syncthreads();
             for (int wi = 0; wi < nwin; ++wi) {
                 const int q0 = wst[wi], q1 = wst[wi + 1];
                 if (q0 == q1) continue;
-                const int32_t wbase = mn + (wi << kLimWinLog);
-                for (int q = q0 + threadIdx.x; q < q1; q += kLimThreads) {
+                const int32_t wbase = mn + (wi << C::kWinLog);
+                for (int q = q0 + threadIdx.x; q < q1; q += C::kThreads) {
                     const int x = sc_col[q] - wbase;
                     smem_add_f64(acc + x, (double)sc_val[q]);
                     atomicOr(bits + (x >> 5), 1u << (x & 31));
                 }
                 __syncthreads();
-                constexpr int WPT = kLimWords >= kLimThreads ? kLimWords / kLimThreads : 1;
-                const bool own = threadIdx.x * WPT < kLimWords;   // threads past the bitmap: no words
+                constexpr int WPT = C::kWords >= C::kThreads ? C::kWords / C::kThreads : 1;
+                const bool own = threadIdx.x * WPT < C::kWords;   // threads past the bitmap: no words
                 int cntw = 0;
                 uint32_t word[WPT];
 #pragma unroll
@@ -1140,16 +1155,16 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
         }
         if (dense) {
             double *acc = (double *)smem_raw;
-            uint32_t *bits = (uint32_t *)(smem_raw + kLimWindow * 8);
-            for (int t = threadIdx.x; t < kLimWindow; t += kLimThreads) acc[t] = 0.0;
-            for (int t = threadIdx.x; t < kLimWindow / 32; t += kLimThreads) bits[t] = 0u;
+            uint32_t *bits = (uint32_t *)(smem_raw + C::kWindow * 8);
+            for (int t = threadIdx.x; t < C::kWindow; t += C::kThreads) acc[t] = 0.0;
+            for (int t = threadIdx.x; t < C::kWindow / 32; t += C::kThreads) bits[t] = 0u;
             __syncthreads();
-            for (int64_t w0 = mn; w0 <= mx; w0 += kLimWindow) {
-                const int32_t wend = (int32_t)min((int64_t)mx + 1, w0 + kLimWindow);
+            for (int64_t w0 = mn; w0 <= mx; w0 += C::kWindow) {
+                const int32_t wend = (int32_t)min((int64_t)mx + 1, w0 + C::kWindow);
                 // warp per run, 32 products per step: a run contributes L / (R * #windows) < 2
                 // products to a window on average, so a wider probe mostly loads entries of later
                 // windows (measured: 4 vectors per lane made C3's densest rows 4x slower)
-                for (int q = w; q < R; q += kLimNW) {
+                for (int q = w; q < R; q += C::kNW) {
                     const int64_t b = rbase[q];
                     const int len = rlen[q];
                     int cur = cursor[q];
@@ -1169,8 +1184,8 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     if (lane == 0) cursor[q] = cur;
                 }
                 __syncthreads();
-                constexpr int WPT = kLimWords >= kLimThreads ? kLimWords / kLimThreads : 1;
-                const bool own = threadIdx.x * WPT < kLimWords;   // threads past the bitmap: no words
+                constexpr int WPT = C::kWords >= C::kThreads ? C::kWords / C::kThreads : 1;
+                const bool own = threadIdx.x * WPT < C::kWords;   // threads past the bitmap: no words
                 int cntw = 0;
                 uint32_t word[WPT];
 #pragma unroll
@@ -1209,20 +1224,21 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     }
                 };
                 // sparse long row: coarse column partition through global scratch (two coalesced passes)
-                //  1. histogram over kCoarseBins column ranges; greedy groups of <= kLimCap entries
+                //  1. histogram over kCoarseBins column ranges; greedy groups of <= C::kCap entries
                 //  2. scatter the row into the block's scratch, grouped by column range
                 //  3. per group (ascending): smem bucket sort (merge-path fallback), merged entries
                 //     appended at the head of the row's bucket -- the row now lives in scratch
-                int *fh = (int *)(smem_raw + kLimSortBytes);      // [kCoarseBins] counts -> group id
+                int *fh = (int *)(smem_raw + C::kSortBytes);      // [kCoarseBins] counts -> group id
                 int *gstart = fh + kCoarseBins;                    // [kCoarseBins + 1]
                 int *gcur = gstart + kCoarseBins + 1;              // [kCoarseBins]
+                int *gbin = gcur + kCoarseBins;                    // [kCoarseBins + 1] first bin of each group
                 __shared__ int s_ngroups, s_bad;
                 const uint32_t span32 = (uint32_t)(mx - mn);
                 const int bits = span32 ? 32 - __clz(span32) : 0;
                 const int shc = max(0, bits - kCoarseLog);
-                for (int t = threadIdx.x; t < kCoarseBins; t += kLimThreads) fh[t] = 0;
+                for (int t = threadIdx.x; t < kCoarseBins; t += C::kThreads) fh[t] = 0;
                 __syncthreads();
-                for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+                for (int64_t p = threadIdx.x; p < (cap >> 2); p += C::kThreads) {
                     const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
                     if (c4.x != kKeyPad) atomicAdd(&fh[(c4.x - mn) >> shc], 1);
                     if (c4.y != kKeyPad) atomicAdd(&fh[(c4.y - mn) >> shc], 1);
@@ -1230,9 +1246,9 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     if (c4.w != kKeyPad) atomicAdd(&fh[(c4.w - mn) >> shc], 1);
                 }
                 __syncthreads();
-                {   // grouping of consecutive bins: group(b) = floor(prefix(b) / (kLimCap/2)); with no bin
-                    // above kLimCap/2 a group holds < kLimCap products.  Bins per thread: 2 (1024 / 512).
-                    constexpr int BPT = kCoarseBins / kLimThreads;
+                {   // grouping of consecutive bins: group(b) = floor(prefix(b) / (C::kCap/2)); with no bin
+                    // above C::kCap/2 a group holds < C::kCap products.  Bins per thread: 2 (1024 / 512).
+                    constexpr int BPT = kCoarseBins / C::kThreads;
                     int c[BPT], cnt = 0, mxb = 0;
 #pragma unroll
                     for (int u = 0; u < BPT; ++u) {
@@ -1243,47 +1259,57 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     int tot;
                     int ex = grp.excl_sum(cnt, sc, &tot);
                     mxb = grp.reduce_max(mxb, sc);
-                    // groups < T + max bin <= kLimCap: 3/4 of the sorter when no bin exceeds 1/4 of it
+                    // groups < T + max bin <= C::kCap: 3/4 of the sorter when no bin exceeds 1/4 of it
                     // (fewer, fuller sorts: C3 182 -> 159 ms; 7/8: same speed), else 1/2, so rows
                     // with one heavy column range still take this path (C5: 3/4 alone sent them to
                     // the window path, limited merge 86 -> 115 ms)
-                    const int T = mxb <= kLimCap / 4 ? kLimCap * 3 / 4 : kLimCap / 2;
+                    const int T = mxb <= C::kCap / 4 ? C::kCap * 3 / 4 : C::kCap / 2;
 #pragma unroll
                     for (int u = 0; u < BPT; ++u) {
                         fh[threadIdx.x * BPT + u] = ex / T;     // group id of the bin
                         ex += c[u];
                     }
                     const int ng = (tot + T - 1) / T;
+                    // (group ids are prefix / T: more of them than table slots when the row holds more than
+                    // kCoarseBins * T products -- the smaller sorters of 2 / 4 blocks per SM: not this path)
+                    const bool over = ng > kCoarseBins;
                     // group start = first prefix value >= gi*T, i.e. prefix of the first bin of group gi
-                    for (int gi = threadIdx.x; gi <= ng; gi += kLimThreads) gstart[gi] = 0x7fffffff;
+                    if (!over)
+                        for (int gi = threadIdx.x; gi <= ng; gi += C::kThreads) { gstart[gi] = 0x7fffffff; gbin[gi] = 0x7fffffff; }
                     __syncthreads();
                     int pre = ex - cnt;
+                    if (!over) {
 #pragma unroll
-                    for (int u = 0; u < BPT; ++u) {
-                        atomicMin(&gstart[pre / T], pre);
-                        pre += c[u];
+                        for (int u = 0; u < BPT; ++u) {
+                            atomicMin(&gstart[pre / T], pre);
+                            atomicMin(&gbin[pre / T], threadIdx.x * BPT + u);
+                            pre += c[u];
+                        }
                     }
                     if (threadIdx.x == 0) {
                         s_ngroups = ng;
-                        s_bad = mxb > kLimCap - T;
-                        gstart[ng] = tot;
+                        s_bad = over || mxb > C::kCap - T;
+                        if (!over) {
+                            gstart[ng] = tot;
+                            gbin[ng] = kCoarseBins;
+                        }
                     }
                     __syncthreads();
                     // groups with no bin starting inside them cannot exist (bins are contiguous), but
                     // guard: an untouched start inherits the next group's start (empty group)
-                    if (threadIdx.x == 0)
+                    if (threadIdx.x == 0 && !over)
                         for (int gi = ng - 1; gi >= 0; --gi)
-                            if (gstart[gi] == 0x7fffffff) gstart[gi] = gstart[gi + 1];
+                            if (gstart[gi] == 0x7fffffff) { gstart[gi] = gstart[gi + 1]; gbin[gi] = gbin[gi + 1]; }
                 }
                 __syncthreads();
                 sub(10);   // min/max, histogram, grouping
-                if (!s_bad) {   // (a single column range holding > kLimCap products: window path)
+                if (!s_bad) {   // (a single column range holding > C::kCap products: window path)
                     const int ng = s_ngroups;
                     int32_t *sc_col = g.scratch_col + (int64_t)blockIdx.x * g.stage_cap;
                     float *sc_val = g.scratch_val + (int64_t)blockIdx.x * g.stage_cap;
-                    for (int t = threadIdx.x; t < ng; t += kLimThreads) gcur[t] = gstart[t];
+                    for (int t = threadIdx.x; t < ng; t += C::kThreads) gcur[t] = gstart[t];
                     __syncthreads();
-                    for (int64_t p = threadIdx.x; p < (cap >> 2); p += kLimThreads) {
+                    for (int64_t p = threadIdx.x; p < (cap >> 2); p += C::kThreads) {
                         const int4 c4 = *reinterpret_cast<const int4 *>(g.chat_col + s + 4 * p);
                         const float4 v4 = *reinterpret_cast<const float4 *>(g.chat_val + s + 4 * p);
                         const int32_t cc[4] = {c4.x, c4.y, c4.z, c4.w};
@@ -1308,12 +1334,15 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     for (int gi = 0; gi < ng; ++gi) {
                         const int g0 = gstart[gi], n = gstart[gi + 1] - g0;
                         if (n == 0) continue;
-                        int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(
-                            grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + kLimCap * 4),
-                            (int32_t *)(smem_raw + kLimCap * 8), (float *)(smem_raw + kLimCap * 12),
-                            (int *)(smem_raw + kLimCap * 16), oc + nout, ov + nout, sc);
+                        // the group's column range from its coarse bins (no min / max reduction)
+                        const int32_t gmn = (int32_t)((int64_t)mn + ((int64_t)gbin[gi] << shc));
+                        const int32_t gmx = (int32_t)min((int64_t)mx, (int64_t)mn + ((int64_t)gbin[gi + 1] << shc) - 1);
+                        int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, true>(
+                            grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + C::kCap * 4),
+                            (int32_t *)(smem_raw + C::kCap * 8), (float *)(smem_raw + C::kCap * 12),
+                            (int *)(smem_raw + C::kCap * 16), oc + nout, ov + nout, sc, gmn, gmx);
                         if (U < 0)
-                            U = merge_row_in_smem<kLimNW, 1, kLimCap>(grp, smem_raw, sc, sc_col, sc_val, g0, n, n,
+                            U = merge_row_in_smem<C::kNW, 1, C::kCap>(grp, smem_raw, sc, sc_col, sc_val, g0, n, n,
                                                                       oc + nout, ov + nout);
                         nout += U;
                         __syncthreads();
@@ -1327,13 +1356,17 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 __syncthreads();
             }
             if (done_coarse) { rec(1); continue; }
+            if (g.defer_list) {   // (a column range too heavy for this block's sorter: the 1-per-SM launch)
+                if (threadIdx.x == 0) g.defer_list[atomicAdd(g.defer_count, 1u)] = (int32_t)r;
+                continue;
+            }
             // sparse: windows whose products fit the smem sorter
             int32_t *k0 = (int32_t *)smem_raw;
-            float *v0 = (float *)(smem_raw + kLimCap * 4);
+            float *v0 = (float *)(smem_raw + C::kCap * 4);
             int64_t remaining = L;
             int64_t w0 = mn;
             while (w0 <= mx) {
-                int64_t width = max((int64_t)1, (int64_t)((double)(mx + 1 - w0) * (kLimCap / 2) / (double)max(remaining, (int64_t)1)));
+                int64_t width = max((int64_t)1, (int64_t)((double)(mx + 1 - w0) * (C::kCap / 2) / (double)max(remaining, (int64_t)1)));
                 int total = 0;
                 int32_t wend = 0;
                 int32_t head = kKeyPad;
@@ -1341,7 +1374,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     wend = (int32_t)min((int64_t)mx + 1, w0 + width);
                     int part = 0;
                     int32_t hmin = kKeyPad;
-                    for (int q = threadIdx.x; q < R; q += kLimThreads) {
+                    for (int q = threadIdx.x; q < R; q += C::kThreads) {
                         const int64_t b = rbase[q];
                         const int cur = cursor[q], len = rlen[q];
                         if (cur < len) hmin = min(hmin, g.chat_col[b + cur]);
@@ -1353,28 +1386,28 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                     grp.excl_sum(part, sc, &tot);
                     total = tot;
                     head = grp.reduce_min(hmin, sc);
-                    if (total <= kLimCap || width == 1) break;
+                    if (total <= C::kCap || width == 1) break;
                     width = max((int64_t)1, width / 2);
                 }
                 if (total == 0) {              // empty window: jump to the next product's column
                     w0 = max((int64_t)wend, (int64_t)head);
                     continue;
                 }
-                if (total > kLimCap) {         // one column (w0) present in > kLimCap runs
+                if (total > C::kCap) {         // one column (w0) present in > C::kCap runs
                     double part = 0.0;
-                    for (int q = threadIdx.x; q < R; q += kLimThreads) {
+                    for (int q = threadIdx.x; q < R; q += C::kThreads) {
                         if (cnt[q] > 0) {
                             part += (double)g.chat_val[rbase[q] + cursor[q]];
                             cursor[q] += 1;
                         }
                     }
                     part = warp_sum(part);
-                    __shared__ double dred[kLimNW];
+                    __shared__ double dred[C::kNW];
                     if (lane == 0) dred[w] = part;
                     __syncthreads();
                     if (threadIdx.x == 0) {
                         double t = 0.0;
-                        for (int q = 0; q < kLimNW; ++q) t += dred[q];
+                        for (int q = 0; q < C::kNW; ++q) t += dred[q];
                         st_col[nout] = (int32_t)w0;
                         st_val[nout] = (float)t;
                     }
@@ -1386,7 +1419,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 // exclusive scan of cnt[0..R) into offsets (cnt[R] = total), then warp-per-run gather
                 int base_off = 0;
-                for (int q0 = 0; q0 < R; q0 += kLimThreads) {
+                for (int q0 = 0; q0 < R; q0 += C::kThreads) {
                     const int q = q0 + threadIdx.x;
                     const int c = q < R ? cnt[q] : 0;
                     int tot;
@@ -1396,7 +1429,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 if (threadIdx.x == 0) cnt[R] = base_off;
                 __syncthreads();
-                for (int q = w; q < R; q += kLimNW) {
+                for (int q = w; q < R; q += C::kNW) {
                     const int off = cnt[q], c = cnt[q + 1] - off;
                     if (c == 0) continue;
                     const int64_t b = rbase[q] + cursor[q];
@@ -1408,18 +1441,18 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
                 }
                 cp_async_wait_all();
                 __syncthreads();
-                int U = bucket_sort_reduce<kLimNW, 1, kLimEPT, 0, true>(grp, k0, v0, total, k0, v0,
-                                                                (int32_t *)(smem_raw + kLimCap * 8),
-                                                                (float *)(smem_raw + kLimCap * 12),
-                                                                (int *)(smem_raw + kLimCap * 16), st_col + nout,
+                int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, true>(grp, k0, v0, total, k0, v0,
+                                                                (int32_t *)(smem_raw + C::kCap * 8),
+                                                                (float *)(smem_raw + C::kCap * 12),
+                                                                (int *)(smem_raw + C::kCap * 16), st_col + nout,
                                                                 st_val + nout, sc);
                 if (U < 0) {
-                    int32_t *k1 = (int32_t *)(smem_raw + kLimCap * 8);
-                    float *v1 = (float *)(smem_raw + kLimCap * 12);
-                    int *bA = (int *)(smem_raw + kLimCap * 16);
-                    int *bB = bA + SortSmem<kLimCap>::kBoundsA;
-                    const int which = natural_merge_sort<kLimNW, 1, kLimCap>(grp, k0, v0, k1, v1, bA, bB, total, sc);
-                    U = segmented_reduce_out<kLimNW, 1>(grp, which ? k1 : k0, which ? v1 : v0, total,
+                    int32_t *k1 = (int32_t *)(smem_raw + C::kCap * 8);
+                    float *v1 = (float *)(smem_raw + C::kCap * 12);
+                    int *bA = (int *)(smem_raw + C::kCap * 16);
+                    int *bB = bA + SortSmem<C::kCap>::kBoundsA;
+                    const int which = natural_merge_sort<C::kNW, 1, C::kCap>(grp, k0, v0, k1, v1, bA, bB, total, sc);
+                    U = segmented_reduce_out<C::kNW, 1>(grp, which ? k1 : k0, which ? v1 : v0, total,
                                                         st_col + nout, st_val + nout, sc);
                 }
                 __syncthreads();
@@ -1429,7 +1462,7 @@ __global__ void __launch_bounds__(kLimThreads, 1) k_merge_limited(LimitedArgs g)
             }
         }
         // copy the merged row to its output (side buffer, or the head of its Ĉ bucket)
-        for (int64_t p = threadIdx.x; p < nout; p += kLimThreads) {
+        for (int64_t p = threadIdx.x; p < nout; p += C::kThreads) {
             oc[p] = st_col[p];
             ov[p] = st_val[p];
         }

@@ -151,8 +151,6 @@ struct spgemm_plan_s {
     Piece *pieces = nullptr;       // split pieces, whole Normal blocks, gathered Low-performer blocks
     int64_t *piece_uoff = nullptr; // unit (16-byte vector) prefix over pieces
     int64_t *tile_p0 = nullptr;    // first piece of every expansion tile
-    int64_t *piece_eoff = nullptr; // A-entry prefix over pieces (run-per-thread expansion)
-    int64_t *tile_e0 = nullptr;    // first piece of every run tile
     int64_t n_low = 0, n_pieces_all = 0;
     // B' (rows padded to 4 slots, row k at bp_start(b_rowptr[k], k)): cols, values
     int32_t *bp_col = nullptr;
@@ -180,6 +178,7 @@ struct spgemm_plan_s {
     int64_t *row_rng = nullptr;    // (rowmn, rowmx) as int2 in row_order (pipelined bucket bins)
     bool chat_external = false;
     bool c_in_chat = false;        // C compact at the head of the Ĉ arrays (tile merge)
+    int32_t *lim_defer = nullptr;     // B-Limited rows deferred to the 1-per-SM launch (limit_ctas_per_sm > 1)
     unsigned long long *unit_ticket = nullptr;   // profile buffer of the merge kernels (options.reserved[1])
     // merge tiles (merge_tiles.cuh): tile table, look-back words
     TileDesc *tiles = nullptr;
@@ -349,6 +348,38 @@ static int launch_bucket_bin(spgemm_plan_s *p, cudaStream_t s, const int32_t *ro
 }
 
 // ------------------------------------------------------------------ ABI ------------------
+// B-Limited long rows (merge.cuh k_merge_limited<NT>): limit_ctas_per_sm = 1 / 2 / 4 resident limited
+// blocks per SM of 1024 / 512 / 256 threads (PAPER.md L463-L469 L, Fig. 14: the number of blocks
+// an SM holds for the long rows); lim_grid = #SMs x that, persistent, rows claimed longest first.
+template <int NT>
+static int launch_limited_nt(spgemm_plan_s *p, cudaStream_t s, const LimitedArgs &g) {
+    using C = LimCfg<NT>;
+    TRY(kernel_occupancy((const void *)k_merge_limited<NT>, C::kSmem, 0, nullptr));
+    LAUNCH("merge_limited_win", s, k_merge_limited<NT><<<(unsigned)p->lim_grid, NT, C::kSmem, s>>>(g));
+    return SPGEMM_OK;
+}
+
+static int launch_limited(spgemm_plan_s *p, cudaStream_t s, const LimitedArgs &g0) {
+    const int c = p->opt.limit_ctas_per_sm;
+    if (c < 2) return launch_limited_nt<1024>(p, s, g0);
+    // 2 / 4 blocks per SM; rows whose heaviest column range exceeds the smaller sorter are deferred to
+    // a second, 1-per-SM launch (the heaviest rows get a whole SM's shared memory)
+    LimitedArgs g = g0;
+    g.defer_list = p->lim_defer;
+    g.defer_count = (unsigned *)(p->row_counter + 1);
+    CK(cudaMemsetAsync(p->row_counter + 1, 0, 16, s));
+    TRY(c >= 4 ? launch_limited_nt<256>(p, s, g) : launch_limited_nt<512>(p, s, g));
+    LimitedArgs h = g0;
+    h.row_counter = p->row_counter + 2;
+    h.rlist = p->lim_defer;
+    h.rlist_count = (const unsigned *)(p->row_counter + 1);
+    const int grid = p->lim_grid;
+    p->lim_grid = (int)std::min<int64_t>(p->num_sms, p->nlim);
+    const int rc = launch_limited_nt<1024>(p, s, h);
+    p->lim_grid = grid;
+    return rc;
+}
+
 extern "C" {
 
 int spgemm_abi_version(void) { return SPGEMM_ABI_VERSION; }
@@ -658,28 +689,20 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         LAUNCH("piece_whole", s, k_piece_whole<<<grid_for(p->n_low, 256), 256, 0, s>>>(
             p->pair_order + g_lo, p->n_low, p->a_colptr, p->b_rowptr, p->pieces + p->n_split_pieces + p->n_whole));
     TRY(palloc(p, &p->piece_uoff, p->n_pieces_all + 1, s));
-    TRY(palloc(p, &p->piece_eoff, p->n_pieces_all + 1, s));
     if (p->n_pieces_all > 0) {
-        Temp tu(s), ta(s);
-        int64_t *units, *alen;
+        Temp tu(s);
+        int64_t *units;
         TRY(talloc(p, tu, &units, p->n_pieces_all));
-        TRY(talloc(p, ta, &alen, p->n_pieces_all));
         LAUNCH("piece_units", s, k_piece_units<<<grid_for(p->n_pieces_all, 256), 256, 0, s>>>(
-            p->pieces, p->n_pieces_all, units, alen));
+            p->pieces, p->n_pieces_all, units));
         TRY(scan_excl(p, units, p->n_pieces_all, p->piece_uoff, s, "piece_scan"));
-        TRY(scan_excl(p, alen, p->n_pieces_all, p->piece_eoff, s, "piece_scan"));
-        // (units <= nnz(Ĉ)/4 + #pieces and A entries <= units; the tile maps are sized for that
-        // bound, no host sync)
+        // (units <= nnz(Ĉ)/4 + #pieces; the tile map is sized for that bound, no host sync)
         const int64_t ntiles_max = cdiv(p->chat_cap / 4 + p->n_pieces_all, kExpTile);
         TRY(palloc(p, &p->tile_p0, ntiles_max + 1, s));
-        TRY(palloc(p, &p->tile_e0, ntiles_max + 1, s));
         LAUNCH("piece_scan", s, k_tile_first_piece<<<grid_for(ntiles_max + 1, 256), 256, 0, s>>>(
             p->piece_uoff, p->n_pieces_all, ntiles_max, p->tile_p0));
-        LAUNCH("piece_scan", s, k_tile_first_piece<<<grid_for(ntiles_max + 1, 256), 256, 0, s>>>(
-            p->piece_eoff, p->n_pieces_all, ntiles_max, p->tile_e0));
     } else {
         CK(cudaMemsetAsync(p->piece_uoff, 0, 8, s));
-        CK(cudaMemsetAsync(p->piece_eoff, 0, 8, s));
     }
     // B' = B with rows padded to 4 slots (16-byte aligned vector loads in the expansion)
     {   // one allocation: cols then values
@@ -741,7 +764,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
         p->lim_runs = (int64_t)p->h_scal.lim_runs;
         p->lim_max_deg = (int64_t)p->h_scal.lim_max_deg;
         p->lim_max_L = (int64_t)p->h_scal.lim_max_L;
-        p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * o.limit_ctas_per_sm, p->nlim);
+        p->lim_grid = (int)std::min<int64_t>((int64_t)p->num_sms * (o.limit_ctas_per_sm >= 4 ? 4 : o.limit_ctas_per_sm >= 2 ? 2 : 1),
+                                              p->nlim);
         if (!p->long_groups) {   // legacy long-row kernels: run lists + per-CTA whole-row scratch
             TRY(palloc(p, &p->run_base, p->lim_runs, s));
             TRY(palloc(p, &p->run_len, p->lim_runs, s));
@@ -754,7 +778,8 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
             p->lim_max_deg += 1;   // per-block stride of the cursor / cnt scratch (cnt holds R+1 offsets)
             TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
             TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
-            TRY(palloc(p, &p->row_counter, 1, s));
+            TRY(palloc(p, &p->row_counter, 3, s));
+            TRY(palloc(p, &p->lim_defer, p->nlim, s));
         }
     }
     // merge state; Ĉ itself is allocated by spgemm_expand (or is the caller's C, spgemm_execute)
@@ -815,14 +840,10 @@ int spgemm_expand(spgemm_plan_t p, void *stream) {
                 p->pieces, nblk, p->b_rowptr, p->bp_col, p->bp_val, p->a_val, p->base, p->chat_col, p->chat_val,
                 p->exp_ticket, p->lbi));
         }
-        // the gathered Low performers: a run per thread (options.reserved[9] = 2: a vector per
-        // thread, the round-1 unit mapping)
-        if (nblk < p->n_pieces_all && p->opt.reserved[9] == 0)
-            LAUNCH("expand", s, k_expand_flat<true><<<(unsigned)p->num_sms * 5, kExpThreads, 0, s>>>(
-                p->pieces, p->piece_eoff, p->n_pieces_all, p->tile_e0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
-                p->base, p->chat_col, p->chat_val, p->lbi, p->piece_eoff + nblk));
-        else if (nblk < p->n_pieces_all)
-            LAUNCH("expand", s, k_expand_flat<false><<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
+        // the gathered Low performers (and the rest, reserved[9] = 1): 16-byte units over fixed tiles
+        // (a micro-block of W lanes per run and a run per thread measured slower: DESIGN.md §5d)
+        if (nblk < p->n_pieces_all)
+            LAUNCH("expand", s, k_expand_flat<<<(unsigned)p->num_sms * kExpCtasPerSM, kExpThreads, 0, s>>>(
                 p->pieces, p->piece_uoff, p->n_pieces_all, p->tile_p0, p->b_rowptr, p->bp_col, p->bp_val, p->a_val,
                 p->base, p->chat_col, p->chat_val, p->lbi, p->piece_uoff + nblk));
     }
@@ -888,7 +909,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     }
     if (p->nlim > 0) {
         CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
-        LimitedArgs g;
+        LimitedArgs g{};
         g.rows = p->row_order + p->row_starts[kRowBucketLim0];
         g.nrows = p->nlim;
         g.rowoff = p->rowoff;
@@ -917,8 +938,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
-        TRY(kernel_occupancy((const void *)k_merge_limited, kLimSmem, 0, nullptr));
-        LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
+        TRY(launch_limited(p, s, g));
     }
     TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
     return SPGEMM_OK;
@@ -928,7 +948,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
 static int merge_limited_in_place(spgemm_plan_s *p, cudaStream_t s) {
     if (p->nlim == 0) return SPGEMM_OK;
     CK(cudaMemsetAsync(p->row_counter, 0, 8, s));
-    LimitedArgs g;
+    LimitedArgs g{};
     g.rows = p->row_order + p->row_starts[kRowBucketLim0];
     g.nrows = p->nlim;
     g.rowoff = p->rowoff;
@@ -957,8 +977,7 @@ static int merge_limited_in_place(spgemm_plan_s *p, cudaStream_t s) {
     // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
     // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
     TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
-    TRY(kernel_occupancy((const void *)k_merge_limited, kLimSmem, 0, nullptr));
-    LAUNCH("merge_limited_win", s, k_merge_limited<<<(unsigned)p->lim_grid, kLimThreads, kLimSmem, s>>>(g));
+    TRY(launch_limited(p, s, g));
     return SPGEMM_OK;
 }
 

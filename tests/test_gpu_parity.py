@@ -284,12 +284,13 @@ def _wide_inputs(m, k, n, a_density, run_len, seed, hub_col=False, narrow=False,
     (16, 100, 30000, 0.3, 2000, False, False),     # dense rows: fp64 column windows
     (2, 10000, 1000000, 1.0, 21, True, False),     # column 0 in 10000 runs: single-column overflow
 ])
-@pytest.mark.parametrize("fused", [False, "tiles", "tiles_inplace"])
+@pytest.mark.parametrize("fused", [False, "lim2", "lim4", "tiles", "tiles_inplace"])
 def test_limited_paths(m, k, n, dens, run_len, hub, narrow, fused):
     """B-Limited merge: rows longer than the non-limited capacity, through every sub-path."""
     inp = _wide_inputs(m, k, n, dens, run_len, 3, hub_col=hub, narrow=narrow)
     A, B = spg.from_inputs(inp, "cuda")
-    opts = {False: {}, "tiles": TILES, "tiles_inplace": TILES_INPLACE}[fused]
+    opts = {False: {}, "lim2": dict(limit_ctas_per_sm=2), "lim4": dict(limit_ctas_per_sm=4),   # B-Limiting 2 / 4 per SM
+            "tiles": TILES, "tiles_inplace": TILES_INPLACE}[fused]
     with spg.Plan(A, B, **opts) as p:
         st = p.stats()
         assert st["n_rows_bin"][5] > 0
@@ -493,6 +494,26 @@ def test_limited_bucket_overflow_many_heavy_buckets():
             assert p.stats()["n_rows_bin"][5] == 1   # the row is B-Limited (9108 padded slots)
             C = p.execute()
         assert_c_matches(C, inp)
+
+
+@pytest.mark.parametrize("lim", [1, 2, 4])
+def test_limited_huge_row_every_blocks_per_sm(lim):
+    """B-Limiting at 1 / 2 / 4 limited blocks per SM (PAPER.md L463-L469 L, Fig. 14) on two rows of
+    ~1.1M products each spread over 20M columns: more column groups than the coarse tables hold for
+    the smaller sorters, so those rows are deferred to the 1-per-SM launch; C matches the oracle."""
+    rng = np.random.default_rng(7)
+    k, run, n = 1100, 1000, 20_000_000
+    bc = np.concatenate([np.sort(rng.choice(n, run, replace=False)) for _ in range(k)]).astype(np.int32)
+    br = np.repeat(np.arange(k, dtype=np.int32), run)
+    ar = np.repeat(np.arange(2, dtype=np.int32), k)
+    ac = np.tile(np.arange(k, dtype=np.int32), 2)
+    inp = synth.from_coo("huge", 2, k, n, (ar, ac, synth.edge_values(ar, ac, 1)),
+                         (br, bc, synth.edge_values(br, bc, 2)))
+    A, B = spg.from_inputs(inp, "cuda")
+    with spg.Plan(A, B, limit_ctas_per_sm=lim) as p:
+        assert p.stats()["n_rows_bin"][5] == 2
+        C = p.execute()
+    assert_c_matches(C, inp)
 
 
 # ------------------------------------------------------------------ LBI (Eq. 3) ---------------
