@@ -57,18 +57,23 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("config")
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--only", choices=["split", "limit"], default=None)
     args = ap.parse_args()
     inp = synth.make_inputs(args.config)
     A, B = spg.from_inputs(inp, "cuda")
-    for f in ["off", 0, 1, 2, 4, 8, 16, 32, 64]:
+    for f in (["off", 0, 1, 2, 4, 8, 16, 32, 64] if args.only != "limit" else []):
         if f == "off":
             r = run(A, B, args.reps, enable_split=0)
         else:
             r = run(A, B, args.reps, reserved=(0,) * 7 + (f,) + (0,) * 8)
         print(json.dumps({"sweep": "splitting_factor", "config": args.config, "factor": f, **r}), flush=True)
-    for cap in [1, 2, 3]:
+    if args.only == "split":
+        return
+    for cap in [1, 2, 4]:   # B-Limiting: limited blocks of 1024 / 512 / 256 threads per SM (Fig. 14)
         r = run(A, B, args.reps, limit_ctas_per_sm=cap)
         print(json.dumps({"sweep": "limit_ctas_per_sm", "config": args.config, "cap": cap, **r}), flush=True)
+    if args.only == "limit":
+        return
     tiles = (0,) * 5 + (2,) + (0,) * 10   # tile merge: the long-row partition kernel's residency
     for cap in [1, 2]:
         r = run(A, B, args.reps, limit_ctas_per_sm=cap, reserved=tiles)
