@@ -895,6 +895,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS) k_merge_rows(const int32_t *
 // (measured: 256 threads / 3584 slots at 2 blocks per SM made C3's long rows 8.6x slower -- bins
 // of the coarse partition overflow the smaller sorter and fall back to the window search)
 constexpr int kLimBucketCap = 9216;               // rows up to this were merged by the bucket launch
+constexpr int64_t kLimSmallStage = 1 << 18;       // per-block scratch (slots) of the 2 / 4 per SM launch
 constexpr int cmax3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
 constexpr int kCoarseLog = 10;
 constexpr int kCoarseBins = 1 << kCoarseLog;
@@ -1007,6 +1008,10 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
             }
         };
         if (cap <= kLimBucketCap && g.skip_small && g.ccount[i] >= 0) continue;   // merged by the bucket launch
+        if (g.defer_list && cap > g.stage_cap) {   // (longer than this launch's per-block scratch)
+            if (threadIdx.x == 0) g.defer_list[atomicAdd(g.defer_count, 1u)] = (int32_t)r;
+            continue;
+        }
         int32_t *const oc = g.out_col ? g.out_col + g.out_off[i] : g.chat_col + s;
         float *const ov = g.out_col ? g.out_val + g.out_off[i] : g.chat_val + s;
         if (cap <= C::kCap) {

@@ -165,6 +165,7 @@ struct spgemm_plan_s {
     int32_t *scr_cursor = nullptr, *scr_cnt = nullptr, *scr_col = nullptr;
     float *scr_val = nullptr;
     int64_t stage_cap = 0;
+    int64_t stage_cap_small = 0;   // per-block scratch of the 2 / 4 per SM limited launch
     int lim_grid = 0;
     unsigned long long *row_counter = nullptr;
     // stage 3/4
@@ -365,6 +366,8 @@ static int launch_limited(spgemm_plan_s *p, cudaStream_t s, const LimitedArgs &g
     // 2 / 4 blocks per SM; rows whose heaviest column range exceeds the smaller sorter are deferred to
     // a second, 1-per-SM launch (the heaviest rows get a whole SM's shared memory)
     LimitedArgs g = g0;
+    g.stage_cap = p->stage_cap_small;
+    g.coarse_cap = std::min<int64_t>(p->stage_cap_small, p->n);
     g.defer_list = p->lim_defer;
     g.defer_count = (unsigned *)(p->row_counter + 1);
     CK(cudaMemsetAsync(p->row_counter + 1, 0, 16, s));
@@ -773,11 +776,16 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
                 p->a_colptr, p->a_rowidx, K, p->nnz_a, p->b_rowptr, p->base, p->lim_index, p->run_start, p->run_fill,
                 p->run_base, p->run_len));
             p->stage_cap = p->lim_max_L;   // whole-row scratch (dense rows are regrouped by window)
+            // 2 / 4 limited blocks per SM: their scratch is capped (rows above it are deferred to the
+            // 1-per-SM launch), so the allocation stays ~#SMs x the longest row
+            const int64_t nsm = std::min<int64_t>(p->num_sms, p->nlim);
+            p->stage_cap_small = p->lim_grid > nsm ? std::min<int64_t>(p->lim_max_L, kLimSmallStage) : p->lim_max_L;
+            const int64_t scr = std::max<int64_t>(nsm * p->stage_cap, (int64_t)p->lim_grid * p->stage_cap_small);
             TRY(palloc(p, &p->scr_cursor, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
             TRY(palloc(p, &p->scr_cnt, (int64_t)p->lim_grid * (p->lim_max_deg + 1), s));
             p->lim_max_deg += 1;   // per-block stride of the cursor / cnt scratch (cnt holds R+1 offsets)
-            TRY(palloc(p, &p->scr_col, (int64_t)p->lim_grid * p->stage_cap, s));
-            TRY(palloc(p, &p->scr_val, (int64_t)p->lim_grid * p->stage_cap, s));
+            TRY(palloc(p, &p->scr_col, scr, s));
+            TRY(palloc(p, &p->scr_val, scr, s));
             TRY(palloc(p, &p->row_counter, 3, s));
             TRY(palloc(p, &p->lim_defer, p->nlim, s));
         }

@@ -1,0 +1,13 @@
+#!/bin/bash
+# round-2 batch 16: coarse scatter aggregated per 4-product vector;
+# capped small-block scratch.  Limited tests, then C5 / C3 lines
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
+timeout 1200 python -m pytest tests/test_gpu_parity.py -x -q -k "limited or clustered or c_matches or computed" 2>&1 | tail -4 > gpurun_out/b16_pytest.txt
+cat gpurun_out/b16_pytest.txt
+for cfg in C5 C3; do
+  SPGEMM_RESERVED=1=3 timeout 900 python bench.py --config $cfg --steps 3 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/b16_bench_$cfg.jsonl 2> gpurun_out/b16_$cfg.err
+  grep unit-profile gpurun_out/b16_$cfg.err | tail -1
+  python scripts/bench_show.py gpurun_out/b16_bench_$cfg.jsonl | tail -2
+done
