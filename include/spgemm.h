@@ -144,7 +144,9 @@ typedef struct {
                                  [8] 1 = record per-SM busy times for the LBI (SPGEMM_VIEW_LBI);
                                  [9] expansion mapping: 0 block path (split pieces + Normal blocks,
                                      TMA-staged) + a 16-byte vector per thread for the gathered
-                                     Low performers, 1 every block a vector per thread (round 1) */
+                                     Low performers, 1 every block a vector per thread (round 1);
+                                 [11] 1 = rows of 33-256 slots by the warp merge path (round 1)
+                                     instead of a warp-per-row bucket sort (64 / 128 / 256 slots) */
 } spgemm_options_t;
 
 /* Sizes and bin populations of a plan (spgemm_get_stats). */

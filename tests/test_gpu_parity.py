@@ -82,6 +82,7 @@ CASES = [
     ("C1", dict(beta=10.0, enable_limit=0)),
     ("C1", dict(reserved=(0,) * 9 + (1,) + (0,) * 6)),   # expansion: every block through the flat kernel
     ("C1", dict(reserved=(0,) * 9 + (2,) + (0,) * 6)),   # expansion: Low performers a vector per thread
+    ("C1", dict(reserved=(0,) * 11 + (1,) + (0,) * 4)),   # rows of <= 256 slots: warp merge path (round 1)
     ("C1", dict(reserved=(0,) * 7 + (4,) + (0,) * 8)),   # fixed splitting factor 4 (Fig. 11 sweep)
     ("C1", dict(reserved=(0,) * 7 + (64,) + (0,) * 8)),
     ("C1", TILES),
