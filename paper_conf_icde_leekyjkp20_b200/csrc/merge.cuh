@@ -945,6 +945,7 @@ struct LimitedArgs {
     unsigned long long *lbi;      // NULL, or per-SM busy times (LBI, Eq. (3))
     int32_t *defer_list;          // non-NULL: rows the coarse partition cannot take go here (row list index)
     unsigned *defer_count;
+    int dense_div;                // a row is "dense" (fp64 window accumulator) when products * dense_div >= its span
     const int32_t *rlist;         // non-NULL: process only these row list indices (*rlist_count of them)
     const unsigned *rlist_count;
 };
@@ -1045,7 +1046,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
         mx = grp.reduce_max(mx, sc);
         const int64_t span = (int64_t)mx - mn + 1;
         const int64_t nwin_dense = (span + C::kWindow - 1) / C::kWindow;
-        const bool dense = L * 4 >= span && (int64_t)R * nwin_dense <= 2 * L;
+        const bool dense = L * g.dense_div >= span && (int64_t)R * nwin_dense <= 2 * L;
         int64_t nout = 0;
         const int64_t nwin_pow = (span + C::kWindow - 1) >> C::kWinLog;
         if (dense && cap <= g.stage_cap && nwin_pow <= kCoarseBins) {

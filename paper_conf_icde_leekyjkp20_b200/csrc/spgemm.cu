@@ -955,6 +955,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
         g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
         g.lbi = p->lbi ? p->lbi + kLbiSlots : nullptr;
+        g.dense_div = p->opt.reserved[12] > 0 ? p->opt.reserved[12] : 4;   // (tuning knob)
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
@@ -994,6 +995,7 @@ static int merge_limited_in_place(spgemm_plan_s *p, cudaStream_t s) {
     if (g.prof) CK(cudaMemsetAsync(g.prof, 0, 16 * 8, s));
     g.coarse_cap = std::min<int64_t>(p->stage_cap, p->n);
     g.lbi = p->lbi ? p->lbi + kLbiSlots : nullptr;
+        g.dense_div = p->opt.reserved[12] > 0 ? p->opt.reserved[12] : 4;   // (tuning knob)
     // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
     // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
     TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));

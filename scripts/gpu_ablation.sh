@@ -6,7 +6,7 @@ python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 : > gpurun_out/ablation.jsonl
 for c in $1; do
   for o in "" "--opt enable_split=0" "--opt enable_gather=0" "--opt enable_split=0 --opt enable_gather=0" "--opt beta=10 --opt enable_limit=1" "--opt beta=10 --opt enable_limit=0"; do
-    timeout 1200 python bench.py --config $c --steps 3 --warmup 2 --no-e2e --no-cpu-baseline $o > gpurun_out/abl.log 2>&1
+    timeout 400 python bench.py --config $c --steps 3 --warmup 2 --no-e2e --no-cpu-baseline $o > gpurun_out/abl.log 2>&1
     echo "== $c [$o] exit $?"
     grep '^{' gpurun_out/abl.log | python -c "
 import json, sys

@@ -52,6 +52,12 @@ def main():
     for kv in args.opt:
         k, v = kv.split("=")
         opts[k] = float(v) if k in ("alpha", "beta") else int(v)
+    if os.environ.get("SPGEMM_RESERVED"):   # tuning knobs, as bench.py: "index=value,..."
+        res = [0] * 16
+        for kv in os.environ["SPGEMM_RESERVED"].split(","):
+            q, v = kv.split("=")
+            res[int(q)] = int(v)
+        opts["reserved"] = tuple(res)
     inp = synth.make_inputs(args.config)
     A, B = spg.from_inputs(inp, "cuda")
     flush = torch.zeros(512 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
