@@ -315,6 +315,12 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // more than kBucketMax entries (many distinct columns packed into a narrow range) makes the
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
 constexpr int kBucketMax = 64;
+#ifndef SPG_LIM_UNR2
+#define SPG_LIM_UNR2 false   // B-Limited groups: one code per ranking step (two: C5 limited merge 63.6 -> 67.5 ms)
+#endif
+#ifndef SPG_BIN_UNR2
+#define SPG_BIN_UNR2 false   // regular bins: one code per ranking step (two: C2 merge 4.68 -> 5.62 ms)
+#endif
 
 __device__ __forceinline__ int nextpow2_log(int x) { return x <= 1 ? 0 : 32 - __clz(x - 1); }
 
@@ -543,7 +549,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k
         const int L = (int)(rowoff[i + 1] - s);
         if (L > S::kCap) continue;          // (limited list) rows above this kernel's capacity
         const int64_t o = out_col ? crowptr[i] : s;
-        const int U = bucket_sort_reduce<NW, GROUPS, EPT, LS>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
+        const int U = bucket_sort_reduce<NW, GROUPS, EPT, LS, SPG_BIN_UNR2>(g, chat_col + s, chat_val + s, L, dk, dv, dk2, dv2, hist,
                                                           (out_col ? out_col : chat_col) + o,
                                                           (out_col ? out_val : chat_val) + o, sc_all[g.gid],
                                                           rowmn ? rowmn[i] : 1, rowmn ? rowmx[i] : 0);
@@ -618,7 +624,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
         bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, min(m1.L, S::kCap), kn, vn);
         const RowMeta m2 = r + 2 * stride < nrows ? meta[r + 2 * stride] : none;
         if (m0.L <= S::kCap) {
-            const int U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, false, hidx(S::kNb)>(
+            const int U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, SPG_BIN_UNR2, hidx(S::kNb)>(
                 g, key, val, m0.L, dk, dv, dk2, dv2, hist, chat_col + m0.s, chat_val + m0.s, sc_all[g.gid], rg.x, rg.y);
             if (g.gtid == 0) {
                 if (U >= 0) ccount[m0.i] = U;
@@ -1021,7 +1027,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
             int32_t *dk2 = (int32_t *)(smem_raw + C::kCap * 8);
             float *dv2 = (float *)(smem_raw + C::kCap * 12);
             int *hist = (int *)(smem_raw + C::kCap * 16);
-            int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, true>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
+            int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
                                                             dv2, hist, oc, ov, sc);
             if (U < 0)
                 U = merge_row_in_smem<C::kNW, 1, C::kCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
@@ -1343,7 +1349,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
                         // the group's column range from its coarse bins (no min / max reduction)
                         const int32_t gmn = (int32_t)((int64_t)mn + ((int64_t)gbin[gi] << shc));
                         const int32_t gmx = (int32_t)min((int64_t)mx, (int64_t)mn + ((int64_t)gbin[gi + 1] << shc) - 1);
-                        int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, true>(
+                        int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(
                             grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + C::kCap * 4),
                             (int32_t *)(smem_raw + C::kCap * 8), (float *)(smem_raw + C::kCap * 12),
                             (int *)(smem_raw + C::kCap * 16), oc + nout, ov + nout, sc, gmn, gmx);
@@ -1447,7 +1453,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
                 }
                 cp_async_wait_all();
                 __syncthreads();
-                int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, true>(grp, k0, v0, total, k0, v0,
+                int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(grp, k0, v0, total, k0, v0,
                                                                 (int32_t *)(smem_raw + C::kCap * 8),
                                                                 (float *)(smem_raw + C::kCap * 12),
                                                                 (int *)(smem_raw + C::kCap * 16), st_col + nout,
