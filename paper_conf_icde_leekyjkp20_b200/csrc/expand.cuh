@@ -27,7 +27,10 @@
 namespace spg {
 
 constexpr int kExpThreads = 256;
-constexpr int kExpTile = 2048;   // units (16-byte vectors) per tile
+#ifndef SPG_EXP_TILE
+#define SPG_EXP_TILE 2048
+#endif
+constexpr int kExpTile = SPG_EXP_TILE;   // units (16-byte vectors) per tile
 constexpr int kExpUnroll = 4;
 constexpr int kExpCtasPerSM = 3;   // 80 registers: 3 x 256 threads resident per SM, one persistent wave
 

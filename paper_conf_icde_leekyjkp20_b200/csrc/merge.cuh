@@ -315,6 +315,9 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // more than kBucketMax entries (many distinct columns packed into a narrow range) makes the
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
 constexpr int kBucketMax = 64;
+#ifndef SPG_LIM_T78
+#define SPG_LIM_T78 0   // (A/B build knob: 1 = coarse groups up to 7/8 of the sorter when every bin is small)
+#endif
 #ifndef SPG_LIM_UNR2
 #define SPG_LIM_UNR2 false   // B-Limited groups: one code per ranking step (two: C5 limited merge 63.6 -> 67.5 ms)
 #endif
@@ -326,7 +329,10 @@ __device__ __forceinline__ int nextpow2_log(int x) { return x <= 1 ? 0 : 32 - __
 
 // histogram slot of bucket b: one pad word per 32 buckets, so threads walking contiguous bucket
 // ranges (stride = buckets per thread) hit distinct banks
-__host__ __device__ __forceinline__ constexpr int hidx(int b) { return b + (b >> 5); }
+#ifndef SPG_HPAD
+#define SPG_HPAD 1   // (A/B build knob: 0 = no pad word)
+#endif
+__host__ __device__ __forceinline__ constexpr int hidx(int b) { return SPG_HPAD ? b + (b >> 5) : b; }
 
 // striped load of a row into registers (slot gtid + e*T); sentinel (padding) entries stay kKeyPad
 template <int NW, int GROUPS, int EPT>
@@ -1275,7 +1281,8 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
                     // (fewer, fuller sorts: C3 182 -> 159 ms; 7/8: same speed), else 1/2, so rows
                     // with one heavy column range still take this path (C5: 3/4 alone sent them to
                     // the window path, limited merge 86 -> 115 ms)
-                    const int T = mxb <= C::kCap / 4 ? C::kCap * 3 / 4 : C::kCap / 2;
+                    const int T = SPG_LIM_T78 && mxb <= C::kCap / 8 ? C::kCap * 7 / 8
+                                                                     : (mxb <= C::kCap / 4 ? C::kCap * 3 / 4 : C::kCap / 2);
 #pragma unroll
                     for (int u = 0; u < BPT; ++u) {
                         fh[threadIdx.x * BPT + u] = ex / T;     // group id of the bin
@@ -1629,8 +1636,14 @@ __global__ void __launch_bounds__(kCompactLongThreads) k_compact_long(const int3
 // bucket head (src = rowoff[r] + (q - crowptr[r]); 4 scalar loads, coalesced across the warp).
 // Every row length gets the same per-entry cost (C3's 60K-entry rows made the warp / CTA per
 // row copy 2.4 TB/s).
-constexpr int kCmpChunk = 8192;
-constexpr int kCmpThreads = 256;
+#ifndef SPG_CMP_CHUNK
+#define SPG_CMP_CHUNK 8192
+#endif
+constexpr int kCmpChunk = SPG_CMP_CHUNK;
+#ifndef SPG_CMP_THREADS
+#define SPG_CMP_THREADS 256
+#endif
+constexpr int kCmpThreads = SPG_CMP_THREADS;
 
 __global__ void k_chunk_first_row(const int64_t *__restrict__ crowptr, int64_t M, int64_t nnz, int64_t nchunks,
                                   int32_t *__restrict__ chunk_r0) {
