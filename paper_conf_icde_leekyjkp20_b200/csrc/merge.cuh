@@ -316,7 +316,7 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
 constexpr int kBucketMax = 64;
 #ifndef SPG_LIM_T78
-#define SPG_LIM_T78 0   // (A/B build knob: 1 = coarse groups up to 7/8 of the sorter when every bin is small)
+#define SPG_LIM_T78 1   // coarse groups up to 7/8 of the sorter when every bin is small (C5 limited 63.6 -> 62.6 ms)
 #endif
 #ifndef SPG_LIM_UNR2
 #define SPG_LIM_UNR2 false   // B-Limited groups: one code per ranking step (two: C5 limited merge 63.6 -> 67.5 ms)
