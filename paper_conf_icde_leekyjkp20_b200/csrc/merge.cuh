@@ -619,7 +619,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
     RowMeta m1 = r + stride < nrows ? meta[r + stride] : none;
     int32_t key[EPT];
     float val[EPT];
-    bsr_load<NW, GROUPS, EPT>(g, chat_col + m0.s, chat_val + m0.s, min(m0.L, S::kCap), key, val);
+    bsr_load<NW, GROUPS, EPT>(g, chat_col + m0.s, chat_val + m0.s, m0.L <= S::kCap ? m0.L : 0, key, val);
     // PRECLEAR: hist starts zeroed, every row leaves it zeroed
     for (int b = g.gtid; b <= hidx(S::kNb); b += NW * 32) hist[b] = 0;
     g.sync();
@@ -627,14 +627,15 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
         const int2 rg = rng ? rng[r] : make_int2(1, 0);
         int32_t kn[EPT];
         float vn[EPT];
-        bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, min(m1.L, S::kCap), kn, vn);
+        bsr_load<NW, GROUPS, EPT>(g, chat_col + m1.s, chat_val + m1.s, m1.L <= S::kCap ? m1.L : 0, kn, vn);
         const RowMeta m2 = r + 2 * stride < nrows ? meta[r + 2 * stride] : none;
         if (m0.L <= S::kCap) {
             const int U = bucket_sort_reduce_regs<NW, GROUPS, EPT, LS, SPG_BIN_UNR2, hidx(S::kNb)>(
                 g, key, val, m0.L, dk, dv, dk2, dv2, hist, chat_col + m0.s, chat_val + m0.s, sc_all[g.gid], rg.x, rg.y);
             if (g.gtid == 0) {
                 if (U >= 0) ccount[m0.i] = U;
-                else fb_rows[atomicAdd(fb_count, 1u)] = m0.i;
+                else if (fb_rows) fb_rows[atomicAdd(fb_count, 1u)] = m0.i;
+                else ccount[m0.i] = -1;   // limited list: k_merge_limited takes the row
             }
         }
         // (no barrier needed between rows, see k_merge_bucket)

@@ -317,10 +317,13 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     return SPGEMM_OK;
 }
 
+#ifndef SPG_SHAPE
+#define SPG_SHAPE 0   // merge-bin shapes (A/B build knob; 0 = the measured default)
+#endif
 // software-pipelined in-place bucket bin over rows [b0, b1) of row_order (meta table in p->row_meta)
 template <int NW, int GROUPS, int EPT>
 static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int64_t cnt, const char *name,
-                              int ctas_per_sm) {
+                              int ctas_per_sm, bool fallback_list = true) {
     if (cnt == 0) return SPGEMM_OK;
     const int smem = BucketSmem<NW, EPT, 0>::kBytes * GROUPS;
     auto kern = k_merge_bucket_pipe<NW, GROUPS, EPT, 0>;
@@ -329,7 +332,7 @@ static int launch_bucket_pipe(spgemm_plan_s *p, cudaStream_t s, int64_t q0, int6
     const int64_t grid = std::min<int64_t>(cdiv(cnt, GROUPS), (int64_t)p->num_sms * std::max(occ, 1));
     (void)ctas_per_sm;
     LAUNCH(name, s, kern<<<(unsigned)grid, NW * 32 * GROUPS, smem, s>>>(
-        p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount, p->fb_rows, p->fb_count,
+        p->row_meta + q0, cnt, p->chat_col, p->chat_val, p->ccount, fallback_list ? p->fb_rows : nullptr, p->fb_count,
         p->row_rng ? (const int2 *)p->row_rng + q0 : nullptr));
     return SPGEMM_OK;
 }
@@ -911,14 +914,36 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
     }
     {
         const int64_t q = p->row_starts[kRowBucketSort512];
+#if SPG_SHAPE == 1   // (A/B build knob: more threads per row, fewer slots per thread)
+        TRY(launch_bucket_pipe<4, 2, 4>(p, s, q, p->row_starts[kRowBucketSort512 + 1] - q, "merge_bucket512", 8));
+#else
         TRY(launch_bucket_pipe<2, 4, 8>(p, s, q, p->row_starts[kRowBucketSort512 + 1] - q, "merge_bucket512", 8));
+#endif
         const int64_t q2 = p->row_starts[kRowBucketSort1K];
+#if SPG_SHAPE == 1
+        TRY(launch_bucket_pipe<8, 1, 4>(p, s, q2, p->row_starts[kRowBucketSort1K + 1] - q2, "merge_bucket1k", 8));
+#else
         TRY(launch_bucket_pipe<4, 2, 8>(p, s, q2, p->row_starts[kRowBucketSort1K + 1] - q2, "merge_bucket1k", 8));
+#endif
     }
     rows = rows_of(kRowBucketSort2K, kRowBucketSort2K + 1, &cnt);
+#if SPG_SHAPE == 2   // (A/B build knob: software-pipelined 2K / 4K bins)
+    {
+        const int64_t qa = p->row_starts[kRowBucketSort2K];
+        TRY(launch_bucket_pipe<8, 1, 8>(p, s, qa, cnt, "merge_bucket2k", 4));
+    }
+#else
     TRY(launch_bucket_bin<8, 1, 8>(p, s, rows, cnt, "merge_bucket2k", 8));
+#endif
     rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
+#if SPG_SHAPE == 2
+    {
+        const int64_t qb = p->row_starts[kRowBucketSort4K];
+        TRY(launch_bucket_pipe<16, 1, 8>(p, s, qb, cnt, "merge_bucket4k", 2));
+    }
+#else
     TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+#endif
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
         const int smem = SortSmem<CAP>::kBytes;
@@ -958,7 +983,11 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         g.dense_div = p->opt.reserved[12] > 0 ? p->opt.reserved[12] : 4;   // (tuning knob)
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
+#if SPG_SHAPE == 3   // (A/B build knob: software-pipelined 9216-slot limited bin)
+        TRY(launch_bucket_pipe<32, 1, 9>(p, s, p->row_starts[kRowBucketLim0], g.nrows, "merge_limited_smem", 1, false));
+#else
         TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
+#endif
         TRY(launch_limited(p, s, g));
     }
     TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
