@@ -315,6 +315,12 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // more than kBucketMax entries (many distinct columns packed into a narrow range) makes the
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
 constexpr int kBucketMax = 64;
+#ifndef SPG_LIM_GPIPE
+#define SPG_LIM_GPIPE 0   // (A/B build knob: software-pipelined B-Limited group sorts)
+#endif
+#ifndef SPG_SCATTER_BALLOT
+#define SPG_SCATTER_BALLOT 0   // (A/B build knob: coarse scatter by per-group ballots when a warp spans < 4 groups)
+#endif
 #ifndef SPG_LIM_T78
 #define SPG_LIM_T78 1   // coarse groups up to 7/8 of the sorter when every bin is small (C5 limited 63.6 -> 62.6 ms)
 #endif
@@ -1337,6 +1343,29 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
 #pragma unroll
                         for (int u = 0; u < 4; ++u) {     // warp-aggregated cursor bumps per group
                             const int gid = cc[u] == kKeyPad ? -1 - lane_id() : fh[(cc[u] - mn) >> shc];
+#if SPG_SCATTER_BALLOT
+                            {   // the warp's groups span a few ids: one ballot per id instead of a match
+                                const unsigned act = __activemask();
+                                const int glo = __reduce_min_sync(act, gid >= 0 ? gid : 0x7fffffff);
+                                const int ghi = __reduce_max_sync(act, gid);
+                                if (ghi - glo < 4) {
+                                    for (int gq = glo; gq <= ghi; ++gq) {
+                                        const unsigned m = __ballot_sync(act, gid == gq);
+                                        if (!m) continue;
+                                        const int leader = __ffs(m) - 1;
+                                        int q0 = 0;
+                                        if (lane_id() == leader) q0 = atomicAdd(&gcur[gq], __popc(m));
+                                        q0 = __shfl_sync(act, q0, leader);
+                                        if (gid == gq) {
+                                            const int q = q0 + __popc(m & lanemask_lt());
+                                            sc_col[q] = cc[u];
+                                            sc_val[q] = vv[u];
+                                        }
+                                    }
+                                    continue;
+                                }
+                            }
+#endif
                             const unsigned peers = __match_any_sync(__activemask(), gid);
                             if (gid >= 0) {
                                 const int leader = __ffs(peers) - 1;
@@ -1351,21 +1380,50 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
                     }
                     __syncthreads();
                     sub(11);   // scatter into scratch
+#if SPG_LIM_GPIPE
+                    // software-pipelined group sorts: group gi + 1's products are loaded from the scratch
+                    // (L2) into registers while group gi sorts
+                    int32_t key[C::kEPT];
+                    float val[C::kEPT];
+                    bsr_load<C::kNW, 1, C::kEPT>(grp, sc_col + gstart[0], sc_val + gstart[0], ng > 0 ? gstart[1] - gstart[0] : 0,
+                                                 key, val);
+#endif
                     for (int gi = 0; gi < ng; ++gi) {
                         const int g0 = gstart[gi], n = gstart[gi + 1] - g0;
-                        if (n == 0) continue;
+#if SPG_LIM_GPIPE
+                        int32_t kn[C::kEPT];
+                        float vn[C::kEPT];
+                        {
+                            const int g1 = gi + 1 < ng ? gstart[gi + 1] : 0;
+                            const int n1 = gi + 1 < ng ? gstart[gi + 2] - g1 : 0;
+                            bsr_load<C::kNW, 1, C::kEPT>(grp, sc_col + g1, sc_val + g1, n1, kn, vn);
+                        }
+#endif
+                        if (n > 0) {
                         // the group's column range from its coarse bins (no min / max reduction)
                         const int32_t gmn = (int32_t)((int64_t)mn + ((int64_t)gbin[gi] << shc));
                         const int32_t gmx = (int32_t)min((int64_t)mx, (int64_t)mn + ((int64_t)gbin[gi + 1] << shc) - 1);
+#if SPG_LIM_GPIPE
+                        int U = bucket_sort_reduce_regs<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(
+                            grp, key, val, n, (int32_t *)smem_raw, (float *)(smem_raw + C::kCap * 4),
+                            (int32_t *)(smem_raw + C::kCap * 8), (float *)(smem_raw + C::kCap * 12),
+                            (int *)(smem_raw + C::kCap * 16), oc + nout, ov + nout, sc, gmn, gmx);
+#else
                         int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(
                             grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + C::kCap * 4),
                             (int32_t *)(smem_raw + C::kCap * 8), (float *)(smem_raw + C::kCap * 12),
                             (int *)(smem_raw + C::kCap * 16), oc + nout, ov + nout, sc, gmn, gmx);
+#endif
                         if (U < 0)
                             U = merge_row_in_smem<C::kNW, 1, C::kCap>(grp, smem_raw, sc, sc_col, sc_val, g0, n, n,
                                                                       oc + nout, ov + nout);
                         nout += U;
                         __syncthreads();
+                        }
+#if SPG_LIM_GPIPE
+#pragma unroll
+                        for (int e = 0; e < C::kEPT; ++e) { key[e] = kn[e]; val[e] = vn[e]; }
+#endif
                     }
                     if (threadIdx.x == 0) g.ccount[i] = nout;
                     __syncthreads();

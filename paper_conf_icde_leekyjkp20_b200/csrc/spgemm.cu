@@ -983,11 +983,9 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         g.dense_div = p->opt.reserved[12] > 0 ? p->opt.reserved[12] : 4;   // (tuning knob)
         // limited rows whose bucket fits 9216 slots: one 1024-thread bucket-sort CTA per SM
         // (B-Limiting: 213 KB of shared memory each); the others: windowed kernel below
-#if SPG_SHAPE == 3   // (A/B build knob: software-pipelined 9216-slot limited bin)
+        // limited rows of <= 9216 slots: software-pipelined 1024-thread bucket sort, the next row's slots
+        // loaded while this one sorts (C5 20.9 -> 20.0 ms, C3 14.9 -> 14.0 ms vs the plain bin)
         TRY(launch_bucket_pipe<32, 1, 9>(p, s, p->row_starts[kRowBucketLim0], g.nrows, "merge_limited_smem", 1, false));
-#else
-        TRY(launch_bucket_bin<32, 1, 9>(p, s, g.rows, g.nrows, "merge_limited_smem", 1, false));
-#endif
         TRY(launch_limited(p, s, g));
     }
     TRY(scan_excl(p, p->ccount, M, p->crowptr, s, "c_rowptr"));
