@@ -315,6 +315,9 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // more than kBucketMax entries (many distinct columns packed into a narrow range) makes the
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
 constexpr int kBucketMax = 64;
+#ifndef SPG_BIN_THREADS_SM
+#define SPG_BIN_THREADS_SM 1280   // k_merge_bucket: resident threads per SM the register budget targets
+#endif
 #ifndef SPG_LIM_GPIPE
 #define SPG_LIM_GPIPE 0   // (A/B build knob: software-pipelined B-Limited group sorts)
 #endif
@@ -533,7 +536,7 @@ struct BucketSmem {
 
 // Rows of one bin: bucket sort per row; rows whose buckets overflow go to a fallback list.
 template <int NW, int GROUPS, int EPT, int LS = 0>
-__global__ void __launch_bounds__(NW * 32 * GROUPS, 1280 / (NW * 32 * GROUPS)) k_merge_bucket(const int32_t *__restrict__ rows, int64_t nrows,
+__global__ void __launch_bounds__(NW * 32 * GROUPS, SPG_BIN_THREADS_SM / (NW * 32 * GROUPS)) k_merge_bucket(const int32_t *__restrict__ rows, int64_t nrows,
                                                                   const int64_t *__restrict__ rowoff,
                                                                   int32_t *__restrict__ chat_col,
                                                                   float *__restrict__ chat_val,

@@ -317,6 +317,9 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     return SPGEMM_OK;
 }
 
+#ifndef SPG_WB_PIPE
+#define SPG_WB_PIPE 0
+#endif
 #ifndef SPG_SHAPE
 #define SPG_SHAPE 0   // merge-bin shapes (A/B build knob; 0 = the measured default)
 #endif
@@ -895,11 +898,19 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
                                       // reserved[11] = 1: the warp merge path, round 1)
         int64_t c1;
         const int32_t *r1 = rows_of(kRowBucketWarp64, kRowBucketWarp64 + 1, &c1);
+#if SPG_WB_PIPE   // (A/B build knob: software-pipelined warp-per-row bins)
+        TRY(launch_bucket_pipe<1, 8, 2>(p, s, p->row_starts[kRowBucketWarp64], c1, "merge_wbucket64", 8));
+        r1 = rows_of(kRowBucketWarp128, kRowBucketWarp128 + 1, &c1);
+        TRY(launch_bucket_pipe<1, 8, 4>(p, s, p->row_starts[kRowBucketWarp128], c1, "merge_wbucket128", 8));
+        r1 = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &c1);
+        TRY(launch_bucket_pipe<1, 8, 8>(p, s, p->row_starts[kRowBucketSort256], c1, "merge_wbucket256", 8));
+#else
         TRY(launch_bucket_bin<1, 8, 2>(p, s, r1, c1, "merge_wbucket64", 8));
         r1 = rows_of(kRowBucketWarp128, kRowBucketWarp128 + 1, &c1);
         TRY(launch_bucket_bin<1, 8, 4>(p, s, r1, c1, "merge_wbucket128", 8));
         r1 = rows_of(kRowBucketSort256, kRowBucketSort256 + 1, &c1);
         TRY(launch_bucket_bin<1, 8, 8>(p, s, r1, c1, "merge_wbucket256", 8));
+#endif
         cnt = 0;
     }
     if (cnt > 0) {
