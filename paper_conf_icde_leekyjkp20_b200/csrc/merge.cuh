@@ -316,7 +316,7 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
 constexpr int kBucketMax = 64;
 #ifndef SPG_BIN_THREADS_SM
-#define SPG_BIN_THREADS_SM 1280   // k_merge_bucket: resident threads per SM the register budget targets
+#define SPG_BIN_THREADS_SM 1024   // k_merge_bucket: 64 registers, no spills (1280: C5 +0.5 ms)
 #endif
 #ifndef SPG_LIM_GPIPE
 #define SPG_LIM_GPIPE 0   // (A/B build knob: software-pipelined B-Limited group sorts)
