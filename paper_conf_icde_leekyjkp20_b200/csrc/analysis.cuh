@@ -393,9 +393,9 @@ __global__ void k_piece_whole(const int32_t *__restrict__ list, int64_t n, const
     }
 }
 
-// B' (B with rows padded to 4 slots) row k starts at bp_start(b_rowptr[k], k) = b_rowptr[k] + 7k
-// rounded up to 4 slots: 16-byte aligned and clear of row k + 1 (row k ends by b_rowptr[k+1] + 7k + 6)
-// without a scan over the padded lengths; B' holds nnz(B) + 7K + 4 slots.
+// B' (B with rows padded to kRunAlign = 8 slots, R16) row k starts at bp_start(b_rowptr[k], k) =
+// b_rowptr[k] + 15k rounded up to 8 slots: 32-byte aligned and clear of row k + 1 (row k ends by
+// b_rowptr[k+1] + 15k + 14) without a scan over the padded lengths; B' holds nnz(B) + 15K + 8 slots.
 __host__ __device__ __forceinline__ int64_t bp_start(int64_t rp, int64_t k) {
     return (rp + (2 * kRunAlign - 1) * k + kRunAlign - 1) & ~(int64_t)(kRunAlign - 1);
 }

@@ -4,7 +4,7 @@
 // each product (i, j, a_ik*b_kj) is stored in Ĉ (L321-L323 L).  The row-wise offsets of
 // stage (1) place every product of row i inside row i's bucket (L289-L291 R): the run of
 // A entry e = (i, k) is Ĉ[base[e] .. base[e] + nnz(b_k*)), in B's (ascending) column order,
-// padded with sentinel slots to a multiple of 4 (16 bytes).
+// padded with sentinel slots to a multiple of 8 (one 32-byte sector of columns and one of values, R16).
 //
 // Ĉ layout: SoA, row implicit: chat_col int32[nnz(Ĉ)], chat_val fp32[nnz(Ĉ)] (8 B/product).
 //
@@ -34,8 +34,8 @@ constexpr int kExpTile = SPG_EXP_TILE;   // units (16-byte vectors) per tile
 constexpr int kExpUnroll = 4;
 constexpr int kExpCtasPerSM = 3;   // 80 registers: 3 x 256 threads resident per SM, one persistent wave
 
-// vectors of one run written by a block: the B sub-row rounded up to 4 slots (B tiles start on
-// 4-slot boundaries, so the last tile of a row also writes the run's sentinel padding)
+// vectors of one run written by a block: the B sub-row rounded up to 8 slots (B tiles start on
+// 8-slot boundaries, so the last tile of a row also writes the run's sentinel padding)
 __device__ __forceinline__ int piece_nvec(const Piece &pc) { return (int)(pad_run(pc.b_len) >> 2); }
 
 __global__ void k_piece_units(const Piece *__restrict__ pieces, int64_t n, int64_t *__restrict__ units) {

@@ -659,7 +659,7 @@ __global__ void __launch_bounds__(NW * 32 * GROUPS, 1024 / (NW * 32 * GROUPS)) k
 
 // -------------------------------------------- warp merge-path natural merge sort (WMP) ---
 // No shared-memory atomics (see k_count_rows).  A row's bucket is a concatenation of runs (one
-// per stored a_ik, ascending, sentinel-padded to 4 slots), so it is sorted by merging them.
+// per stored a_ik, ascending, sentinel-padded to 8 slots), so it is sorted by merging them.
 // A group of NW warps (T = 32*NW threads) per row:
 //   1. 16-byte vector loads; (col, val) packed into one u64 (col in the high word) in smem;
 //      runs start at vector boundaries where the column descends (or the previous run ended

@@ -152,7 +152,7 @@ struct spgemm_plan_s {
     int64_t *piece_uoff = nullptr; // unit (16-byte vector) prefix over pieces
     int64_t *tile_p0 = nullptr;    // first piece of every expansion tile
     int64_t n_low = 0, n_pieces_all = 0;
-    // B' (rows padded to 4 slots, row k at bp_start(b_rowptr[k], k)): cols, values
+    // B' (rows padded to 8 slots, row k at bp_start(b_rowptr[k], k)): cols, values
     int32_t *bp_col = nullptr;
     size_t bp_bytes = 0;
     float *bp_val = nullptr;
@@ -713,7 +713,7 @@ static int plan_impl(spgemm_plan_s *p, const spgemm_csc_t *A, const spgemm_csr_t
     } else {
         CK(cudaMemsetAsync(p->piece_uoff, 0, 8, s));
     }
-    // B' = B with rows padded to 4 slots (16-byte aligned vector loads in the expansion)
+    // B' = B with rows padded to 8 slots (32-byte aligned rows: vector loads, bulk copies in the expansion)
     {   // one allocation: cols then values
         const int64_t nbp = (p->nnz_b + (2 * kRunAlign - 1) * K + kRunAlign + 63) & ~(int64_t)63;   // (bp_start)
         TRY(palloc(p, &p->bp_col, 2 * nbp, s));
