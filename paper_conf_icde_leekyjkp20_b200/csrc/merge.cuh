@@ -318,6 +318,9 @@ constexpr int kBucketMax = 64;
 #ifndef SPG_BIN_THREADS_SM
 #define SPG_BIN_THREADS_SM 1024   // k_merge_bucket: 64 registers, no spills (1280: C5 +0.5 ms)
 #endif
+#ifndef SPG_LIM_LS
+#define SPG_LIM_LS 0   // (A/B build knob: 1 = twice the buckets in the B-Limited sorts, capped at 16384)
+#endif
 #ifndef SPG_LIM_GPIPE
 #define SPG_LIM_GPIPE 0   // (A/B build knob: software-pipelined B-Limited group sorts)
 #endif
@@ -396,7 +399,7 @@ __device__ __forceinline__ int bucket_sort_reduce_regs(const Group<NW, GROUPS> &
     }
     const uint32_t span = (uint32_t)(mx - mn);
     // (>= 64 buckets: sh <= 25, so a key's in-bucket bits and its 7-bit atomic rank fit 32 bits)
-    const int lognb = max(6, nextpow2_log(L) + LS);
+    const int lognb = LS > 0 ? min(14, max(6, nextpow2_log(L) + LS)) : max(6, nextpow2_log(L));   // (LS: <= 16384 buckets)
     const int nb = 1 << lognb;
     const int bits = span ? 32 - __clz(span) : 0;
     const int sh = max(0, bits - lognb);
@@ -1043,7 +1046,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
             int32_t *dk2 = (int32_t *)(smem_raw + C::kCap * 8);
             float *dv2 = (float *)(smem_raw + C::kCap * 12);
             int *hist = (int *)(smem_raw + C::kCap * 16);
-            int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
+            int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, (NT >= 1024 ? SPG_LIM_LS : 0), SPG_LIM_UNR2>(grp, g.chat_col + s, g.chat_val + s, (int)cap, dk, dv, dk2,
                                                             dv2, hist, oc, ov, sc);
             if (U < 0)
                 U = merge_row_in_smem<C::kNW, 1, C::kCap>(grp, smem_raw, sc, g.chat_col, g.chat_val, s, (int)cap, (int)L,
@@ -1412,7 +1415,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
                             (int32_t *)(smem_raw + C::kCap * 8), (float *)(smem_raw + C::kCap * 12),
                             (int *)(smem_raw + C::kCap * 16), oc + nout, ov + nout, sc, gmn, gmx);
 #else
-                        int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(
+                        int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, (NT >= 1024 ? SPG_LIM_LS : 0), SPG_LIM_UNR2>(
                             grp, sc_col + g0, sc_val + g0, n, (int32_t *)smem_raw, (float *)(smem_raw + C::kCap * 4),
                             (int32_t *)(smem_raw + C::kCap * 8), (float *)(smem_raw + C::kCap * 12),
                             (int *)(smem_raw + C::kCap * 16), oc + nout, ov + nout, sc, gmn, gmx);
@@ -1522,7 +1525,7 @@ __global__ void __launch_bounds__(NT, 1024 / NT) k_merge_limited(LimitedArgs g) 
                 }
                 cp_async_wait_all();
                 __syncthreads();
-                int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, 0, SPG_LIM_UNR2>(grp, k0, v0, total, k0, v0,
+                int U = bucket_sort_reduce<C::kNW, 1, C::kEPT, (NT >= 1024 ? SPG_LIM_LS : 0), SPG_LIM_UNR2>(grp, k0, v0, total, k0, v0,
                                                                 (int32_t *)(smem_raw + C::kCap * 8),
                                                                 (float *)(smem_raw + C::kCap * 12),
                                                                 (int *)(smem_raw + C::kCap * 16), st_col + nout,

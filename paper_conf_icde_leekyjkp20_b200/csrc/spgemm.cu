@@ -317,6 +317,9 @@ static int partition(spgemm_plan_s *p, const uint8_t *bucket, int64_t n, int nb,
     return SPGEMM_OK;
 }
 
+#ifndef SPG_BIN_LS
+#define SPG_BIN_LS 0   // (A/B build knob: 1 = twice the buckets in the 2K / 4K bins)
+#endif
 #ifndef SPG_WB_PIPE
 #define SPG_WB_PIPE 0
 #endif
@@ -944,7 +947,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         TRY(launch_bucket_pipe<8, 1, 8>(p, s, qa, cnt, "merge_bucket2k", 4));
     }
 #else
-    TRY(launch_bucket_bin<8, 1, 8>(p, s, rows, cnt, "merge_bucket2k", 8));
+    TRY(launch_bucket_bin<8, 1, 8, SPG_BIN_LS>(p, s, rows, cnt, "merge_bucket2k", 8));
 #endif
     rows = rows_of(kRowBucketSort4K, kRowBucketSort4K + 1, &cnt);
 #if SPG_SHAPE == 2
@@ -953,7 +956,7 @@ static int merge_bins(spgemm_plan_s *p, cudaStream_t s) {
         TRY(launch_bucket_pipe<16, 1, 8>(p, s, qb, cnt, "merge_bucket4k", 2));
     }
 #else
-    TRY(launch_bucket_bin<16, 1, 8>(p, s, rows, cnt, "merge_bucket4k", 4));
+    TRY(launch_bucket_bin<16, 1, 8, SPG_BIN_LS>(p, s, rows, cnt, "merge_bucket4k", 4));
 #endif
     {   // rows whose buckets overflowed: natural merge sort (count read on the device)
         constexpr int CAP = 4096;
