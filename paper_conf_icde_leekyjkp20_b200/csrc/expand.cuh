@@ -27,6 +27,9 @@
 namespace spg {
 
 constexpr int kExpThreads = 256;
+#ifndef SPG_EXP_PREFETCH
+#define SPG_EXP_PREFETCH 0   // (A/B build knob: L2 prefetch of a tile's A values / run bases)
+#endif
 #ifndef SPG_EXP_TILE
 #define SPG_EXP_TILE 2048
 #endif
@@ -154,6 +157,25 @@ __global__ void __launch_bounds__(kExpThreads) k_expand_flat(
             if (threadIdx.x == 0) s_uoff[np] = INT64_MAX;
         }
         __syncthreads();
+#if SPG_EXP_PREFETCH
+        if (cached) {   // L2 prefetch of the A values / run bases the tile's units will load
+            for (int q = threadIdx.x; q < np; q += kExpThreads) {
+                const int64_t u0 = max(s_uoff[q], f0) - s_uoff[q], u1 = min(s_uoff[q + 1], f1) - s_uoff[q];
+                if (u1 <= u0) continue;
+                const int nv = s_nv[q];
+                const int64_t e0 = s_alo[q] + u0 / nv, e1 = s_alo[q] + (u1 - 1) / nv;
+                for (int64_t e = e0 & ~(int64_t)15; e <= e1; e += 16)   // 128-byte lines of base[]
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(base + e));
+                for (int64_t e = e0 & ~(int64_t)31; e <= e1; e += 32)   // ... of a_val[]
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(a_val + e));
+                if (SPG_EXP_PREFETCH >= 2)   // ... and of the block's B' row (columns, values)
+                    for (int64_t j = s_bsrc[q] & ~(int64_t)31; j < s_bsrc[q] + 4 * nv; j += 32) {
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(bp_col + j));
+                        asm volatile("prefetch.global.L2 [%0];" ::"l"(bp_val + j));
+                    }
+            }
+        }
+#endif
         // kExpUnroll units per thread per step, their loads issued together
         int pj = 0;             // cached: local block index (never decreases)
         int64_t gj = p0;        // uncached: global block index
