@@ -314,7 +314,11 @@ __device__ __forceinline__ int segmented_reduce_out(const Group<NW, GROUPS> &g, 
 // Equal columns always share a bucket, so no segment crosses a thread's range.  A bucket with
 // more than kBucketMax entries (many distinct columns packed into a narrow range) makes the
 // function return -1 before anything is written; the caller falls back to the natural merge sort.
-constexpr int kBucketMax = 64;
+#ifndef SPG_BUCKET_MAX
+#define SPG_BUCKET_MAX 127   // (<= 127: the sort code keeps 7 bits of atomic rank; 64: C3 +5.4 ms)
+#endif
+constexpr int kBucketMax = SPG_BUCKET_MAX;
+static_assert(kBucketMax <= 127, "sort codes hold 7 bits of in-bucket rank");
 #ifndef SPG_BIN_THREADS_SM
 #define SPG_BIN_THREADS_SM 1024   // k_merge_bucket: 64 registers, no spills (1280: C5 +0.5 ms)
 #endif

@@ -477,11 +477,13 @@ def test_computed_zeros_long_rows():
 
 
 # ------------------------------------------------------------------ overflow regression -----
-def test_limited_bucket_overflow_many_heavy_buckets():
-    """one limited row of <= 9216 slots in which >= 128 buckets overflow (69 runs of
-    the same 130 columns spread over ~130K columns: 130 buckets of 69 equal keys).  The overflow flag
-    of the bucket scan must not wrap; the row takes the fallback and matches the oracle."""
-    k, run = 69, 130
+@pytest.mark.parametrize("k,run", [(69, 130), (140, 60)])
+def test_limited_bucket_overflow_many_heavy_buckets(k, run):
+    """one limited row made of k runs of the same `run` columns spread
+    over ~130K columns: `run` buckets of k equal keys.  (69, 130): 130 heavy buckets below the
+    overflow threshold (kBucketMax = 127), ranked by their sort codes; (140, 60): 60 buckets above it
+    -- the overflow flag of the bucket scan must not wrap and the row takes the fallback.  Both match
+    the oracle."""
     cols = np.sort(np.random.default_rng(4).choice(130_000, run, replace=False)).astype(np.int32)
     br = np.repeat(np.arange(k, dtype=np.int32), run)
     bc = np.tile(cols, k)
@@ -492,7 +494,7 @@ def test_limited_bucket_overflow_many_heavy_buckets():
     A, B = spg.from_inputs(inp, "cuda")
     for opts in ({}, TILES):
         with spg.Plan(A, B, **opts) as p:
-            assert p.stats()["n_rows_bin"][5] == 1   # the row is B-Limited (9108 padded slots)
+            assert p.stats()["n_rows_bin"][5] == 1   # the row is B-Limited (9384 / 8960 padded slots)
             C = p.execute()
         assert_c_matches(C, inp)
 
